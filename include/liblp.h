@@ -1,0 +1,198 @@
+/*
+ * liblp.h -- C ABI of the B200-native Lazy Persistency (LP) hot path.
+ *
+ * Method: Yudha, Kimura, Zhou, Solihin, "Scalable and Fast Lazy Persistency on
+ * GPUs", IISWC 2020.  Citations are PAPER.md line numbers L<n> + section.
+ * Readings of passages the paper leaves open are DESIGN.md R1..R20.
+ *
+ *   lp_config          ~ "#pragma nvm lpcuda_init(tab, nelems, selem)" and the
+ *                        checksum type of "lpcuda_checksum(type, tab, key..)"
+ *                        (L357, L526-538, §VI)
+ *   lp_cksum_init      table initialisation before the protected kernel (L528)
+ *   lp_run_protected   the LP region kernel: region body + checksum epilogue +
+ *                      lock-free store into the hash-table-less checksum array
+ *                      indexed by region id (L181 §IV-A, L192 §IV-B,
+ *                      L220-258 Listings 3-4, L349 §V)
+ *   lp_validate        recovery-kernel validation: recompute each region's
+ *                      checksum from the output, compare with the table,
+ *                      compact the failed region ids (L183 §IV-A)
+ *   lp_recover         re-execute only the failed regions (idempotent region =
+ *                      the original body, L183)
+ *
+ * Conventions (all calls):
+ *  - Every call returns lp_status; nothing throws across the ABI.  On error a
+ *    thread-local message is available from lp_last_error().
+ *  - Ownership: the caller owns every buffer.  Device buffers (out, cksum,
+ *    failed_list, d_n_failed, workspace, rids, stale, records, workload a/b)
+ *    are device pointers on cfg.device, allocated by the caller (torch in the
+ *    Python binding).  liblp never allocates or frees device memory; the
+ *    handle owns only host state.
+ *  - Asynchrony: every device-side operation is enqueued on `stream` (a
+ *    cudaStream_t passed as void*; NULL = legacy default stream) and the call
+ *    returns without synchronising.  Counts live in device memory (int64) so
+ *    recovery and NCCL can consume them without a host round trip.
+ *  - Argument errors are reported synchronously (LP_ERR_INVALID_ARG) before
+ *    anything is enqueued: NULL pointers, M % region_m or N % region_n != 0,
+ *    region_n*es % 16 != 0, pointers not 16-byte aligned, failed_cap < R,
+ *    unsupported dtype / workload combinations (LP_ERR_UNSUPPORTED), a device
+ *    that is not sm_100 (LP_ERR_UNSUPPORTED).  Launch failures return
+ *    LP_ERR_CUDA.  Device-side hash-table exhaustion is reported by lp_stats.
+ *  - Region ids are GLOBAL: rid = (row_offset/region_m + p) * (n/region_n) + q
+ *    for region (p, q) of this shard (Listing 6 keys (blockIdx.x, blockIdx.y),
+ *    L553, linearised row-major: Reading R9), so row shards produce disjoint
+ *    id ranges.  The array store indexes the caller's table slice with the
+ *    LOCAL rid (rid - rid_offset); hash stores key on the global rid.
+ */
+#ifndef LIBLP_H_
+#define LIBLP_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#if defined(__GNUC__)
+#define LP_API __attribute__((visibility("default")))
+#else
+#define LP_API
+#endif
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  LP_OK = 0,
+  LP_ERR_INVALID_ARG = 1,
+  LP_ERR_UNSUPPORTED = 2,
+  LP_ERR_CUDA = 3,
+  LP_ERR_CAPACITY = 4,
+  LP_ERR_STATE = 5
+} lp_status;
+
+/* Checksum types, OR-able (L192: parity = XOR of store values, modular = sum
+ * of store values, Adler-32; the paper recommends MOD|XOR, L585).  0 builds
+ * the unprotected twin of the same kernel (the overhead denominator). */
+typedef enum { LP_CK_NONE = 0u, LP_CK_MOD = 1u, LP_CK_XOR = 2u, LP_CK_ADLER32 = 4u } lp_cksum_bits;
+
+/* Checksum store.  ARRAY is the paper's hash-table-less global array indexed
+ * by region id (L349, §V).  QUAD_CAS is the lock-free quadratic-probing table
+ * (atomicCAS on the key slot, L267-272); QUAD_LOCK the same table with every
+ * insert inside one global spin lock (L81-83, L341 Table III, Reading R15). */
+typedef enum { LP_STORE_ARRAY = 0, LP_STORE_QUAD_CAS = 1, LP_STORE_QUAD_LOCK = 2 } lp_store;
+
+typedef enum { LP_F32 = 0, LP_BF16 = 1 } lp_dtype;
+
+/* Region bodies.  TMM = tiled matrix multiply (Listing 2, Listing 6
+ * L546-554), C = A*B, idempotent.  STENCIL5 = 5-point stencil, out-of-place
+ * (stand-in for the paper's bandwidth-bound class, Table I; Reading R19). */
+typedef enum { LP_WL_TMM = 0, LP_WL_STENCIL5 = 1 } lp_wl_kind;
+
+/* TMM body implementation: AUTO picks tcgen05 when the shape allows it. */
+typedef enum { LP_BODY_AUTO = 0, LP_BODY_SIMT = 1, LP_BODY_TCGEN05 = 2 } lp_body;
+
+/* Crash-injection modes (harness only; the paper has no crash model: Reading R11). */
+typedef enum {
+  LP_INJ_STALE_WORDS = 0,  /* a seeded run of m in [1, words] words reverts to the stale image */
+  LP_INJ_STALE_REGION = 1, /* the whole region reverts to the stale image */
+  LP_INJ_BITFLIP = 2,      /* one seeded bit of one seeded word flips */
+  LP_INJ_STALE_RECORD = 3  /* the region's record reverts to the sentinel; data intact */
+} lp_inject_mode;
+
+typedef void* lp_stream_t; /* cudaStream_t */
+
+typedef struct {
+  int32_t region_m, region_n; /* region shape in output elements (L79 granularity trade-off) */
+  uint32_t cksum;             /* OR of lp_cksum_bits; 0 = unprotected twin */
+  int32_t store;              /* lp_store */
+  int32_t device;             /* CUDA device ordinal */
+  int32_t body;               /* lp_body */
+  uint32_t hash_seed;         /* seed of the hash function for QUAD stores (Reading R14) */
+  int32_t reserved;
+} lp_config_t;
+
+typedef struct {
+  int32_t kind;      /* lp_wl_kind */
+  int32_t in_dtype;  /* lp_dtype of a / b */
+  int32_t out_dtype; /* lp_dtype of out */
+  int32_t reserved;
+  int64_t m, n, k;   /* TMM: out[m,n] = a[m,k] * b[k,n].  STENCIL5: m = rows of this shard, n = W, k unused */
+  const void* a;     /* TMM A (row-major, pitch lda elements) / STENCIL5 input (pitch lda) */
+  int64_t lda;
+  const void* b;     /* TMM B (row-major [k, n], pitch ldb elements); unused for STENCIL5 */
+  int64_t ldb;
+  int64_t ldc;       /* out row pitch in elements */
+  int64_t row_offset, global_m; /* shard: rows [row_offset, row_offset+m) of global_m.
+                                   STENCIL5 requires row_offset = 0, global_m = m. */
+} lp_workload_t;
+
+typedef struct lp_ctx* lp_handle;
+
+/* Create a handle for one region shape + checksum type + store. No CUDA call. */
+LP_API lp_status lp_config(const lp_config_t* cfg, lp_handle* out);
+LP_API lp_status lp_destroy(lp_handle h);
+
+/* R = (m/region_m) * (n/region_n): regions of this shard (L537: nelems = grid.x*grid.y). */
+LP_API lp_status lp_num_regions(lp_handle h, const lp_workload_t* wl, int64_t* r);
+
+/* Bytes of the checksum buffer.  ARRAY: R * 4 * selem (selem = popcount(cksum),
+ * L528 "number of checksums in an element").  QUAD_*: 64-byte header + cap *
+ * 4 * (1 + selem) with cap = smallest prime >= ceil(R / 0.7) (L267 load <= 70%). */
+LP_API lp_status lp_cksum_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
+
+/* Bytes of the scratch `workspace` lp_validate needs (flags + scan counters). */
+LP_API lp_status lp_workspace_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
+
+/* Fill the table with the sentinel 0xFFFFFFFF (Reading R8; hash: all keys empty,
+ * collision counter and error flag zero). */
+LP_API lp_status lp_cksum_init(lp_handle h, const lp_workload_t* wl, void* cksum, lp_stream_t stream);
+
+/* The LP-protected region kernel: computes out = body(wl) and, in the same
+ * kernel, stores one record per region into cksum (no second pass over out).
+ * cfg.cksum == 0 runs the unprotected twin (cksum may be NULL). */
+LP_API lp_status lp_run_protected(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, lp_stream_t stream);
+
+/* Validation: recompute every region's record from `out`, compare with `cksum`
+ * (hash stores: lookup; an absent key counts as failed), write the failed
+ * GLOBAL rids in ascending order to failed_list[0 .. *d_n_failed) and the count
+ * to *d_n_failed (device int64).  failed_cap must be >= R.  workspace must hold
+ * lp_workspace_bytes bytes. */
+LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, const void* cksum, int64_t* failed_list,
+                      int64_t failed_cap, int64_t* d_n_failed, void* workspace, lp_stream_t stream);
+
+/* Selective re-execution (eager recovery, L85): re-runs the region body for
+ * exactly the regions in failed_list[0 .. *d_n_failed) (global rids of this
+ * shard), rewriting their data AND records.  The count is read on the device. */
+LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
+                     const int64_t* d_n_failed, lp_stream_t stream);
+
+/* Records of every region of `out` (uint32 [R][selem], order MOD, XOR, ADLER)
+ * without comparing -- for parity tests against the oracle. */
+LP_API lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,
+                              lp_stream_t stream);
+
+/* Crash injection (harness only): corrupt the n regions whose GLOBAL rids are
+ * in device array rids[0..n) according to `mode` (lp_inject_mode), using the
+ * stale image `stale` (same shape/pitch as out; may be NULL for BITFLIP and
+ * STALE_RECORD) and counter-based choices seeded by `seed`. */
+LP_API lp_status lp_inject(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const void* stale,
+                    const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed, lp_stream_t stream);
+
+/* Hash-store statistics: d_stats (device int64[2]) <- {collisions (sum over
+ * inserts of probes-1), error flag (1 = a probe sequence was exhausted)}.
+ * ARRAY store: {0, 0}. */
+LP_API lp_status lp_stats(lp_handle h, const lp_workload_t* wl, const void* cksum, int64_t* d_stats, lp_stream_t stream);
+
+/* Number of SMs / cached device properties are queried lazily; this returns
+ * the device's SM count (0 if no device). */
+LP_API int32_t lp_device_sm_count(lp_handle h);
+
+/* Thread-local text of the last error ("" if none). */
+LP_API const char* lp_last_error(void);
+
+/* ABI version (major*100 + minor). */
+LP_API int32_t lp_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LIBLP_H_ */

@@ -1,0 +1,411 @@
+// liblp.cu -- host side of the liblp C ABI (include/liblp.h): argument checks,
+// table sizing, dispatch of the region bodies / validation / compaction.
+//
+// lp_config ~ #pragma nvm lpcuda_init(tab, nelems, selem) + the checksum type
+// of lpcuda_checksum (L357, L526-538 §VI); lp_run_protected ~ the annotated
+// kernel (Listing 6); lp_validate + lp_recover ~ the generated
+// check-and-recovery code (Listing 7), in the validate -> compact ->
+// re-execute form (Reading R13).
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "liblp.h"
+#include "lp_device.cuh"
+#include "lp_internal.h"
+
+struct lp_ctx {
+  lp_config_t cfg;
+  uint32_t mask;
+  int selem;
+  int dev_checked;  // 0 = not yet, 1 = ok
+  int sm_count;
+};
+
+namespace {
+
+thread_local std::string g_err;
+
+lp_status fail(lp_status s, const char* fmt, ...) __attribute__((format(printf, 2, 3)));
+lp_status fail(lp_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+lp_status ok() {
+  g_err.clear();
+  return LP_OK;
+}
+
+lp_status cuda_fail(cudaError_t e, const char* where) {
+  return fail(LP_ERR_CUDA, "%s: %s", where, cudaGetErrorString(e));
+}
+
+int es_of(int32_t dt) { return dt == LP_BF16 ? 2 : 4; }
+
+bool is_prime(uint64_t n) {
+  if (n < 2) return false;
+  for (uint64_t d = 2; d * d <= n; ++d)
+    if (n % d == 0) return false;
+  return true;
+}
+
+uint32_t hash_cap(int64_t R) {
+  uint64_t c = (uint64_t)std::ceil((double)R / 0.7);
+  if (c < 2) c = 2;
+  while (!is_prime(c)) ++c;
+  return (uint32_t)c;
+}
+
+bool aligned16(const void* p) { return (((uintptr_t)p) & 15u) == 0; }
+
+// Checks shared by every call on a workload; fills the region geometry.
+lp_status check_wl(const lp_ctx* h, const lp_workload_t* wl, lp::RegionGeom* g) {
+  if (!h) return fail(LP_ERR_INVALID_ARG, "null handle");
+  if (!wl) return fail(LP_ERR_INVALID_ARG, "null workload");
+  if (wl->kind != LP_WL_TMM && wl->kind != LP_WL_STENCIL5) return fail(LP_ERR_INVALID_ARG, "unknown workload kind %d", wl->kind);
+  if ((wl->in_dtype != LP_F32 && wl->in_dtype != LP_BF16) || (wl->out_dtype != LP_F32 && wl->out_dtype != LP_BF16))
+    return fail(LP_ERR_INVALID_ARG, "unknown dtype");
+  if (wl->m <= 0 || wl->n <= 0) return fail(LP_ERR_INVALID_ARG, "m and n must be positive");
+  const int RM = h->cfg.region_m, RN = h->cfg.region_n;
+  if (wl->m % RM || wl->n % RN)
+    return fail(LP_ERR_INVALID_ARG, "m=%lld, n=%lld not divisible by the region %dx%d (Reading R17)", (long long)wl->m,
+                (long long)wl->n, RM, RN);
+  const int es = es_of(wl->out_dtype);
+  if (wl->ldc < wl->n) return fail(LP_ERR_INVALID_ARG, "ldc < n");
+  if ((wl->ldc * es) % 16) return fail(LP_ERR_INVALID_ARG, "ldc*es must be a multiple of 16 bytes");
+  if (wl->row_offset < 0 || wl->global_m < wl->row_offset + wl->m)
+    return fail(LP_ERR_INVALID_ARG, "shard rows [row_offset, row_offset+m) outside global_m");
+  if (wl->row_offset % RM) return fail(LP_ERR_INVALID_ARG, "row_offset not a multiple of region_m");
+  if (wl->kind == LP_WL_TMM) {
+    if (wl->k <= 0) return fail(LP_ERR_INVALID_ARG, "k must be positive");
+  } else {
+    if (wl->in_dtype != LP_F32 || wl->out_dtype != LP_F32) return fail(LP_ERR_UNSUPPORTED, "stencil is fp32 -> fp32");
+    if (wl->row_offset != 0 || wl->global_m != wl->m) return fail(LP_ERR_UNSUPPORTED, "stencil shards are not supported");
+  }
+  g->M = wl->m;
+  g->N = wl->n;
+  g->ldc = wl->ldc;
+  g->es = es;
+  g->RM = RM;
+  g->RN = RN;
+  g->P = wl->m / RM;
+  g->Q = wl->n / RN;
+  g->R = g->P * g->Q;
+  g->rid_offset = (wl->row_offset / RM) * g->Q;
+  if (g->rid_offset + g->R > (int64_t)0xFFFFFFFEll && h->cfg.store != LP_STORE_ARRAY)
+    return fail(LP_ERR_UNSUPPORTED, "hash stores key on 32-bit rids");
+  return LP_OK;
+}
+
+lp_status check_device(lp_ctx* h) {
+  if (h->dev_checked) return LP_OK;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev <= h->cfg.device) {
+    cudaGetLastError();
+    return fail(LP_ERR_UNSUPPORTED, "no CUDA device %d (%s)", h->cfg.device, cudaGetErrorString(e));
+  }
+  cudaDeviceProp prop;
+  e = cudaGetDeviceProperties(&prop, h->cfg.device);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceProperties");
+  if (prop.major != 10 || prop.minor != 0)
+    return fail(LP_ERR_UNSUPPORTED, "liblp is built for sm_100a; device %d is sm_%d%d", h->cfg.device, prop.major,
+                prop.minor);
+  h->sm_count = prop.multiProcessorCount;
+  h->dev_checked = 1;
+  return LP_OK;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+lp::HashInfo hash_info(const lp_ctx* h, const lp::RegionGeom& g) {
+  lp::HashInfo hi;
+  hi.store = h->cfg.store;
+  hi.cap = h->cfg.store == LP_STORE_ARRAY ? 0u : hash_cap(g.R);
+  hi.seed = h->cfg.hash_seed;
+  return hi;
+}
+
+size_t cksum_bytes(const lp_ctx* h, const lp::RegionGeom& g) {
+  if (h->cfg.store == LP_STORE_ARRAY) return (size_t)g.R * 4u * (size_t)h->selem;
+  return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R) * 4u * (size_t)(1 + h->selem);
+}
+
+size_t workspace_bytes(const lp::RegionGeom& g) {
+  const size_t flags = ((size_t)g.R + 255) & ~(size_t)255;
+  return flags + lp::compact_scratch_bytes(g.R) + 256;
+}
+
+// Body dispatch shared by run_protected and recover (list = null for a full run).
+lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
+                   const int64_t* list, const int64_t* d_n, cudaStream_t st) {
+  const lp::HashInfo hi = hash_info(h, g);
+  if (wl->kind == LP_WL_STENCIL5) {
+    if (!lp::stencil_supported(g.RM, g.RN)) return fail(LP_ERR_UNSUPPORTED, "stencil supports 128x128 regions");
+    if (!wl->a) return fail(LP_ERR_INVALID_ARG, "null stencil input");
+    if (!aligned16(wl->a) || !aligned16(out) || (wl->lda * 4) % 16) return fail(LP_ERR_INVALID_ARG, "stencil buffers must be 16-B aligned");
+    if (wl->lda < wl->n) return fail(LP_ERR_INVALID_ARG, "lda < n");
+    lp::StencilArgs a;
+    a.in = (const float*)wl->a;
+    a.ldi = wl->lda;
+    a.out = (float*)out;
+    a.ldo = wl->ldc;
+    a.H = wl->m;
+    a.W = wl->n;
+    a.RM = g.RM;
+    a.RN = g.RN;
+    a.mask = h->mask;
+    a.hash = hi;
+    a.ck = (uint32_t*)ck;
+    a.rid_offset = g.rid_offset;
+    a.list = list;
+    a.d_n = d_n;
+    a.sm_count = h->sm_count;
+    cudaError_t e = lp::launch_stencil(a, st);
+    return e == cudaSuccess ? ok() : cuda_fail(e, "stencil launch");
+  }
+  if (!wl->a || !wl->b) return fail(LP_ERR_INVALID_ARG, "null A or B");
+  if (wl->lda < wl->k || wl->ldb < wl->n) return fail(LP_ERR_INVALID_ARG, "lda < k or ldb < n");
+  lp::TmmArgs a;
+  a.A = wl->a;
+  a.lda = wl->lda;
+  a.B = wl->b;
+  a.ldb = wl->ldb;
+  a.C = out;
+  a.ldc = wl->ldc;
+  a.M = wl->m;
+  a.N = wl->n;
+  a.K = wl->k;
+  a.in_bf16 = wl->in_dtype == LP_BF16;
+  a.out_bf16 = wl->out_dtype == LP_BF16;
+  a.RM = g.RM;
+  a.RN = g.RN;
+  a.mask = h->mask;
+  a.hash = hi;
+  a.ck = (uint32_t*)ck;
+  a.rid_offset = g.rid_offset;
+  a.list = list;
+  a.d_n = d_n;
+  a.sm_count = h->sm_count;
+  const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
+                                          wl->a, wl->b, out);
+  int body = h->cfg.body;
+  if (body == LP_BODY_AUTO) body = tc_ok ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
+  if (body == LP_BODY_TCGEN05) {
+    if (!tc_ok)
+      return fail(LP_ERR_UNSUPPORTED,
+                  "tcgen05 body needs bf16 input, m%%128 == 0, n%%256 == 0, k%%64 == 0, region 128x128 or 32x32 "
+                  "dividing the 128x256 tile, 16-B aligned pitches");
+    const char* why = nullptr;
+    cudaError_t e = lp::launch_tmm_tc(a, st, &why);
+    if (e != cudaSuccess) return why ? fail(LP_ERR_CUDA, "tcgen05 launch: %s", why) : cuda_fail(e, "tcgen05 launch");
+    return ok();
+  }
+  if (!lp::tmm_simt_supported(g.RM, g.RN, a.in_bf16, a.out_bf16))
+    return fail(LP_ERR_UNSUPPORTED, "SIMT body supports 32x32, 64x64 and 128x128 regions");
+  if (wl->k % 16) return fail(LP_ERR_UNSUPPORTED, "SIMT body needs k %% 16 == 0");
+  cudaError_t e = lp::launch_tmm_simt(a, st);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "SIMT TMM launch");
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t lp_abi_version(void) { return 100; }
+
+const char* lp_last_error(void) { return g_err.c_str(); }
+
+lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
+  if (!cfg || !out) return fail(LP_ERR_INVALID_ARG, "null argument");
+  *out = nullptr;
+  if (cfg->region_m <= 0 || cfg->region_n <= 0) return fail(LP_ERR_INVALID_ARG, "region shape must be positive");
+  if (cfg->cksum & ~7u) return fail(LP_ERR_INVALID_ARG, "unknown checksum bits 0x%x", cfg->cksum);
+  if (cfg->store < LP_STORE_ARRAY || cfg->store > LP_STORE_QUAD_LOCK) return fail(LP_ERR_INVALID_ARG, "unknown store %d", cfg->store);
+  if (cfg->store != LP_STORE_ARRAY && cfg->cksum == 0) return fail(LP_ERR_INVALID_ARG, "a hash store needs a checksum");
+  if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
+  if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
+  if ((int64_t)cfg->region_m * cfg->region_n * 4 > (16ll << 20))
+    return fail(LP_ERR_UNSUPPORTED, "regions larger than 16 MiB are not supported");
+  lp_ctx* h = new lp_ctx();
+  h->cfg = *cfg;
+  h->mask = cfg->cksum;
+  h->selem = lp::selem_of(cfg->cksum);
+  h->dev_checked = 0;
+  h->sm_count = 0;
+  *out = h;
+  return ok();
+}
+
+lp_status lp_destroy(lp_handle h) {
+  delete h;
+  return ok();
+}
+
+int32_t lp_device_sm_count(lp_handle h) {
+  if (!h) return 0;
+  if (check_device(h) != LP_OK) return 0;
+  return h->sm_count;
+}
+
+lp_status lp_num_regions(lp_handle h, const lp_workload_t* wl, int64_t* r) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!r) return fail(LP_ERR_INVALID_ARG, "null output");
+  *r = g.R;
+  return ok();
+}
+
+lp_status lp_cksum_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!bytes) return fail(LP_ERR_INVALID_ARG, "null output");
+  *bytes = cksum_bytes(h, g);
+  return ok();
+}
+
+lp_status lp_workspace_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!bytes) return fail(LP_ERR_INVALID_ARG, "null output");
+  *bytes = workspace_bytes(g);
+  return ok();
+}
+
+lp_status lp_cksum_init(lp_handle h, const lp_workload_t* wl, void* cksum, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (h->mask == 0) return ok();  // unprotected twin: no table
+  if (!cksum) return fail(LP_ERR_INVALID_ARG, "null cksum");
+  if (!aligned16(cksum)) return fail(LP_ERR_INVALID_ARG, "cksum must be 16-B aligned");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e = lp::launch_cksum_init(cksum, cksum_bytes(h, g), hash_info(h, g), (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "cksum init");
+}
+
+lp_status lp_run_protected(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!out) return fail(LP_ERR_INVALID_ARG, "null out");
+  if (!aligned16(out)) return fail(LP_ERR_INVALID_ARG, "out must be 16-B aligned");
+  if (h->mask && !cksum) return fail(LP_ERR_INVALID_ARG, "null cksum");
+  if (h->mask && !aligned16(cksum)) return fail(LP_ERR_INVALID_ARG, "cksum must be 16-B aligned");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  return run_body(h, wl, g, out, cksum, nullptr, nullptr, (cudaStream_t)stream);
+}
+
+lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, const void* cksum, int64_t* failed_list,
+                      int64_t failed_cap, int64_t* d_n_failed, void* workspace, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (h->mask == 0) return fail(LP_ERR_STATE, "validation needs a checksum (cfg.cksum != 0)");
+  if (!out || !cksum || !failed_list || !d_n_failed || !workspace) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (failed_cap < g.R) return fail(LP_ERR_INVALID_ARG, "failed_cap %lld < R %lld", (long long)failed_cap, (long long)g.R);
+  if (!aligned16(out) || !aligned16(cksum) || !aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "buffers must be 16-B aligned");
+  if ((g.RN * g.es) % 16) return fail(LP_ERR_INVALID_ARG, "region_n*es must be a multiple of 16 bytes");
+  {
+    const int cpr = g.RN * g.es / 16;
+    if (cpr & (cpr - 1)) return fail(LP_ERR_UNSUPPORTED, "region_n*es/16 must be a power of two");
+  }
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  uint8_t* flags = (uint8_t*)workspace;
+  uint32_t* counts = (uint32_t*)((uint8_t*)workspace + (((size_t)g.R + 255) & ~(size_t)255));
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st);
+  if (e != cudaSuccess) return cuda_fail(e, "validate launch");
+  e = lp::launch_compact(g, flags, counts, failed_list, d_n_failed, st);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "compact launch");
+}
+
+lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
+                     const int64_t* d_n_failed, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!out || !failed_list || !d_n_failed) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (h->mask && !cksum) return fail(LP_ERR_INVALID_ARG, "null cksum");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  return run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream);
+}
+
+lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,
+                              lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (h->mask == 0) return fail(LP_ERR_STATE, "records need a checksum (cfg.cksum != 0)");
+  if (!out || !records) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (!aligned16(out)) return fail(LP_ERR_INVALID_ARG, "out must be 16-B aligned");
+  {
+    const int cpr = g.RN * g.es / 16;
+    if ((g.RN * g.es) % 16 || (cpr & (cpr - 1))) return fail(LP_ERR_UNSUPPORTED, "region_n*es/16 must be a power of two");
+  }
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e =
+      lp::launch_validate(g, h->mask, hash_info(h, g), out, nullptr, nullptr, records, h->sm_count, (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "records launch");
+}
+
+lp_status lp_inject(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const void* stale,
+                    const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (mode > LP_INJ_STALE_RECORD) return fail(LP_ERR_INVALID_ARG, "unknown injection mode %u", mode);
+  if (n < 0 || n > g.R) return fail(LP_ERR_INVALID_ARG, "n outside [0, R]");
+  if (n == 0) return ok();
+  if (!out || !rids) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if ((mode == LP_INJ_STALE_WORDS || mode == LP_INJ_STALE_REGION) && !stale)
+    return fail(LP_ERR_INVALID_ARG, "stale image required for this mode");
+  if (mode == LP_INJ_STALE_RECORD && (h->mask == 0 || !cksum)) return fail(LP_ERR_INVALID_ARG, "STALE_RECORD needs a table");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e = lp::launch_inject(g, h->mask, hash_info(h, g), out, cksum, stale, rids, n, mode, seed,
+                                    (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "inject launch");
+}
+
+lp_status lp_stats(lp_handle h, const lp_workload_t* wl, const void* cksum, int64_t* d_stats, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!d_stats) return fail(LP_ERR_INVALID_ARG, "null d_stats");
+  if (h->cfg.store != LP_STORE_ARRAY && !cksum) return fail(LP_ERR_INVALID_ARG, "null cksum");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e = lp::launch_stats(hash_info(h, g), cksum, d_stats, (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "stats launch");
+}
+
+}  // extern "C"

@@ -1,0 +1,258 @@
+// lp_device.cuh -- device-side LP building blocks shared by every CUDA kernel of liblp.
+//
+//  * per-thread checksum partials over the exact 32-bit words a kernel stores
+//    (L192 §IV-B: parity = XOR, modular = sum, Adler-32; L260-261 Fig. 2: the
+//    float's raw bits are the word -- Readings R1, R2, R5, R6);
+//  * warp reduction with one redux.sync per checksum (the B200 form of
+//    Listing 4's shfl_down ladder, L244-258) and the block combine through a
+//    small shared array (Listing 3);
+//  * the lock-free record store into the hash-table-less array (L349 §V) and
+//    the hash-store ablation (L265-274, L341).
+//
+// Adler-32 uses the order-free closed form so the partials can be reduced in
+// any order: for region bytes d_1..d_n,
+//   A = (1 + S) mod 65521,  B = (n + (n+1) S - W) mod 65521,
+//   S = sum d_i,  W = sum i*d_i.
+// Each 32-bit word at 1-based byte position p contributes S += dp4a(w, 1111),
+// W += p*dp4a(w,1111) + dp4a(w, 0x03020100).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace lp {
+
+constexpr uint32_t kMod = 1u, kXor = 2u, kAdler = 4u;
+constexpr uint32_t kAdlerBase = 65521u;
+constexpr uint32_t kSentinel = 0xFFFFFFFFu;
+constexpr uint32_t kEmptyKey = 0xFFFFFFFFu;
+
+__host__ __device__ constexpr int selem_of(uint32_t mask) {
+  return (int)((mask & 1u) + ((mask >> 1) & 1u) + ((mask >> 2) & 1u));
+}
+
+// Per-thread partials.  MASK is a compile-time checksum set so the unprotected
+// twin (MASK = 0) compiles to exactly the body.
+template <uint32_t MASK>
+struct CkPartial {
+  uint32_t mod = 0, xr = 0, s = 0;
+  uint64_t w = 0;
+
+  // word: the stored 32-bit pattern; pos: 1-based byte position of its first
+  // byte inside the region's byte stream (only used by Adler).
+  __device__ __forceinline__ void add(uint32_t word, uint32_t pos) {
+    if constexpr ((MASK & kMod) != 0) mod += word;
+    if constexpr ((MASK & kXor) != 0) xr ^= word;
+    if constexpr ((MASK & kAdler) != 0) {
+      const uint32_t bs = (uint32_t)__dp4a(word, 0x01010101u, 0u);
+      const uint32_t ws = (uint32_t)__dp4a(word, 0x03020100u, 0u);
+      s += bs;
+      w += (uint64_t)pos * bs + ws;
+    }
+  }
+  __device__ __forceinline__ void merge(const CkPartial& o) {
+    mod += o.mod;
+    xr ^= o.xr;
+    s += o.s;
+    w += o.w;
+  }
+};
+
+// Reduced record of one region (the value every lane holds after warp_reduce).
+struct CkRecord {
+  uint32_t mod, xr, s, wmod;  // s = byte sum (exact), wmod = W mod 65521
+};
+
+template <uint32_t MASK>
+__device__ __forceinline__ CkRecord warp_reduce(const CkPartial<MASK>& p, uint32_t lanes = 0xFFFFFFFFu) {
+  CkRecord r{0u, 0u, 0u, 0u};
+  if constexpr ((MASK & kMod) != 0) r.mod = __reduce_add_sync(lanes, p.mod);
+  if constexpr ((MASK & kXor) != 0) r.xr = __reduce_xor_sync(lanes, p.xr);
+  if constexpr ((MASK & kAdler) != 0) {
+    r.s = __reduce_add_sync(lanes, p.s);
+    r.wmod = __reduce_add_sync(lanes, (uint32_t)(p.w % kAdlerBase));
+  }
+  return r;
+}
+
+__device__ __forceinline__ CkRecord combine(CkRecord a, const CkRecord& b) {
+  a.mod += b.mod;
+  a.xr ^= b.xr;
+  a.s += b.s;
+  a.wmod = (a.wmod % kAdlerBase) + (b.wmod % kAdlerBase);
+  return a;
+}
+
+// Final Adler-32 value of a region of nbytes bytes from (S, W mod 65521).
+__device__ __forceinline__ uint32_t adler_finish(uint32_t s, uint32_t wmod, uint64_t nbytes) {
+  const uint64_t P = kAdlerBase;
+  const uint64_t a = (1ull + s) % P;
+  const uint64_t n = nbytes % P, n1 = (nbytes + 1) % P;
+  const uint64_t b = (n + (n1 * (s % P)) % P + P - (wmod % P)) % P;
+  return (uint32_t)((b << 16) | a);
+}
+
+// Record words in the fixed order MOD, XOR, ADLER (Reading R7).
+template <uint32_t MASK>
+__device__ __forceinline__ int record_words(const CkRecord& r, uint64_t nbytes, uint32_t* out3) {
+  int k = 0;
+  if constexpr ((MASK & kMod) != 0) out3[k++] = r.mod;
+  if constexpr ((MASK & kXor) != 0) out3[k++] = r.xr;
+  if constexpr ((MASK & kAdler) != 0) out3[k++] = adler_finish(r.s, r.wmod, nbytes);
+  return k;
+}
+
+// ---------------------------------------------------------------------------
+// Stores.  Array store (L349): one plain store per region into
+// table[local_rid * selem], no atomics and no fences (lazy persist, L55).
+template <uint32_t MASK>
+__device__ __forceinline__ void store_array(uint32_t* table, int64_t local_rid, const uint32_t* w) {
+  constexpr int S = selem_of(MASK);
+  uint32_t* dst = table + local_rid * S;
+  if constexpr (S == 1) {
+    dst[0] = w[0];
+  } else if constexpr (S == 2) {
+    if ((((uintptr_t)dst) & 7u) == 0) {
+      *reinterpret_cast<uint2*>(dst) = make_uint2(w[0], w[1]);
+    } else {
+      dst[0] = w[0];
+      dst[1] = w[1];
+    }
+  } else if constexpr (S == 3) {
+    dst[0] = w[0];
+    dst[1] = w[1];
+    dst[2] = w[2];
+  }
+}
+
+// Hash-store layout inside the caller's cksum buffer (Reading R14):
+//   [0]  u32 cap      [1] u32 seed     [2] u32 lock word   [3] u32 error flag
+//   [4..5] u64 collisions (sum of probes-1)       [6..15] reserved
+//   then cap entries of (1 + selem) u32: key (0xFFFFFFFF = empty), record.
+struct HashHeader {
+  uint32_t cap, seed, lock, error;
+  unsigned long long collisions;
+  uint32_t reserved[10];
+};
+static_assert(sizeof(HashHeader) == 64, "hash header is 64 bytes");
+
+__host__ __device__ __forceinline__ uint32_t hash_fmix32(uint32_t key, uint32_t seed) {
+  uint32_t h = key ^ seed;
+  h ^= h >> 16;
+  h *= 0x85ebca6bu;
+  h ^= h >> 13;
+  h *= 0xc2b2ae35u;
+  h ^= h >> 16;
+  return h;
+}
+
+// Lock-free insert (L272: atomicCAS on the key slot makes sure the entry is
+// empty before inserting; probe i visits home + i^2, L267).  Called by ONE
+// thread per region.  Returns the number of probes.
+template <uint32_t MASK>
+__device__ uint32_t quad_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+  constexpr int S = selem_of(MASK);
+  HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
+  uint32_t* ent = ckbuf + sizeof(HashHeader) / 4;
+  const uint32_t cap = hdr->cap;
+  const uint32_t home = hash_fmix32(rid, hdr->seed) % cap;
+  for (uint32_t i = 0; i < cap; ++i) {
+    const uint32_t slot = (uint32_t)(((uint64_t)home + (uint64_t)i * i) % cap);
+    uint32_t* e = ent + (uint64_t)slot * (1 + S);
+    const uint32_t prev = atomicCAS(e, kEmptyKey, rid);
+    if (prev == kEmptyKey || prev == rid) {
+#pragma unroll
+      for (int s = 0; s < S; ++s) e[1 + s] = w[s];
+      if (i) atomicAdd(&hdr->collisions, (unsigned long long)i);
+      return i + 1;
+    }
+  }
+  atomicExch(&hdr->error, 1u);
+  return 0;
+}
+
+// Lock-based variant (L81-83 CPU style; L341 "lock-based"): the whole probe +
+// insert runs inside one global spin lock (Reading R15).
+template <uint32_t MASK>
+__device__ uint32_t quad_insert_locked(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+  constexpr int S = selem_of(MASK);
+  HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
+  uint32_t* ent = ckbuf + sizeof(HashHeader) / 4;
+  while (atomicCAS(&hdr->lock, 0u, 1u) != 0u) {
+    __nanosleep(32);
+  }
+  __threadfence();
+  const uint32_t cap = *((volatile uint32_t*)&hdr->cap);
+  const uint32_t home = hash_fmix32(rid, hdr->seed) % cap;
+  uint32_t probes = 0;
+  for (uint32_t i = 0; i < cap; ++i) {
+    const uint32_t slot = (uint32_t)(((uint64_t)home + (uint64_t)i * i) % cap);
+    volatile uint32_t* e = ent + (uint64_t)slot * (1 + S);
+    const uint32_t k = e[0];
+    if (k == kEmptyKey || k == rid) {
+      e[0] = rid;
+#pragma unroll
+      for (int s = 0; s < S; ++s) e[1 + s] = w[s];
+      if (i) hdr->collisions += i;
+      probes = i + 1;
+      break;
+    }
+  }
+  if (!probes) hdr->error = 1u;
+  __threadfence();
+  atomicExch(&hdr->lock, 0u);
+  return probes;
+}
+
+// Lookup used by validation (L270: lookups are off the critical path).
+// Returns true and the stored record words if rid is present.
+template <int S>
+__device__ __forceinline__ bool quad_lookup(const uint32_t* ckbuf, uint32_t rid, uint32_t* w) {
+  const HashHeader* hdr = reinterpret_cast<const HashHeader*>(ckbuf);
+  const uint32_t* ent = ckbuf + sizeof(HashHeader) / 4;
+  const uint32_t cap = hdr->cap;
+  const uint32_t home = hash_fmix32(rid, hdr->seed) % cap;
+  for (uint32_t i = 0; i < cap; ++i) {
+    const uint32_t slot = (uint32_t)(((uint64_t)home + (uint64_t)i * i) % cap);
+    const uint32_t* e = ent + (uint64_t)slot * (1 + S);
+    const uint32_t k = e[0];
+    if (k == rid) {
+#pragma unroll
+      for (int s = 0; s < S; ++s) w[s] = e[1 + s];
+      return true;
+    }
+    if (k == kEmptyKey) return false;
+  }
+  return false;
+}
+
+// Dispatch of the record store on the runtime store kind.
+template <uint32_t MASK>
+__device__ __forceinline__ void store_record(uint32_t* ck, int store, int64_t local_rid, uint32_t global_rid,
+                                             const uint32_t* w) {
+  if (store == 0) {
+    store_array<MASK>(ck, local_rid, w);
+  } else if (store == 1) {
+    quad_insert<MASK>(ck, global_rid, w);
+  } else {
+    quad_insert_locked<MASK>(ck, global_rid, w);
+  }
+}
+
+// Streaming 16-byte load that does not allocate in L1 (validate reads `out` once).
+__device__ __forceinline__ uint4 ld_stream_u4(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ uint64_t mix64(uint64_t z) {
+  z += 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+}  // namespace lp

@@ -1,0 +1,85 @@
+// lp_internal.h -- launcher interface between the liblp host API (liblp.cu) and
+// the kernel translation units.  Not part of the public ABI (include/liblp.h).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace lp {
+
+// Geometry of one output matrix split into regions.
+struct RegionGeom {
+  int64_t M, N;        // output rows / cols of this shard
+  int64_t ldc;         // row pitch in elements
+  int es;              // element size (bytes)
+  int RM, RN;          // region shape (elements)
+  int64_t P, Q, R;     // region rows, region cols, regions
+  int64_t rid_offset;  // global rid of local region 0
+};
+
+struct HashInfo {
+  int store;      // 0 array, 1 quad CAS, 2 quad lock
+  uint32_t cap;   // hash capacity (0 for array)
+  uint32_t seed;
+};
+
+// ---- lp_kernels.cu
+cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaStream_t st);
+cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
+                            uint8_t* flags, uint32_t* records /* non-null => records mode */, int sm_count,
+                            cudaStream_t st);
+cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* block_counts, int64_t* list,
+                           int64_t* d_n, cudaStream_t st);
+size_t compact_scratch_bytes(int64_t R);
+cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi, void* out, void* ck,
+                          const void* stale, const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed,
+                          cudaStream_t st);
+cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
+
+// ---- tmm_simt.cu : SIMT region body (CTA tile == region), paper-shaped
+struct TmmArgs {
+  const void* A;
+  int64_t lda;
+  const void* B;
+  int64_t ldb;
+  void* C;
+  int64_t ldc;
+  int64_t M, N, K;
+  int in_bf16, out_bf16;
+  int RM, RN;
+  uint32_t mask;
+  HashInfo hash;
+  uint32_t* ck;
+  int64_t rid_offset;
+  const int64_t* list;  // list mode (recovery) when non-null
+  const int64_t* d_n;
+  int sm_count;
+};
+bool tmm_simt_supported(int RM, int RN, int in_bf16, int out_bf16);
+cudaError_t launch_tmm_simt(const TmmArgs& a, cudaStream_t st);
+
+// ---- tmm_tc.cu : tcgen05 / TMEM / TMA region body (bf16 in)
+bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int64_t lda, int64_t ldb,
+                      int64_t ldc, const void* A, const void* B, const void* C);
+cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why);
+
+// ---- stencil.cu : 5-point stencil region body
+struct StencilArgs {
+  const float* in;
+  int64_t ldi;
+  float* out;
+  int64_t ldo;
+  int64_t H, W;
+  int RM, RN;
+  uint32_t mask;
+  HashInfo hash;
+  uint32_t* ck;
+  int64_t rid_offset;
+  const int64_t* list;
+  const int64_t* d_n;
+  int sm_count;
+};
+bool stencil_supported(int RM, int RN);
+cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st);
+
+}  // namespace lp

@@ -1,0 +1,379 @@
+// lp_kernels.cu -- validation, compaction, table init, crash injection, stats.
+//
+// Validation is the recovery kernel's first half (L183 §IV-A): "fetching the
+// corresponding data from memory, computing their checksums, and then
+// comparing them with the ones stored in the checksum table".  On B200 it is an
+// HBM-streaming reduction: one warp per region, 16-byte non-allocating loads,
+// eight loads in flight per lane, one redux.sync per checksum.  The failed
+// regions are then compacted into an ascending list (Reading R12/R13) so that
+// recovery re-executes only those.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "lp_device.cuh"
+#include "lp_internal.h"
+
+namespace lp {
+namespace {
+
+constexpr int kValThreads = 256;
+constexpr int kValUnroll = 8;
+
+// One warp per region.  MODE 0 = compare with array table, 1 = compare with a
+// quad hash table (lookup by global rid), 2 = write records (no compare).
+template <uint32_t MASK, int MODE>
+__global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
+                                                                int64_t Q, int64_t R, int RM, int row_bytes,
+                                                                int cpr_log2, const uint32_t* __restrict__ ck,
+                                                                int64_t rid_offset, uint8_t* __restrict__ flags,
+                                                                uint32_t* __restrict__ records) {
+  constexpr int S = selem_of(MASK);
+  const int lane = threadIdx.x & 31;
+  const int64_t nwarps = (int64_t)gridDim.x * (kValThreads / 32);
+  const int cpr_mask = (1 << cpr_log2) - 1;
+  const int chunks = RM << cpr_log2;
+  const uint64_t nbytes = (uint64_t)RM * (uint64_t)row_bytes;
+  for (int64_t r = (int64_t)blockIdx.x * (kValThreads / 32) + (threadIdx.x >> 5); r < R; r += nwarps) {
+    const int64_t p = r / Q, q = r - p * Q;
+    const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
+    CkPartial<MASK> part;
+    for (int c0 = 0; c0 < chunks; c0 += 32 * kValUnroll) {
+      uint4 v[kValUnroll];
+#pragma unroll
+      for (int u = 0; u < kValUnroll; ++u) {
+        const int c = c0 + u * 32 + lane;
+        if (c < chunks) v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cpr_mask) << 4));
+      }
+#pragma unroll
+      for (int u = 0; u < kValUnroll; ++u) {
+        const int c = c0 + u * 32 + lane;
+        if (c < chunks) {
+          const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cpr_mask) << 4) + 1);
+          part.add(v[u].x, pos);
+          part.add(v[u].y, pos + 4);
+          part.add(v[u].z, pos + 8);
+          part.add(v[u].w, pos + 12);
+        }
+      }
+    }
+    const CkRecord rec = warp_reduce<MASK>(part);
+    if (lane == 0) {
+      uint32_t w[3];
+      record_words<MASK>(rec, nbytes, w);
+      if constexpr (MODE == 2) {
+#pragma unroll
+        for (int s = 0; s < S; ++s) records[r * S + s] = w[s];
+      } else if constexpr (MODE == 0) {
+        bool bad = false;
+#pragma unroll
+        for (int s = 0; s < S; ++s) bad |= (ck[r * S + s] != w[s]);
+        flags[r] = bad ? 1 : 0;
+      } else {
+        uint32_t stored[3];
+        bool bad = !quad_lookup<S>(ck, (uint32_t)(r + rid_offset), stored);
+#pragma unroll
+        for (int s = 0; s < S; ++s) bad |= (!bad && stored[s] != w[s]);
+        flags[r] = bad ? 1 : 0;
+      }
+    }
+  }
+}
+
+template <uint32_t MASK>
+cudaError_t validate_dispatch_mode(int mode, dim3 grid, cudaStream_t st, const uint8_t* out, int64_t ldc_bytes,
+                                   int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2, const uint32_t* ck,
+                                   int64_t rid_offset, uint8_t* flags, uint32_t* records) {
+  if (mode == 0)
+    validate_kernel<MASK, 0><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                           rid_offset, flags, records);
+  else if (mode == 1)
+    validate_kernel<MASK, 1><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                           rid_offset, flags, records);
+  else
+    validate_kernel<MASK, 2><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                           rid_offset, flags, records);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Ordered compaction: flags[R] -> ascending list of global rids + count.
+constexpr int kCompactThreads = 256;
+constexpr int kCompactPerThread = 32;  // two uint4 of flags
+constexpr int kCompactChunk = kCompactThreads * kCompactPerThread;
+
+__device__ __forceinline__ int count_flags_u4(uint4 v) {
+  // flags are 0/1 bytes
+  return __popc(v.x) + __popc(v.y) + __popc(v.z) + __popc(v.w);
+}
+
+__device__ __forceinline__ void load_flags(const uint8_t* flags, int64_t R, int64_t idx0, uint32_t f[8]) {
+  if (idx0 + kCompactPerThread <= R && ((((uintptr_t)(flags + idx0)) & 15u) == 0)) {
+    const uint4 a = *reinterpret_cast<const uint4*>(flags + idx0);
+    const uint4 b = *reinterpret_cast<const uint4*>(flags + idx0 + 16);
+    f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w;
+    f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      uint32_t w = 0;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int64_t k = idx0 + i * 4 + j;
+        if (k < R && flags[k]) w |= 1u << (8 * j);
+      }
+      f[i] = w;
+    }
+  }
+}
+
+__device__ __forceinline__ int block_exclusive_scan(int v, int* smem_warp, int* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) smem_warp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    int s = lane < kCompactThreads / 32 ? smem_warp[lane] : 0;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xFFFFFFFFu, s, o);
+      if (lane >= o) s += y;
+    }
+    if (lane < kCompactThreads / 32) smem_warp[lane] = s;  // inclusive
+  }
+  __syncthreads();
+  const int warp_off = wid ? smem_warp[wid - 1] : 0;
+  *total = smem_warp[kCompactThreads / 32 - 1];
+  return warp_off + x - v;
+}
+
+__global__ void __launch_bounds__(kCompactThreads) compact_count_kernel(const uint8_t* __restrict__ flags, int64_t R,
+                                                                        uint32_t* __restrict__ block_counts) {
+  __shared__ int warp_s[kCompactThreads / 32];
+  const int64_t idx0 = (int64_t)blockIdx.x * kCompactChunk + (int64_t)threadIdx.x * kCompactPerThread;
+  uint32_t f[8];
+  load_flags(flags, R, idx0, f);
+  int c = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) c += __popc(f[i]);
+  int total;
+  block_exclusive_scan(c, warp_s, &total);
+  if (threadIdx.x == 0) block_counts[blockIdx.x] = (uint32_t)total;
+}
+
+__global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const uint8_t* __restrict__ flags, int64_t R,
+                                                                          const uint32_t* __restrict__ block_counts,
+                                                                          int nblocks, int64_t rid_offset,
+                                                                          int64_t* __restrict__ list,
+                                                                          int64_t* __restrict__ d_n) {
+  __shared__ int warp_s[kCompactThreads / 32];
+  __shared__ long long s_base;
+  // base offset of this block = sum of the counts of the blocks before it
+  long long mine = 0, all = 0;
+  for (int b = threadIdx.x; b < nblocks; b += kCompactThreads) {
+    const long long c = block_counts[b];
+    all += c;
+    if (b < (int)blockIdx.x) mine += c;
+  }
+  {
+    // block-reduce two values through shuffles + smem
+    for (int o = 16; o > 0; o >>= 1) {
+      mine += __shfl_xor_sync(0xFFFFFFFFu, mine, o);
+      all += __shfl_xor_sync(0xFFFFFFFFu, all, o);
+    }
+    __shared__ long long red[2][kCompactThreads / 32];
+    if ((threadIdx.x & 31) == 0) {
+      red[0][threadIdx.x >> 5] = mine;
+      red[1][threadIdx.x >> 5] = all;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      long long m = 0, a = 0;
+      for (int w = 0; w < kCompactThreads / 32; ++w) {
+        m += red[0][w];
+        a += red[1][w];
+      }
+      s_base = m;
+      if (blockIdx.x == 0) *d_n = a;
+    }
+    __syncthreads();
+  }
+  const int64_t idx0 = (int64_t)blockIdx.x * kCompactChunk + (int64_t)threadIdx.x * kCompactPerThread;
+  uint32_t f[8];
+  load_flags(flags, R, idx0, f);
+  int c = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) c += __popc(f[i]);
+  int total;
+  const int off = block_exclusive_scan(c, warp_s, &total);
+  int64_t o = s_base + off;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      if ((f[i] >> (8 * j)) & 0xFFu) list[o++] = rid_offset + idx0 + i * 4 + j;
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------
+__global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed) {
+  HashHeader* h = reinterpret_cast<HashHeader*>(ck);
+  h->cap = cap;
+  h->seed = seed;
+  h->lock = 0;
+  h->error = 0;
+  h->collisions = 0ull;
+}
+
+__global__ void stats_kernel(const uint32_t* ck, int has_hash, int64_t* d_stats) {
+  if (has_hash) {
+    const HashHeader* h = reinterpret_cast<const HashHeader*>(ck);
+    d_stats[0] = (int64_t)h->collisions;
+    d_stats[1] = (int64_t)h->error;
+  } else {
+    d_stats[0] = 0;
+    d_stats[1] = 0;
+  }
+}
+
+// Crash injection (harness; Reading R11).  One block per injected region.
+template <int S>
+__global__ void inject_kernel(uint8_t* out, int64_t ldc_bytes, int64_t Q, int RM, int row_bytes,
+                              const uint8_t* stale, uint32_t* ck, int store, const int64_t* rids, int64_t rid_offset,
+                              uint32_t mode, uint64_t seed) {
+  const int64_t grid = rids[blockIdx.x];
+  const int64_t r = grid - rid_offset;
+  const int64_t p = r / Q, q = r - p * Q;
+  const int64_t base = p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
+  const int wpr = row_bytes / 4;
+  const int words = RM * wpr;
+  const uint64_t h = mix64(seed ^ (0xD1B54A32D192ED03ull * (uint64_t)(grid + 1)));
+  if (mode == 0 || mode == 1) {  // stale words / stale region
+    const int m = mode == 1 ? words : 1 + (int)(h % (uint64_t)words);
+    const int start = mode == 1 ? 0 : (int)((h >> 32) % (uint64_t)words);
+    for (int i = threadIdx.x; i < m; i += blockDim.x) {
+      const int wi = (start + i) % words;
+      const int64_t off = base + (int64_t)(wi / wpr) * ldc_bytes + (wi % wpr) * 4;
+      *reinterpret_cast<uint32_t*>(out + off) = *reinterpret_cast<const uint32_t*>(stale + off);
+    }
+  } else if (mode == 2) {  // bit flip
+    if (threadIdx.x == 0) {
+      const int wi = (int)(h % (uint64_t)words);
+      const int bit = (int)((h >> 40) & 31u);
+      const int64_t off = base + (int64_t)(wi / wpr) * ldc_bytes + (wi % wpr) * 4;
+      *reinterpret_cast<uint32_t*>(out + off) ^= (1u << bit);
+    }
+  } else {  // stale record
+    if (threadIdx.x == 0) {
+      if (store == 0) {
+        for (int s = 0; s < S; ++s) ck[r * S + s] = kSentinel;
+      } else {
+        const HashHeader* hdr = reinterpret_cast<const HashHeader*>(ck);
+        uint32_t* ent = ck + sizeof(HashHeader) / 4;
+        const uint32_t cap = hdr->cap;
+        const uint32_t home = hash_fmix32((uint32_t)grid, hdr->seed) % cap;
+        for (uint32_t i = 0; i < cap; ++i) {
+          const uint32_t slot = (uint32_t)(((uint64_t)home + (uint64_t)i * i) % cap);
+          uint32_t* e = ent + (uint64_t)slot * (1 + S);
+          if (e[0] == (uint32_t)grid) {
+            for (int s = 0; s < S; ++s) e[1 + s] = kSentinel;
+            break;
+          }
+          if (e[0] == kEmptyKey) break;
+        }
+      }
+    }
+  }
+}
+
+}  // namespace
+
+// ===========================================================================
+cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(ck, 0xFF, bytes, st);
+  if (e != cudaSuccess) return e;
+  if (hi.store != 0) {
+    hash_header_kernel<<<1, 1, 0, st>>>((uint32_t*)ck, hi.cap, hi.seed);
+    e = cudaGetLastError();
+  }
+  return e;
+}
+
+cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
+                            uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st) {
+  const int row_bytes = g.RN * g.es;
+  const int cpr = row_bytes / 16;
+  int cpr_log2 = 0;
+  while ((1 << cpr_log2) < cpr) ++cpr_log2;
+  const int64_t warps_needed = g.R;
+  int64_t blocks = (warps_needed + (kValThreads / 32) - 1) / (kValThreads / 32);
+  const int64_t cap_blocks = (int64_t)sm_count * 8;  // 8 x 256 threads = 2048 threads/SM
+  if (blocks > cap_blocks) blocks = cap_blocks;
+  if (blocks < 1) blocks = 1;
+  const int mode = records ? 2 : (hi.store == 0 ? 0 : 1);
+  const uint8_t* o = (const uint8_t*)out;
+  const int64_t ldcb = g.ldc * g.es;
+  dim3 grid((unsigned)blocks);
+  switch (mask) {
+#define LP_VCASE(M)                                                                                          \
+  case M:                                                                                                    \
+    return validate_dispatch_mode<M>(mode, grid, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,          \
+                                     (const uint32_t*)ck, g.rid_offset, flags, records);
+    LP_VCASE(1)
+    LP_VCASE(2)
+    LP_VCASE(3)
+    LP_VCASE(4)
+    LP_VCASE(5)
+    LP_VCASE(6)
+    LP_VCASE(7)
+#undef LP_VCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+}
+
+size_t compact_scratch_bytes(int64_t R) {
+  const int64_t nb = (R + kCompactChunk - 1) / kCompactChunk;
+  return (size_t)(nb > 0 ? nb : 1) * sizeof(uint32_t);
+}
+
+cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* block_counts, int64_t* list,
+                           int64_t* d_n, cudaStream_t st) {
+  int64_t nb = (g.R + kCompactChunk - 1) / kCompactChunk;
+  if (nb < 1) nb = 1;
+  compact_count_kernel<<<(unsigned)nb, kCompactThreads, 0, st>>>(flags, g.R, block_counts);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  compact_scatter_kernel<<<(unsigned)nb, kCompactThreads, 0, st>>>(flags, g.R, block_counts, (int)nb, g.rid_offset,
+                                                                   list, d_n);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi, void* out, void* ck,
+                          const void* stale, const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed,
+                          cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  const int S = selem_of(mask);
+  const int row_bytes = g.RN * g.es;
+#define LP_ICASE(SV)                                                                                           \
+  inject_kernel<SV><<<(unsigned)n, 256, 0, st>>>((uint8_t*)out, g.ldc * g.es, g.Q, g.RM, row_bytes,           \
+                                                 (const uint8_t*)stale, (uint32_t*)ck, hi.store, rids,        \
+                                                 g.rid_offset, mode, seed)
+  if (S == 1) LP_ICASE(1);
+  else if (S == 2) LP_ICASE(2);
+  else LP_ICASE(3);
+#undef LP_ICASE
+  return cudaGetLastError();
+}
+
+cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st) {
+  stats_kernel<<<1, 1, 0, st>>>((const uint32_t*)ck, hi.store != 0 ? 1 : 0, d_stats);
+  return cudaGetLastError();
+}
+
+}  // namespace lp

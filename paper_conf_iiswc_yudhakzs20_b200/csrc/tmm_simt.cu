@@ -1,0 +1,214 @@
+// tmm_simt.cu -- SIMT LP-protected tiled matrix multiply, paper-shaped.
+//
+// The paper's TMM (Listing 2; Listing 6) is a SIMT kernel
+// whose thread block computes one output tile through shared-memory A/B tiles
+// and is the LP region (L181 §IV-A).  This is that design on sm_100a, kept as
+// the prior-art body (and the fp32-input body): CTA tile == region, 256
+// threads with a register micro-tile, fp32 FFMA accumulate, K in fixed order
+// (deterministic: recovery reproduces the golden bits, Reading R18).
+//
+// LP epilogue (fused, no extra pass over C): every thread folds the exact
+// 32-bit words it stores into its checksum partials (L192), the warp reduces
+// them with one redux.sync per checksum (Listing 4 L244-258 -> redux), warps
+// combine through shared memory (Listing 3), and one thread stores
+// the record lock-free at table[rid] (L349 §V).
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "lp_device.cuh"
+#include "lp_internal.h"
+
+namespace lp {
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kBK = 16;
+
+template <typename T>
+__device__ __forceinline__ float to_f(T v);
+template <>
+__device__ __forceinline__ float to_f<float>(float v) { return v; }
+template <>
+__device__ __forceinline__ float to_f<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
+
+template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK>
+__global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
+                                                            const TIn* __restrict__ B, int64_t ldb,
+                                                            TOut* __restrict__ C, int64_t ldc, int64_t K,
+                                                            int64_t Q, int64_t R, uint32_t* __restrict__ ck,
+                                                            int store, int64_t rid_offset,
+                                                            const int64_t* __restrict__ list,
+                                                            const int64_t* __restrict__ d_n) {
+  static_assert((BM / UM) * (BN / UN) == kThreads, "256 threads");
+  static_assert(UN % 2 == 0, "bf16 words pair two columns");
+  constexpr int TX = BN / UN;  // threads along N
+  constexpr int A_PER = BM * kBK / kThreads;
+  constexpr int B_PER = BN * kBK / kThreads;
+  static_assert(A_PER >= 1 && B_PER >= 1, "tile too small");
+  constexpr int ES = (int)sizeof(TOut);
+
+  __shared__ float As[2][kBK][BM + 4];
+  __shared__ float Bs[2][kBK][BN + 4];
+  __shared__ CkRecord warp_rec[kThreads / 32];
+
+  const int tid = threadIdx.x;
+  const int tx = tid % TX, ty = tid / TX;
+
+  const int64_t ntiles = list ? *d_n : R;
+  for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    const int64_t rid = list ? (list[t] - rid_offset) : t;
+    const int64_t p = rid / Q, q = rid - p * Q;
+    const int64_t row0 = p * BM, col0 = q * BN;
+
+    float acc[UM][UN];
+#pragma unroll
+    for (int i = 0; i < UM; ++i)
+#pragma unroll
+      for (int j = 0; j < UN; ++j) acc[i][j] = 0.f;
+
+    float ra[A_PER], rb[B_PER];
+    auto gload = [&](int64_t k0) {
+#pragma unroll
+      for (int i = 0; i < A_PER; ++i) {
+        const int e = tid + i * kThreads;
+        const int m = e / kBK, k = e % kBK;
+        ra[i] = to_f(A[(row0 + m) * lda + k0 + k]);
+      }
+#pragma unroll
+      for (int i = 0; i < B_PER; ++i) {
+        const int e = tid + i * kThreads;
+        const int k = e / BN, n = e % BN;
+        rb[i] = to_f(B[(k0 + k) * ldb + col0 + n]);
+      }
+    };
+    auto sstore = [&](int buf) {
+#pragma unroll
+      for (int i = 0; i < A_PER; ++i) {
+        const int e = tid + i * kThreads;
+        As[buf][e % kBK][e / kBK] = ra[i];
+      }
+#pragma unroll
+      for (int i = 0; i < B_PER; ++i) {
+        const int e = tid + i * kThreads;
+        Bs[buf][e / BN][e % BN] = rb[i];
+      }
+    };
+
+    __syncthreads();  // previous tile's smem readers are done
+    gload(0);
+    sstore(0);
+    __syncthreads();
+    const int64_t nk = K / kBK;
+    for (int64_t kt = 0; kt < nk; ++kt) {
+      const int buf = (int)(kt & 1);
+      if (kt + 1 < nk) gload((kt + 1) * kBK);
+#pragma unroll
+      for (int k = 0; k < kBK; ++k) {
+        float a[UM], b[UN];
+#pragma unroll
+        for (int i = 0; i < UM; ++i) a[i] = As[buf][k][ty * UM + i];
+#pragma unroll
+        for (int j = 0; j < UN; ++j) b[j] = Bs[buf][k][tx * UN + j];
+#pragma unroll
+        for (int i = 0; i < UM; ++i)
+#pragma unroll
+          for (int j = 0; j < UN; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+      }
+      if (kt + 1 < nk) sstore(buf ^ 1);
+      __syncthreads();
+    }
+
+    // ---- epilogue: store + checksum over the exact stored words
+    CkPartial<MASK> part;
+#pragma unroll
+    for (int i = 0; i < UM; ++i) {
+      const int lr = ty * UM + i;
+      TOut* crow = C + (row0 + lr) * ldc + col0 + tx * UN;
+#pragma unroll
+      for (int j = 0; j < UN; j += 2) {
+        uint32_t w0, w1 = 0;
+        if constexpr (ES == 4) {
+          w0 = __float_as_uint(acc[i][j]);
+          w1 = __float_as_uint(acc[i][j + 1]);
+          *reinterpret_cast<float2*>(crow + j) = make_float2(acc[i][j], acc[i][j + 1]);
+        } else {
+          __nv_bfloat162 h = __floats2bfloat162_rn(acc[i][j], acc[i][j + 1]);  // .x (even col) -> low half
+          w0 = *reinterpret_cast<uint32_t*>(&h);
+          *reinterpret_cast<__nv_bfloat162*>(crow + j) = h;
+        }
+        if constexpr (MASK != 0) {
+          const uint32_t pos = (uint32_t)(lr * BN * ES + (tx * UN + j) * ES + 1);
+          part.add(w0, pos);
+          if constexpr (ES == 4) part.add(w1, pos + 4);
+        }
+      }
+    }
+    if constexpr (MASK != 0) {
+      const CkRecord wr = warp_reduce<MASK>(part);
+      if ((tid & 31) == 0) warp_rec[tid >> 5] = wr;
+      __syncthreads();
+      if (tid == 0) {
+        CkRecord r = warp_rec[0];
+#pragma unroll
+        for (int w = 1; w < kThreads / 32; ++w) r = combine(r, warp_rec[w]);
+        uint32_t words[3];
+        record_words<MASK>(r, (uint64_t)BM * BN * ES, words);
+        store_record<MASK>(ck, store, rid, (uint32_t)(rid + rid_offset), words);
+      }
+    }
+  }
+}
+
+template <typename TIn, typename TOut, int BM, int BN, int UM, int UN>
+cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
+  const int64_t Q = a.N / BN, R = (a.M / BM) * Q;
+  int64_t grid = a.list ? (int64_t)a.sm_count * 4 : R;
+  if (a.list && grid > R) grid = R;
+  if (grid < 1) grid = 1;
+  const TIn* A = (const TIn*)a.A;
+  const TIn* B = (const TIn*)a.B;
+  TOut* C = (TOut*)a.C;
+  switch (a.mask) {
+#define LP_SCASE(M)                                                                                            \
+  case M:                                                                                                      \
+    tmm_simt_kernel<TIn, TOut, BM, BN, UM, UN, M><<<(unsigned)grid, kThreads, 0, st>>>(                        \
+        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.hash.store, a.rid_offset, a.list, a.d_n);             \
+    break;
+    LP_SCASE(0)
+    LP_SCASE(1)
+    LP_SCASE(2)
+    LP_SCASE(3)
+    LP_SCASE(4)
+    LP_SCASE(5)
+    LP_SCASE(6)
+    LP_SCASE(7)
+#undef LP_SCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+template <typename TIn, typename TOut>
+cudaError_t launch_shape(const TmmArgs& a, cudaStream_t st) {
+  if (a.RM == 32 && a.RN == 32) return launch_mask<TIn, TOut, 32, 32, 2, 2>(a, st);
+  if (a.RM == 64 && a.RN == 64) return launch_mask<TIn, TOut, 64, 64, 4, 4>(a, st);
+  if (a.RM == 128 && a.RN == 128) return launch_mask<TIn, TOut, 128, 128, 8, 8>(a, st);
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace
+
+bool tmm_simt_supported(int RM, int RN, int, int) {
+  return (RM == 32 && RN == 32) || (RM == 64 && RN == 64) || (RM == 128 && RN == 128);
+}
+
+cudaError_t launch_tmm_simt(const TmmArgs& a, cudaStream_t st) {
+  if (a.in_bf16) {
+    return a.out_bf16 ? launch_shape<__nv_bfloat16, __nv_bfloat16>(a, st) : launch_shape<__nv_bfloat16, float>(a, st);
+  }
+  return a.out_bf16 ? launch_shape<float, __nv_bfloat16>(a, st) : launch_shape<float, float>(a, st);
+}
+
+}  // namespace lp

@@ -1,0 +1,70 @@
+"""GPU parity: LP-protected 5-point stencil (config C4 shape family) vs the CPU oracle."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from lpsynth import gen
+from paper_conf_iiswc_yudhakzs20_b200 import lp
+from tests.gpu_util import dev_to_host, host_to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def stencil_cycle(H, W, kind, mask, mode, frac, seed=2, store="array"):
+    h = lp.LP(128, 128, cksum=mask, store=store)
+    X = gen.generate(seed, H, W, kind, "f32")
+    x = host_to_dev(X, "f32")
+    wl = lp.Workload.stencil(x)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = host_to_dev(gen.generate(seed + 500, H, W, "bits", "f32"), "f32")
+    out.copy_(stale)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    torch.cuda.synchronize()
+    R = h.num_regions(wl)
+    sel = oracle.selem(h.mask)
+    golden = dev_to_host(out)
+    ck_golden = dev_to_host(ck)
+    # values: bit-exact against the exact-order fp32 oracle (Reading R19)
+    assert np.array_equal(golden.view(np.uint32), oracle.stencil5(X).view(np.uint32))
+    if store == "array":
+        assert np.array_equal(ck_golden[:R * sel].reshape(R, sel), oracle.records(golden, 128, 128, h.mask))
+    h.validate(wl, out, ck, failed, d_n, ws)
+    assert int(d_n.item()) == 0
+    inj = torch.from_numpy(lp.choose_regions(R, frac, 1000 + seed)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode=mode, seed=1000 + seed)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    nf = int(d_n.item())
+    got = failed[:nf].cpu().numpy()
+    if store == "array":
+        exp = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * sel], 128, 128, h.mask)
+        assert np.array_equal(got, exp)
+    assert set(got.tolist()) <= set(inj.cpu().numpy().tolist())
+    if mode == "stale_region":
+        assert nf == inj.numel()
+    h.recover(wl, out, ck, failed, d_n)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+    assert np.array_equal(dev_to_host(out).view(np.uint32), golden.view(np.uint32))
+    return nf
+
+
+@pytest.mark.parametrize("kind", ["uniform", "int17"])
+@pytest.mark.parametrize("frac", [0.01, 0.10, 0.50])
+def test_stencil_inject_recover(kind, frac):
+    stencil_cycle(1024, 768, kind, "mod|xor", "stale_region", frac)
+
+
+@pytest.mark.parametrize("mask", ["mod", "xor", "adler", "mod|xor|adler"])
+@pytest.mark.parametrize("mode", ["stale_words", "bitflip", "stale_record"])
+def test_stencil_checksums_and_modes(mask, mode):
+    stencil_cycle(512, 640, "uniform", mask, mode, 0.2)
+
+
+def test_stencil_quad_store():
+    stencil_cycle(512, 512, "uniform", "mod|xor", "stale_words", 0.25, store="quad_cas")

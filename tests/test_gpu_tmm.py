@@ -1,0 +1,133 @@
+"""GPU parity: LP-protected TMM through the C ABI vs the CPU oracle.
+
+Config C1 (BASELINE.json configs[0]): 256x256x256 fp32, 32x32 regions, MOD, 5% of
+regions corrupted then recovered -- plus random/odd shapes, every checksum type
+and every injection mode.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_iiswc_yudhakzs20_b200 import lp
+from tests.gpu_util import dev_to_host, host_to_dev, make_inputs, stale_image
+
+pytestmark = pytest.mark.gpu
+
+
+def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
+              store="array", check_values=True):
+    h = lp.LP(RM, RN, cksum=mask, store=store, body=body)
+    A, B = make_inputs(seed, M, N, K, kind, in_dt)
+    a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
+    wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = host_to_dev(stale_image(seed, M, N, out_dt), out_dt)
+    out.copy_(stale)                                   # the "persistent" array holds stale bits before the run
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    torch.cuda.synchronize()
+    R = h.num_regions(wl)
+    sel = oracle.selem(h.mask)
+    golden = dev_to_host(out)
+    ck_golden = dev_to_host(ck)
+
+    # (4) clean-run check: records stored by the kernel == oracle records of the stored bits
+    recs = oracle.records(golden, RM, RN, h.mask)
+    if store == "array":
+        assert np.array_equal(ck_golden[:R * sel].reshape(R, sel), recs)
+    else:
+        check_hash_table(ck_golden, R, sel, recs)
+    # (5) values vs fp64 oracle
+    if check_values:
+        to32 = (lambda x: x) if out_dt == "f32" else oracle.bf16_bits_to_f32
+        Q = N // RN
+        rids = range(R) if R <= 64 else np.random.default_rng(seed).choice(R, 16, replace=False)
+        for rid in rids:
+            p, q = divmod(int(rid), Q)
+            ref = oracle.gemm_block_f64(A, B, p * RM, q * RN, RM, RN)
+            got = golden[p * RM:(p + 1) * RM, q * RN:(q + 1) * RN]
+            if kind != "uniform":                       # integer-valued: bit-exact (Reading R18)
+                exp = ref.astype(np.float32) if out_dt == "f32" else oracle.round_bf16(ref)
+                assert np.array_equal(got, exp), rid
+            else:
+                tol = 1e-5 if (out_dt == "f32" and in_dt == "f32") else 2e-2
+                if in_dt == "bf16" and out_dt == "f32":
+                    tol = 1e-5
+                assert oracle.rel_err(to32(got), ref) <= tol, rid
+    # clean validate -> 0 failed
+    h.validate(wl, out, ck, failed, d_n, ws)
+    assert int(d_n.item()) == 0
+
+    # (6)(7) inject, validate == oracle on the corrupted state
+    inj = torch.from_numpy(lp.choose_regions(R, frac, 1000 + seed)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode=mode, seed=1000 + seed)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    nf = int(d_n.item())
+    got_failed = failed[:nf].cpu().numpy()
+    bad_out, bad_ck = dev_to_host(out), dev_to_host(ck)
+    if store == "array":
+        exp_failed = oracle.validate_array(bad_out, bad_ck[:R * sel], RM, RN, h.mask)
+    else:
+        cap = int(bad_ck[0])
+        exp_failed = oracle.validate_quad(bad_out, bad_ck[16:16 + cap * (1 + sel)], cap, int(bad_ck[1]), RM, RN,
+                                          h.mask)
+    assert np.array_equal(got_failed, exp_failed)
+    injected = set(inj.cpu().numpy().tolist())
+    assert set(got_failed.tolist()) <= injected
+    if mode in ("bitflip",):
+        assert set(got_failed.tolist()) == injected          # a bit flip always changes MOD and XOR
+    # (8) recover -> out == golden byte-for-byte, records == golden, re-validate == 0
+    h.recover(wl, out, ck, failed, d_n)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+    assert np.array_equal(dev_to_host(out).view(np.uint8), golden.view(np.uint8))
+    if store == "array":
+        assert np.array_equal(dev_to_host(ck)[:R * sel], ck_golden[:R * sel])
+    else:
+        check_hash_table(dev_to_host(ck), R, sel, recs)
+    return h, nf
+
+
+def check_hash_table(ckh, R, sel, recs):
+    """Every rid is found exactly once by the oracle's lookup with its oracle record (SURVEY §4 layer 4)."""
+    cap, seed = int(ckh[0]), int(ckh[1])
+    table = ckh[16:16 + cap * (1 + sel)]
+    keys = table.reshape(cap, 1 + sel)[:, 0]
+    present = keys[keys != oracle.EMPTY_KEY]
+    assert len(present) == R and len(set(present.tolist())) == R
+    for rid in range(R):
+        assert list(oracle.quad_lookup(table, cap, sel, rid, seed)) == list(recs[rid]), rid
+    assert oracle.quad_lookup(table, cap, sel, R + 7, seed) is None
+
+
+@pytest.mark.parametrize("kind", ["uniform", "int5"])
+@pytest.mark.parametrize("mode", ["stale_words", "stale_region", "bitflip", "stale_record"])
+def test_c1_simt_fp32_mod(kind, mode):
+    """BASELINE configs[0]: 256^3 fp32, 32x32 regions, modular checksum, 5% corrupted then recovered."""
+    _, nf = run_cycle(256, 256, 256, 32, 32, "f32", "f32", kind, "mod", "simt", mode=mode)
+    assert nf >= 1
+
+
+@pytest.mark.parametrize("mask", ["mod", "xor", "adler", "mod|xor", "mod|xor|adler", "xor|adler"])
+def test_simt_checksum_types(mask):
+    run_cycle(256, 192, 96, 32, 32, "f32", "f32", "uniform", mask, "simt", mode="stale_words", frac=0.1)
+
+
+@pytest.mark.parametrize("in_dt,out_dt", [("bf16", "bf16"), ("bf16", "f32"), ("f32", "bf16")])
+def test_simt_dtypes(in_dt, out_dt):
+    run_cycle(128, 256, 64, 32, 32, in_dt, out_dt, "int5", "mod|xor|adler", "simt", frac=0.2)
+
+
+@pytest.mark.parametrize("RM", [64, 128])
+def test_simt_larger_regions(RM):
+    run_cycle(256, 384, 160, RM, RM, "f32", "f32", "uniform", "mod|xor", "simt", frac=0.3)
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
+def test_simt_hash_stores(store):
+    h, _ = run_cycle(256, 256, 64, 32, 32, "f32", "f32", "int5", "mod|xor", "simt", store=store, frac=0.1)
