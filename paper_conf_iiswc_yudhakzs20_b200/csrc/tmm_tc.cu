@@ -1,12 +1,490 @@
-// tmm_tc.cu -- placeholder until the tcgen05 body lands.
+// tmm_tc.cu -- LP-protected tiled matrix multiply on the 5th-generation tensor cores.
+//
+// The region body of the paper's TMM (Listing 2, Listing 6)
+// is a dense contraction, so on sm_100a it runs on tcgen05: operands staged in
+// shared memory by TMA (cp.async.bulk.tensor, 128-B swizzle), one elected
+// thread issuing tcgen05.mma (kind::f16, bf16 x bf16 -> fp32) into a TMEM
+// accumulator, and 4 epilogue warps that read the accumulator back with
+// tcgen05.ld.  Persistent CTAs (one per SM) walk the tile list; TMEM holds two
+// 128x256 accumulators so the epilogue of tile i overlaps the mainloop of
+// tile i+1 -- which is where the LP checksum work (L192) hides.
+//
+// LP epilogue (MASK != 0), fused in registers, no extra pass over C:
+//   * every thread owns one output row of the tile (TMEM lane) and folds the
+//     exact 32-bit words it stores -- bf16 pairs packed even-column-low, or
+//     fp32 bits (L260-261 Fig. 2, Readings R2, R6) -- into MOD / XOR / Adler
+//     partials (L192 §IV-B);
+//   * 32x32 regions: one warp-wide redux.sync per checksum per region
+//     (Listing 4) and lane 0 stores the record;
+//   * 128x128 regions: warp redux + a 4-slot shared-memory combine across the
+//     epilogue warps (Listing 3, named barrier among them only);
+//   * the record goes to table[rid] with one plain store, no lock, no atomic,
+//     no fence (hash-table-less global array, L349 §V), or through the hash
+//     ablation (L265-274).
+//
+// Warp roles (192 threads): warp 0 = TMA producer, warp 1 = TMEM allocator +
+// MMA issuer, warps 2..5 = epilogue (TMEM lane quarter = warp % 4).
+// Region <-> tile: a 128x128 region is half of a 128x256 tile (or a whole
+// 128x128 tile in list mode); a 32x32 region is one warp x 32-column chunk.
+#include <cuda.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "lp_device.cuh"
 #include "lp_internal.h"
+
 namespace lp {
-bool tmm_tc_supported(int64_t, int64_t, int64_t, int, int, int, int64_t, int64_t, int64_t, const void*, const void*,
-                      const void*) {
-  return false;
+namespace {
+
+constexpr int kBM = 128;
+constexpr int kBK = 64;      // 64 bf16 = 128 B = one swizzle atom row
+constexpr int kUmmaK = 16;   // K per tcgen05.mma kind::f16
+constexpr int kThreads = 192;
+constexpr int kEpiWarp0 = 2;
+
+template <int BN>
+struct TcCfg {
+  static constexpr int kStages = BN == 256 ? 4 : 6;
+  static constexpr int kABytes = kBM * kBK * 2;            // 16 KiB
+  static constexpr int kBBytes = kBK * BN * 2;             // 32 / 16 KiB
+  static constexpr int kStageBytes = kABytes + kBBytes;
+  static constexpr int kTmemCols = 2 * BN;                 // two accumulators
+  static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*barriers etc.*/ + 1024 /*align slack*/;
+};
+
+// ---------------------------------------------------------------------------- PTX wrappers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
 }
-cudaError_t launch_tmm_tc(const TmmArgs&, cudaStream_t, const char** why) {
-  *why = "not built";
-  return cudaErrorNotSupported;
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
 }
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+
+__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                       uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
+__device__ __forceinline__ void tc_commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+
+#define LP_TMEM_LD32(taddr, r)                                                                                       \
+  asm volatile(                                                                                                      \
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"   \
+      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"                                                 \
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),  \
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),       \
+        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),      \
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])                    \
+      : "r"(taddr))
+
+__device__ __forceinline__ void tc_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
+// Shared-memory matrix descriptor (sm_100 UMMA): start>>4 [0,14), LBO>>4 [16,30),
+// SBO>>4 [32,46), version 1 [46,48), layout SWIZZLE_128B = 2 at [61,64).
+__device__ __forceinline__ uint64_t smem_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;
+  d |= (uint64_t)2 << 61;
+  return d;
+}
+
+// Instruction descriptor kind::f16: D fp32 [4,6)=1, A bf16 [7,10)=1, B bf16 [10,13)=1,
+// A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29).
+template <int BN>
+__host__ __device__ constexpr uint32_t instr_desc() {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
+         ((uint32_t)(kBM >> 4) << 24);
+}
+
+__device__ __forceinline__ void named_bar_epi() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
+
+// Tile order: groups of 16 M-blocks, M fastest inside a group (L2 reuse of B panels).
+__device__ __forceinline__ void tile_coords(int64_t t, int64_t num_m, int64_t num_n, int64_t& mb, int64_t& nb) {
+  constexpr int64_t G = 16;
+  const int64_t per_group = G * num_n;
+  const int64_t g = t / per_group, w = t - g * per_group;
+  const int64_t rows = (num_m - g * G) < G ? (num_m - g * G) : G;
+  mb = g * G + w % rows;
+  nb = w / rows;
+}
+
+struct TileSrc {
+  int64_t num_m, num_n;       // tile grid
+  const int64_t* list;        // list mode: failed global rids
+  const int64_t* d_n;
+  int64_t rid_offset;
+  int64_t Qr;                 // regions per output row band
+  int reg;                    // region edge (32 or 128)
+  __device__ __forceinline__ int64_t count() const { return list ? *d_n : num_m * num_n; }
+  template <int BN>
+  __device__ __forceinline__ void coords(int64_t t, int64_t& mb, int64_t& nb) const {
+    if (!list) {
+      tile_coords(t, num_m, num_n, mb, nb);
+      return;
+    }
+    const int64_t rid = list[t] - rid_offset;
+    const int64_t p = rid / Qr, q = rid - p * Qr;
+    mb = p * reg / kBM;
+    nb = q * reg / BN;
+  }
+};
+
+template <typename OutT, uint32_t MASK, int REG, int BN>
+__global__ void __launch_bounds__(kThreads, 1)
+    tmm_tc_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+                  OutT* __restrict__ C, int64_t ldc, int64_t K, TileSrc src, uint32_t* __restrict__ ck, int store) {
+  using Cfg = TcCfg<BN>;
+  constexpr int S = Cfg::kStages;
+  constexpr int ES = (int)sizeof(OutT);
+  constexpr int NCH = BN / 32;  // 32-column chunks per tile row
+
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + S * Cfg::kABytes;
+  uint64_t* full = (uint64_t*)(smem + S * Cfg::kStageBytes);
+  uint64_t* empty = full + S;
+  uint64_t* tfull = empty + S;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_holder = (uint32_t*)(tempty + 2);
+  CkRecord* srec = (CkRecord*)(tmem_holder + 4);  // [2 acc][BN/128 regions][4 warps]
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (warp == 0 && lane == 0) {
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_a) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"((uint64_t)&tmap_b) : "memory");
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], 1);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&tfull[s], 1);
+      mbar_init(&tempty[s], 4);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_holder)),
+                 "r"((uint32_t)Cfg::kTmemCols)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_holder;
+
+  const int64_t ntiles = src.count();
+  const int nkb = (int)(K / kBK);
+
+  if (warp == 0) {
+    // ===================== TMA producer =====================
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        int64_t mb, nb;
+        src.coords<BN>(t, mb, nb);
+        const int m0 = (int)(mb * kBM), n0 = (int)(nb * BN);
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
+          tma_load_2d(&tmap_a, &full[stage], sA + stage * Cfg::kABytes, kb * kBK, m0);
+#pragma unroll
+          for (int c = 0; c < BN / 64; ++c)
+            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), n0 + c * 64, kb * kBK);
+          if (++stage == S) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ===================== MMA issuer (one thread) =====================
+    if (lane == 0) {
+      constexpr uint32_t idesc = instr_desc<BN>();
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);  // epilogue drained this accumulator
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_addr = smem_u32(sA + stage * Cfg::kABytes);
+          const uint32_t b_addr = smem_u32(sB + stage * Cfg::kBBytes);
+#pragma unroll
+          for (int k = 0; k < kBK / kUmmaK; ++k) {
+            // A: K-major SW128, +32 B per K=16 step inside the 128-B atom; SBO = 8 rows * 128 B.
+            const uint64_t ad = smem_desc(a_addr + k * kUmmaK * 2, 16, 1024);
+            // B: MN-major SW128, LBO = stride between 64-column chunks, SBO = 8 K-rows * 128 B,
+            //    +16 K-rows * 128 B per step.
+            const uint64_t bd = smem_desc(b_addr + k * kUmmaK * 128, kBK * 128, 1024);
+            tc_mma(d_tmem, ad, bd, idesc, (kb | k) ? 1u : 0u);
+          }
+          tc_commit(&empty[stage]);  // frees the smem slot when these MMAs complete
+          if (++stage == S) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc_commit(&tfull[acc]);  // accumulator ready for the epilogue
+        if (++acc == 2) {
+          acc = 0;
+          acc_phase ^= 1;
+        }
+      }
+    }
+  } else {
+    // ===================== epilogue (4 warps, 128 threads) =====================
+    const int wq = warp & 3;              // TMEM lane quarter owned by this warp
+    const int row_in_tile = wq * 32 + lane;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      int64_t mb, nb;
+      src.coords<BN>(t, mb, nb);
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
+      OutT* crow = C + (mb * kBM + row_in_tile) * ldc + nb * BN;
+      CkPartial<MASK> part;
+#pragma unroll 1
+      for (int ch = 0; ch < NCH; ++ch) {
+        uint32_t r[32];
+        LP_TMEM_LD32(t_row + ch * 32, r);
+        tc_wait_ld();
+        if constexpr (ES == 2) {
+          uint32_t w[16];
+#pragma unroll
+          for (int i = 0; i < 16; ++i) {
+            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
+            w[i] = *reinterpret_cast<uint32_t*>(&h);
+          }
+          uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+          if constexpr (MASK != 0) {
+            // byte position of word 0 of this chunk inside its region's stream
+            const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+                                             : (uint32_t)(lane * 32 * ES + 1);
+#pragma unroll
+            for (int i = 0; i < 16; ++i) part.add(w[i], pos0 + 4 * i);
+          }
+        } else {
+          uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
+#pragma unroll
+          for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
+          if constexpr (MASK != 0) {
+            const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+                                             : (uint32_t)(lane * 32 * ES + 1);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) part.add(r[i], pos0 + 4 * i);
+          }
+        }
+        if constexpr (MASK != 0) {
+          if constexpr (REG == 32) {
+            // one 32x32 region = this warp's 32 rows x this 32-column chunk
+            const CkRecord rec = warp_reduce<MASK>(part);
+            if (lane == 0) {
+              const int64_t p = mb * (kBM / 32) + wq, q = (nb * BN + ch * 32) / 32;
+              const int64_t rid = p * src.Qr + q;
+              uint32_t words[3];
+              record_words<MASK>(rec, (uint64_t)32 * 32 * ES, words);
+              store_record<MASK>(ck, store, rid, (uint32_t)(rid + src.rid_offset), words);
+            }
+            part = CkPartial<MASK>();
+          } else if ((ch & 3) == 3) {
+            // end of a 128-column region: warp partial -> smem slot
+            const CkRecord rec = warp_reduce<MASK>(part);
+            if (lane == 0) srec[(acc * (BN / 128) + ch / 4) * 4 + wq] = rec;
+            part = CkPartial<MASK>();
+          }
+        }
+      }
+      // all TMEM reads of this accumulator are complete (wait::ld above): release it
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&tempty[acc]);
+      if constexpr (MASK != 0 && REG == 128) {
+        named_bar_epi();
+        if (warp == kEpiWarp0 && lane < BN / 128) {
+          const int j = lane;
+          CkRecord rr = srec[(acc * (BN / 128) + j) * 4 + 0];
+#pragma unroll
+          for (int w = 1; w < 4; ++w) rr = combine(rr, srec[(acc * (BN / 128) + j) * 4 + w]);
+          const int64_t rid = mb * src.Qr + nb * (BN / 128) + j;
+          uint32_t words[3];
+          record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
+          store_record<MASK>(ck, store, rid, (uint32_t)(rid + src.rid_offset), words);
+        }
+      }
+      if (++acc == 2) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "r"((uint32_t)Cfg::kTmemCols)
+                 : "memory");
+  }
+}
+
+// ---------------------------------------------------------------------------- host side
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+PFN_encodeTiled get_encode() {
+  static PFN_encodeTiled fn = nullptr;
+  if (!fn) {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = (PFN_encodeTiled)p;
+  }
+  return fn;
+}
+
+bool make_map_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
+                 uint32_t box_inner, uint32_t box_outer) {
+  PFN_encodeTiled enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld_elems * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+template <typename OutT, int REG, int BN>
+cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
+  using Cfg = TcCfg<BN>;
+  CUtensorMap ma, mb;
+  if (!make_map_2d(&ma, a.A, (uint64_t)a.K, (uint64_t)a.M, (uint64_t)a.lda, kBK, kBM) ||
+      !make_map_2d(&mb, a.B, (uint64_t)a.N, (uint64_t)a.K, (uint64_t)a.ldb, 64, kBK)) {
+    *why = "cuTensorMapEncodeTiled failed";
+    return cudaErrorInvalidValue;
+  }
+  TileSrc src;
+  src.num_m = a.M / kBM;
+  src.num_n = a.N / BN;
+  src.list = a.list;
+  src.d_n = a.d_n;
+  src.rid_offset = a.rid_offset;
+  src.Qr = a.N / REG;
+  src.reg = REG;
+  const int64_t R = (a.M / REG) * (a.N / REG);
+  int64_t grid = a.list ? (R < a.sm_count ? R : a.sm_count) : src.num_m * src.num_n;
+  if (grid > a.sm_count) grid = a.sm_count;
+  if (grid < 1) grid = 1;
+  const int smem = Cfg::kSmemBytes;
+  cudaError_t e = cudaSuccess;
+  switch (a.mask) {
+#define LP_TC_CASE(M)                                                                                       \
+  case M: {                                                                                                 \
+    auto kfn = tmm_tc_kernel<OutT, M, REG, BN>;                                                            \
+    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
+    if (e != cudaSuccess) return e;                                                                         \
+    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, src, a.ck, a.hash.store);  \
+    break;                                                                                                  \
+  }
+    LP_TC_CASE(0)
+    LP_TC_CASE(1)
+    LP_TC_CASE(2)
+    LP_TC_CASE(3)
+    LP_TC_CASE(4)
+    LP_TC_CASE(5)
+    LP_TC_CASE(6)
+    LP_TC_CASE(7)
+#undef LP_TC_CASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+template <typename OutT, int REG>
+cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
+  // list mode with 128x128 regions re-executes exactly one region per tile (BN = 128)
+  const bool bn256 = (a.N % 256 == 0) && !(a.list && REG == 128);
+  return bn256 ? launch_cfg<OutT, REG, 256>(a, st, why) : launch_cfg<OutT, REG, 128>(a, st, why);
+}
+
+}  // namespace
+
+bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int64_t lda, int64_t ldb,
+                      int64_t ldc, const void* A, const void* B, const void* C) {
+  if (!in_bf16) return false;
+  if (!((RM == 128 && RN == 128) || (RM == 32 && RN == 32))) return false;
+  if (M % kBM || N % 128 || K % kBK || K <= 0) return false;
+  if ((lda * 2) % 16 || (ldb * 2) % 16 || (ldc * 2) % 16) return false;
+  if ((((uintptr_t)A) & 15u) || (((uintptr_t)B) & 15u) || (((uintptr_t)C) & 15u)) return false;
+  if (M > (int64_t)INT32_MAX || N > (int64_t)INT32_MAX || K > (int64_t)INT32_MAX) return false;
+  return true;
+}
+
+cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why) {
+  if (a.RM == 128) {
+    return a.out_bf16 ? launch_reg<__nv_bfloat16, 128>(a, st, why) : launch_reg<float, 128>(a, st, why);
+  }
+  return a.out_bf16 ? launch_reg<__nv_bfloat16, 32>(a, st, why) : launch_reg<float, 32>(a, st, why);
+}
+
 }  // namespace lp

@@ -1,0 +1,36 @@
+import sys, time, torch
+sys.path.insert(0, '.')
+import lpsynth
+from paper_conf_iiswc_yudhakzs20_b200 import lp
+M=N=K=8192
+a = torch.empty((M,K), dtype=torch.bfloat16, device='cuda'); b = torch.empty((K,N), dtype=torch.bfloat16, device='cuda')
+lpsynth.device_fill(a, 1, 'uniform', 'bf16'); lpsynth.device_fill(b, 2, 'uniform', 'bf16')
+flush = torch.empty(512<<20, dtype=torch.uint8, device='cuda')
+res = {}
+for name, mask, reg in [('unprot',0,128),('mod',1,128),('xor',2,128),('modxor',3,128),('adler',4,128),('all',7,128),('modxor32',3,32)]:
+    h = lp.LP(reg,reg,cksum=mask,body='tcgen05')
+    wl = lp.Workload.tmm(a,b,out_dtype='bf16')
+    out,ck,failed,d_n,ws = h.alloc(wl)
+    if mask: h.cksum_init(wl,ck)
+    ts=[]
+    for i in range(12):
+        flush.zero_()
+        e0=torch.cuda.Event(enable_timing=True); e1=torch.cuda.Event(enable_timing=True)
+        e0.record(); h.run_protected(wl,out,ck if mask else None); e1.record(); torch.cuda.synchronize()
+        ts.append(e0.elapsed_time(e1))
+    ts=sorted(ts[2:]); t=ts[len(ts)//2]
+    res[name]=t
+    print(f"{name:10s} {t*1e3:8.1f} us  {2*M*N*K/t/1e9:8.1f} TFLOP/s", flush=True)
+    if mask:
+        ts=[]
+        for i in range(10):
+            flush.zero_()
+            e0=torch.cuda.Event(enable_timing=True); e1=torch.cuda.Event(enable_timing=True)
+            e0.record(); h.validate(wl,out,ck,failed,d_n,ws); e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
+        t=sorted(ts)[5]; print(f"   validate {t*1e3:8.1f} us  {M*N*2/t/1e6:8.1f} GB/s  nfail={int(d_n.item())}", flush=True)
+ts=[]
+for i in range(10):
+    flush.zero_()
+    e0=torch.cuda.Event(enable_timing=True); e1=torch.cuda.Event(enable_timing=True)
+    e0.record(); c=a@b; e1.record(); torch.cuda.synchronize(); ts.append(e0.elapsed_time(e1))
+t=sorted(ts)[5]; print(f"torch.matmul {t*1e3:8.1f} us {2*M*N*K/t/1e9:8.1f} TFLOP/s")

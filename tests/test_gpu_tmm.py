@@ -131,3 +131,68 @@ def test_simt_larger_regions(RM):
 @pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
 def test_simt_hash_stores(store):
     h, _ = run_cycle(256, 256, 64, 32, 32, "f32", "f32", "int5", "mod|xor", "simt", store=store, frac=0.1)
+
+
+# ----------------------------------------------------------------------------- tcgen05 body (bf16 in)
+@pytest.mark.parametrize("kind", ["int5", "uniform"])
+@pytest.mark.parametrize("out_dt", ["bf16", "f32"])
+@pytest.mark.parametrize("reg", [128, 32])
+def test_tc_cycle(kind, out_dt, reg):
+    run_cycle(256, 512, 256, reg, reg, "bf16", out_dt, kind, "mod|xor", "tcgen05", mode="stale_words", frac=0.2)
+
+
+@pytest.mark.parametrize("mask", ["mod", "xor", "adler", "mod|xor|adler"])
+def test_tc_checksum_types(mask):
+    run_cycle(384, 768, 192, 128, 128, "bf16", "bf16", "uniform", mask, "tcgen05", mode="bitflip", frac=0.3)
+
+
+def test_tc_n_not_multiple_of_256():
+    run_cycle(256, 384, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", mode="stale_region", frac=0.5)
+
+
+def test_tc_many_tiles_persistent():
+    # more tiles than SMs: persistent scheduling + TMEM double buffering across tiles
+    run_cycle(2048, 2048, 512, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", mode="stale_words",
+              frac=0.05, check_values=True)
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
+def test_tc_hash_stores(store):
+    run_cycle(512, 512, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, frac=0.1)
+
+
+def test_tc_unprotected_twin_same_bits():
+    """cksum=0 builds the same body without the epilogue checksum: identical output bits."""
+    import numpy as np
+    from tests.gpu_util import make_inputs
+    A, B = make_inputs(3, 512, 512, 256, "uniform", "bf16")
+    a, b = host_to_dev(A, "bf16"), host_to_dev(B, "bf16")
+    outs = []
+    for mask in [0, 3]:
+        h = lp.LP(128, 128, cksum=mask, body="tcgen05")
+        wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+        out, ck, *_ = h.alloc(wl)
+        if mask:
+            h.cksum_init(wl, ck)
+        h.run_protected(wl, out, ck if mask else None)
+        torch.cuda.synchronize()
+        outs.append(dev_to_host(out))
+    assert np.array_equal(outs[0], outs[1])
+
+
+def test_tc_matches_simt_integer_valued():
+    """Both bodies are exact on integer-valued inputs: same bits (cross-check of two independent kernels)."""
+    import numpy as np
+    from tests.gpu_util import make_inputs
+    A, B = make_inputs(4, 256, 256, 128, "int5", "bf16")
+    a, b = host_to_dev(A, "bf16"), host_to_dev(B, "bf16")
+    res = []
+    for body in ["simt", "tcgen05"]:
+        h = lp.LP(128, 128, cksum="mod|xor", body=body)
+        wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+        out, ck, *_ = h.alloc(wl)
+        h.cksum_init(wl, ck)
+        h.run_protected(wl, out, ck)
+        torch.cuda.synchronize()
+        res.append((dev_to_host(out), dev_to_host(ck)))
+    assert np.array_equal(res[0][0], res[1][0]) and np.array_equal(res[0][1], res[1][1])
