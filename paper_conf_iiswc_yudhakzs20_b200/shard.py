@@ -1,0 +1,64 @@
+"""Region sharding across GPUs (host logic).
+
+LP regions are associative and independent (L51, L181) and the record array is
+indexed by region id (L349), so each GPU owns a disjoint contiguous band of
+region rows: rank g owns output rows [g*M/G, (g+1)*M/G) -- i.e. global rids
+[g*R/G, (g+1)*R/G) -- together with its A row panel, a full B, its C shard and
+its slice of the record table.  Protected run, validation, compaction and
+recovery are all local; the only exchange is an all-reduce(SUM) of the int64
+counts {n_failed, n_recovered, n_failed_after} (16-24 bytes, latency-bound),
+issued straight from device memory on the compute stream.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+
+@dataclass(frozen=True)
+class Shard:
+    rank: int
+    world: int
+    row_offset: int   # first global output row of this shard
+    rows: int         # rows of this shard
+    rid_offset: int   # first global region id
+    regions: int      # regions of this shard
+
+
+def plan(global_m: int, n: int, region_m: int, region_n: int, world: int, rank: int) -> Shard:
+    """Contiguous row-band shard of a global_m x n output, in whole region rows."""
+    if global_m % region_m or n % region_n:
+        raise ValueError("output must be a whole number of regions")
+    P = global_m // region_m
+    Q = n // region_n
+    if P < world:
+        raise ValueError(f"{P} region rows cannot be split over {world} ranks")
+    lo = (P * rank) // world
+    hi = (P * (rank + 1)) // world
+    return Shard(rank, world, lo * region_m, (hi - lo) * region_m, lo * Q, (hi - lo) * Q)
+
+
+def allreduce_counts(counts, group=None):
+    """SUM all-reduce of the device int64 count vector (the one collective of the path)."""
+    import torch.distributed as dist
+
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(counts, op=dist.ReduceOp.SUM, group=group)
+    return counts
+
+
+def gather_failed(local_failed, group=None):
+    """All-gather of the per-rank failed-rid lists (off the hot path; used by checks)."""
+    import torch
+    import torch.distributed as dist
+
+    if not (dist.is_available() and dist.is_initialized()) or dist.get_world_size(group) == 1:
+        return local_failed
+    n = torch.tensor([local_failed.numel()], dtype=torch.int64, device=local_failed.device)
+    sizes = [torch.zeros_like(n) for _ in range(dist.get_world_size(group))]
+    dist.all_gather(sizes, n, group=group)
+    mx = int(max(int(s.item()) for s in sizes))
+    pad = torch.full((mx,), -1, dtype=torch.int64, device=local_failed.device)
+    pad[:local_failed.numel()] = local_failed
+    outs = [torch.empty_like(pad) for _ in sizes]
+    dist.all_gather(outs, pad, group=group)
+    return torch.cat([o[:int(s.item())] for o, s in zip(outs, sizes)])
