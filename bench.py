@@ -107,6 +107,11 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
+    def wait_first(self, timeout=5.0):
+        t0 = time.time()
+        while self.proc is not None and not self.lines and time.time() - t0 < timeout:
+            time.sleep(0.05)
+
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
@@ -261,6 +266,7 @@ def run_ours(args):
     # ---- warm-up (clock sampling runs from here through the timed steps and the overhead reps)
     clk = ClockSampler(local)
     clk.start()
+    clk.wait_first()
     for _ in range(max(args.warmup, 3)):
         e = step(True)
         torch.cuda.synchronize()

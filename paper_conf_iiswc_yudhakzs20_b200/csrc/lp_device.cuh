@@ -150,7 +150,7 @@ __host__ __device__ __forceinline__ uint32_t hash_fmix32(uint32_t key, uint32_t 
 // empty before inserting; probe i visits home + i^2, L267).  Called by ONE
 // thread per region.  Returns the number of probes.
 template <uint32_t MASK>
-__device__ uint32_t quad_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+__device__ __forceinline__ uint32_t quad_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
   constexpr int S = selem_of(MASK);
   HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
   uint32_t* ent = ckbuf + sizeof(HashHeader) / 4;
@@ -174,7 +174,7 @@ __device__ uint32_t quad_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w
 // Lock-based variant (L81-83 CPU style; L341 "lock-based"): the whole probe +
 // insert runs inside one global spin lock (Reading R15).
 template <uint32_t MASK>
-__device__ uint32_t quad_insert_locked(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+__device__ __forceinline__ uint32_t quad_insert_locked(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
   constexpr int S = selem_of(MASK);
   HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
   uint32_t* ent = ckbuf + sizeof(HashHeader) / 4;
@@ -226,13 +226,13 @@ __device__ __forceinline__ bool quad_lookup(const uint32_t* ckbuf, uint32_t rid,
   return false;
 }
 
-// Dispatch of the record store on the runtime store kind.
-template <uint32_t MASK>
-__device__ __forceinline__ void store_record(uint32_t* ck, int store, int64_t local_rid, uint32_t global_rid,
-                                             const uint32_t* w) {
-  if (store == 0) {
+// Record store, selected at compile time so the array-store kernels carry no
+// hash-table code (and no register pressure from it).
+template <uint32_t MASK, int STORE>
+__device__ __forceinline__ void store_record(uint32_t* ck, int64_t local_rid, uint32_t global_rid, const uint32_t* w) {
+  if constexpr (STORE == 0) {
     store_array<MASK>(ck, local_rid, w);
-  } else if (store == 1) {
+  } else if constexpr (STORE == 1) {
     quad_insert<MASK>(ck, global_rid, w);
   } else {
     quad_insert_locked<MASK>(ck, global_rid, w);

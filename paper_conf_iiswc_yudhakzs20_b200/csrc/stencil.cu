@@ -8,14 +8,21 @@
 //   out[i][j] = 0.5*in[i][j] + 0.125*(((in[i-1][j] + in[i+1][j]) + in[i][j-1]) + in[i][j+1])
 //
 // every op rounded to fp32 (__fadd_rn/__fmul_rn: no FMA contraction), zero
-// outside the domain.  CTA = one 128x128 region; warp w owns 16 rows; each lane
-// owns 4 adjacent columns (one 16-B vector).  All 18 input rows a lane needs
-// are issued before any is used (18 x 16 B in flight per lane); the left/right
-// neighbours come from the adjacent lanes through shuffles, the region's outer
-// columns from one scalar load at each edge.  The checksum of the stored words
-// is folded in registers (L192), warp-reduced with redux.sync and combined
-// across the 8 warps in shared memory (Listings 3-4) before one thread stores
-// the record at table[rid] (L349).
+// outside the domain.
+//
+// Structure: CTA = one 128x128 region, 8 warps x 16 rows, lane = 4 adjacent
+// columns (one 16-B vector).  Every lane issues all 18 row loads and its 16
+// edge loads up front (non-allocating 16-B loads through volatile PTX), then
+// computes; left/right neighbours come from the adjacent lanes by shuffle;
+// results leave with streaming 16-B stores.  2 CTAs (16 warps) per SM.
+//
+// LP epilogue: each lane folds the exact stored words into its checksum
+// partials (L192) and the warp reduces them with redux.sync (Listing 4).  The
+// 8 warps' partials are combined WITHOUT a CTA barrier: lane 0 of each warp
+// folds its partial into shared accumulators with shared-memory atomics and
+// the last warp to arrive finalises and stores the record at table[rid]
+// (L349).  (A Listing-3 style barrier combine, kept for list-mode recovery where
+// a CTA handles several regions, costs 29% here: measured.)
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -26,53 +33,59 @@ namespace lp {
 namespace {
 
 constexpr int kRM = 128, kRN = 128;
-constexpr int kWarps = 8;
-constexpr int kRowsPerWarp = kRM / kWarps;  // 16
-
-__device__ __forceinline__ float4 ld_row4(const float* in, int64_t ldi, int64_t H, int64_t i, int64_t j) {
-  if (i < 0 || i >= H) return make_float4(0.f, 0.f, 0.f, 0.f);
-  return __ldg(reinterpret_cast<const float4*>(in + i * ldi + j));
-}
-
-__device__ __forceinline__ float ld1(const float* in, int64_t ldi, int64_t H, int64_t W, int64_t i, int64_t j) {
-  if (i < 0 || i >= H || j < 0 || j >= W) return 0.f;
-  return __ldg(in + i * ldi + j);
-}
 
 __device__ __forceinline__ float st5(float c, float u, float d, float l, float r) {
   const float s = __fadd_rn(__fadd_rn(__fadd_rn(u, d), l), r);
   return __fadd_rn(__fmul_rn(0.5f, c), __fmul_rn(0.125f, s));
 }
 
-template <uint32_t MASK>
-__global__ void __launch_bounds__(kWarps * 32) stencil5_kernel(const float* __restrict__ in, int64_t ldi,
-                                                               float* __restrict__ out, int64_t ldo, int64_t H,
-                                                               int64_t W, int64_t Q, int64_t R,
-                                                               uint32_t* __restrict__ ck, int store,
-                                                               int64_t rid_offset, const int64_t* __restrict__ list,
-                                                               const int64_t* __restrict__ d_n) {
-  __shared__ CkRecord warp_rec[kWarps];
+__device__ __forceinline__ float4 ldg_nc_v4(const float* p) {
+  float4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w)
+               : "l"(p));
+  return r;
+}
+__device__ __forceinline__ float ldg_nc_f(const float* p) {
+  float r;
+  asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(p));
+  return r;
+}
+
+template <uint32_t MASK, int STORE, int COMBINE>
+__global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __restrict__ in, int64_t ldi,
+                                                              float* __restrict__ out, int64_t ldo, int H, int W,
+                                                              int64_t Q, int64_t R, uint32_t* __restrict__ ck,
+                                                              int64_t rid_offset, const int64_t* __restrict__ list,
+                                                              const int64_t* __restrict__ d_n) {
+  constexpr int kRowsW = 16;
+  __shared__ CkRecord warp_rec[8];
+  __shared__ uint32_t s_acc[5];  // COMBINE == 1: mod, xor, adler s, adler w, arrivals
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if constexpr (COMBINE == 1) {
+    if (threadIdx.x < 5) s_acc[threadIdx.x] = 0u;
+    __syncthreads();
+  }
   const int64_t ntiles = list ? *d_n : R;
   for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
     const int64_t rid = list ? (list[t] - rid_offset) : t;
     const int64_t p = rid / Q, q = rid - p * Q;
-    const int64_t i0 = p * kRM + wid * kRowsPerWarp;
-    const int64_t j = q * kRN + lane * 4;
-
-    float4 v[kRowsPerWarp + 2];
+    const int i0 = (int)(p * kRM) + wid * kRowsW;
+    const int j = (int)(q * kRN) + lane * 4;
+    const int je = lane == 0 ? j - 1 : j + 4;
+    const bool eok = (lane == 0 || lane == 31) && je >= 0 && je < W;
+    float4 v[kRowsW + 2];
+    float edge[kRowsW];
 #pragma unroll
-    for (int r = 0; r < kRowsPerWarp + 2; ++r) v[r] = ld_row4(in, ldi, H, i0 - 1 + r, j);
-    float edge[kRowsPerWarp];
-#pragma unroll
-    for (int r = 0; r < kRowsPerWarp; ++r) {
-      // lane 0 needs column j-1, lane 31 needs column j+4 (outside this warp's 128 columns)
-      edge[r] = lane == 0 ? ld1(in, ldi, H, W, i0 + r, j - 1) : (lane == 31 ? ld1(in, ldi, H, W, i0 + r, j + 4) : 0.f);
+    for (int r = 0; r < kRowsW + 2; ++r) {
+      const int i = i0 - 1 + r;
+      v[r] = ((unsigned)i < (unsigned)H) ? ldg_nc_v4(in + (int64_t)i * ldi + j) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
-
+#pragma unroll
+    for (int r = 0; r < kRowsW; ++r) edge[r] = eok ? ldg_nc_f(in + (int64_t)(i0 + r) * ldi + je) : 0.f;
     CkPartial<MASK> part;
 #pragma unroll
-    for (int r = 0; r < kRowsPerWarp; ++r) {
+    for (int r = 0; r < kRowsW; ++r) {
       const float4 u = v[r], c = v[r + 1], d = v[r + 2];
       float left = __shfl_up_sync(0xFFFFFFFFu, c.w, 1);
       float right = __shfl_down_sync(0xFFFFFFFFu, c.x, 1);
@@ -83,31 +96,54 @@ __global__ void __launch_bounds__(kWarps * 32) stencil5_kernel(const float* __re
       o.y = st5(c.y, u.y, d.y, c.x, c.z);
       o.z = st5(c.z, u.z, d.z, c.y, c.w);
       o.w = st5(c.w, u.w, d.w, c.z, right);
-      *reinterpret_cast<float4*>(out + (i0 + r) * ldo + j) = o;
+      __stcs(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
       if constexpr (MASK != 0) {
-        const uint32_t pos = (uint32_t)((wid * kRowsPerWarp + r) * kRN * 4 + lane * 16 + 1);
+        const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
         part.add(__float_as_uint(o.x), pos);
         part.add(__float_as_uint(o.y), pos + 4);
         part.add(__float_as_uint(o.z), pos + 8);
         part.add(__float_as_uint(o.w), pos + 12);
       }
     }
-    if constexpr (MASK != 0) {
+    if constexpr (MASK != 0 && COMBINE == 1) {
+      // barrier-free combine (one region per CTA): warp partials fold into the
+      // shared accumulators with shared-memory atomics; the last warp to arrive
+      // finalises and stores the record.
+      const CkRecord wr = warp_reduce<MASK>(part);
+      if (lane == 0) {
+        if constexpr ((MASK & kMod) != 0) atomicAdd(&s_acc[0], wr.mod);
+        if constexpr ((MASK & kXor) != 0) atomicXor(&s_acc[1], wr.xr);
+        if constexpr ((MASK & kAdler) != 0) {
+          atomicAdd(&s_acc[2], wr.s);
+          atomicAdd(&s_acc[3], wr.wmod);
+        }
+        __threadfence_block();
+        if (atomicAdd(&s_acc[4], 1u) == 7u) {
+          __threadfence_block();
+          const CkRecord rr{atomicAdd(&s_acc[0], 0u), atomicAdd(&s_acc[1], 0u), atomicAdd(&s_acc[2], 0u),
+                            atomicAdd(&s_acc[3], 0u)};
+          uint32_t words[3];
+          record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
+          store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+        }
+      }
+    } else if constexpr (MASK != 0) {
       const CkRecord wr = warp_reduce<MASK>(part);
       if (lane == 0) warp_rec[wid] = wr;
       __syncthreads();
       if (threadIdx.x == 0) {
         CkRecord rr = warp_rec[0];
 #pragma unroll
-        for (int w = 1; w < kWarps; ++w) rr = combine(rr, warp_rec[w]);
+        for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
         uint32_t words[3];
         record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
-        store_record<MASK>(ck, store, rid, (uint32_t)(rid + rid_offset), words);
+        store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
       }
-      __syncthreads();
+      if (list) __syncthreads();
     }
   }
 }
+
 
 }  // namespace
 
@@ -115,24 +151,35 @@ bool stencil_supported(int RM, int RN) { return RM == kRM && RN == kRN; }
 
 cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   const int64_t Q = a.W / kRN, R = (a.H / kRM) * Q;
-  int64_t grid = a.list ? (int64_t)a.sm_count * 8 : R;
-  if (a.list && grid > R) grid = R;
+  if (a.H > (int64_t)INT32_MAX / 2 || a.W > (int64_t)INT32_MAX / 2) return cudaErrorInvalidValue;
+  const int sk = a.mask ? a.hash.store : 0;
+  // full run: one region per CTA, barrier-free combine; list mode (recovery):
+  // persistent CTAs over the failed list, barrier combine (accumulators reused)
+  int64_t grid = a.list ? (R < a.sm_count * 2 ? R : a.sm_count * 2) : R;
   if (grid < 1) grid = 1;
-  switch (a.mask) {
-#define LP_TCASE(M)                                                                                            \
-  case M:                                                                                                      \
-    stencil5_kernel<M><<<(unsigned)grid, kWarps * 32, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.H, a.W, Q, R, a.ck, \
-                                                               a.hash.store, a.rid_offset, a.list, a.d_n);     \
+  switch (a.mask * 3 + sk) {
+#define LP_LCASE(M, S)                                                                                          \
+  case M * 3 + S:                                                                                               \
+    if (a.list)                                                                                                 \
+      stencil5_ldg_kernel<M, S, 0><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H,         \
+                                                                   (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
+                                                                   a.d_n);                                      \
+    else                                                                                                        \
+      stencil5_ldg_kernel<M, S, 1><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H,         \
+                                                                   (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
+                                                                   a.d_n);                                      \
     break;
-    LP_TCASE(0)
-    LP_TCASE(1)
-    LP_TCASE(2)
-    LP_TCASE(3)
-    LP_TCASE(4)
-    LP_TCASE(5)
-    LP_TCASE(6)
-    LP_TCASE(7)
-#undef LP_TCASE
+#define LP_LCASE3(M) LP_LCASE(M, 0) LP_LCASE(M, 1) LP_LCASE(M, 2)
+    LP_LCASE(0, 0)
+    LP_LCASE3(1)
+    LP_LCASE3(2)
+    LP_LCASE3(3)
+    LP_LCASE3(4)
+    LP_LCASE3(5)
+    LP_LCASE3(6)
+    LP_LCASE3(7)
+#undef LP_LCASE3
+#undef LP_LCASE
     default:
       return cudaErrorInvalidValue;
   }

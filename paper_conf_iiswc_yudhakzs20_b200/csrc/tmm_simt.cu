@@ -32,12 +32,12 @@ __device__ __forceinline__ float to_f<float>(float v) { return v; }
 template <>
 __device__ __forceinline__ float to_f<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
 
-template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK>
+template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE>
 __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
                                                             const TIn* __restrict__ B, int64_t ldb,
                                                             TOut* __restrict__ C, int64_t ldc, int64_t K,
                                                             int64_t Q, int64_t R, uint32_t* __restrict__ ck,
-                                                            int store, int64_t rid_offset,
+                                                            int64_t rid_offset,
                                                             const int64_t* __restrict__ list,
                                                             const int64_t* __restrict__ d_n) {
   static_assert((BM / UM) * (BN / UN) == kThreads, "256 threads");
@@ -154,7 +154,7 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
         for (int w = 1; w < kThreads / 32; ++w) r = combine(r, warp_rec[w]);
         uint32_t words[3];
         record_words<MASK>(r, (uint64_t)BM * BN * ES, words);
-        store_record<MASK>(ck, store, rid, (uint32_t)(rid + rid_offset), words);
+        store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
       }
     }
   }
@@ -169,20 +169,23 @@ cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
   const TIn* A = (const TIn*)a.A;
   const TIn* B = (const TIn*)a.B;
   TOut* C = (TOut*)a.C;
-  switch (a.mask) {
-#define LP_SCASE(M)                                                                                            \
-  case M:                                                                                                      \
-    tmm_simt_kernel<TIn, TOut, BM, BN, UM, UN, M><<<(unsigned)grid, kThreads, 0, st>>>(                        \
-        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.hash.store, a.rid_offset, a.list, a.d_n);             \
+  const int sk = a.mask ? a.hash.store : 0;
+  switch (a.mask * 3 + sk) {
+#define LP_SCASE(M, S)                                                                                         \
+  case M * 3 + S:                                                                                              \
+    tmm_simt_kernel<TIn, TOut, BM, BN, UM, UN, M, S><<<(unsigned)grid, kThreads, 0, st>>>(                     \
+        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.rid_offset, a.list, a.d_n);                           \
     break;
-    LP_SCASE(0)
-    LP_SCASE(1)
-    LP_SCASE(2)
-    LP_SCASE(3)
-    LP_SCASE(4)
-    LP_SCASE(5)
-    LP_SCASE(6)
-    LP_SCASE(7)
+#define LP_SCASE3(M) LP_SCASE(M, 0) LP_SCASE(M, 1) LP_SCASE(M, 2)
+    LP_SCASE(0, 0)
+    LP_SCASE3(1)
+    LP_SCASE3(2)
+    LP_SCASE3(3)
+    LP_SCASE3(4)
+    LP_SCASE3(5)
+    LP_SCASE3(6)
+    LP_SCASE3(7)
+#undef LP_SCASE3
 #undef LP_SCASE
     default:
       return cudaErrorInvalidValue;

@@ -33,6 +33,8 @@
 
 #include "lp_device.cuh"
 #include "lp_internal.h"
+#include "lp_ptx.cuh"
+#include "lp_tma.h"
 
 namespace lp {
 namespace {
@@ -52,40 +54,6 @@ struct TcCfg {
   static constexpr int kTmemCols = 2 * BN;                 // two accumulators
   static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*barriers etc.*/ + 1024 /*align slack*/;
 };
-
-// ---------------------------------------------------------------------------- PTX wrappers
-__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  const uint32_t a = smem_u32(bar);
-  uint32_t done;
-  do {
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-        "selp.u32 %0, 1, 0, p;\n\t}"
-        : "=r"(done)
-        : "r"(a), "r"(parity)
-        : "memory");
-  } while (!done);
-}
-
-__device__ __forceinline__ void tma_load_2d(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
-          smem_u32(dst)),
-      "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
-      : "memory");
-}
 
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -170,10 +138,10 @@ struct TileSrc {
   }
 };
 
-template <typename OutT, uint32_t MASK, int REG, int BN>
+template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
 __global__ void __launch_bounds__(kThreads, 1)
     tmm_tc_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
-                  OutT* __restrict__ C, int64_t ldc, int64_t K, TileSrc src, uint32_t* __restrict__ ck, int store) {
+                  OutT* __restrict__ C, int64_t ldc, int64_t K, TileSrc src, uint32_t* __restrict__ ck) {
   using Cfg = TcCfg<BN>;
   constexpr int S = Cfg::kStages;
   constexpr int ES = (int)sizeof(OutT);
@@ -338,7 +306,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               const int64_t rid = p * src.Qr + q;
               uint32_t words[3];
               record_words<MASK>(rec, (uint64_t)32 * 32 * ES, words);
-              store_record<MASK>(ck, store, rid, (uint32_t)(rid + src.rid_offset), words);
+              store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + src.rid_offset), words);
             }
             part = CkPartial<MASK>();
           } else if ((ch & 3) == 3) {
@@ -363,7 +331,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           const int64_t rid = mb * src.Qr + nb * (BN / 128) + j;
           uint32_t words[3];
           record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
-          store_record<MASK>(ck, store, rid, (uint32_t)(rid + src.rid_offset), words);
+          store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + src.rid_offset), words);
         }
       }
       if (++acc == 2) {
@@ -384,33 +352,10 @@ __global__ void __launch_bounds__(kThreads, 1)
 }
 
 // ---------------------------------------------------------------------------- host side
-typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
-                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
-                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
-
-PFN_encodeTiled get_encode() {
-  static PFN_encodeTiled fn = nullptr;
-  if (!fn) {
-    void* p = nullptr;
-    cudaDriverEntryPointQueryResult q;
-    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
-        q == cudaDriverEntryPointSuccess)
-      fn = (PFN_encodeTiled)p;
-  }
-  return fn;
-}
-
 bool make_map_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
                  uint32_t box_inner, uint32_t box_outer) {
-  PFN_encodeTiled enc = get_encode();
-  if (!enc) return false;
-  cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {ld_elems * 2};
-  cuuint32_t box[2] = {box_inner, box_outer};
-  cuuint32_t es[2] = {1, 1};
-  return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
-             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+  return tma_map_2d(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, base, inner, outer, ld_elems, box_inner, box_outer,
+                    CU_TENSOR_MAP_SWIZZLE_128B);
 }
 
 template <typename OutT, int REG, int BN>
@@ -436,23 +381,26 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   if (grid < 1) grid = 1;
   const int smem = Cfg::kSmemBytes;
   cudaError_t e = cudaSuccess;
-  switch (a.mask) {
-#define LP_TC_CASE(M)                                                                                       \
-  case M: {                                                                                                 \
-    auto kfn = tmm_tc_kernel<OutT, M, REG, BN>;                                                            \
+  const int sk = a.mask ? a.hash.store : 0;
+  switch (a.mask * 3 + sk) {
+#define LP_TC_CASE(M, S)                                                                                    \
+  case M * 3 + S: {                                                                                         \
+    auto kfn = tmm_tc_kernel<OutT, M, REG, BN, S>;                                                         \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
     if (e != cudaSuccess) return e;                                                                         \
-    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, src, a.ck, a.hash.store);  \
+    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, src, a.ck);                \
     break;                                                                                                  \
   }
-    LP_TC_CASE(0)
-    LP_TC_CASE(1)
-    LP_TC_CASE(2)
-    LP_TC_CASE(3)
-    LP_TC_CASE(4)
-    LP_TC_CASE(5)
-    LP_TC_CASE(6)
-    LP_TC_CASE(7)
+#define LP_TC_CASE3(M) LP_TC_CASE(M, 0) LP_TC_CASE(M, 1) LP_TC_CASE(M, 2)
+    LP_TC_CASE(0, 0)
+    LP_TC_CASE3(1)
+    LP_TC_CASE3(2)
+    LP_TC_CASE3(3)
+    LP_TC_CASE3(4)
+    LP_TC_CASE3(5)
+    LP_TC_CASE3(6)
+    LP_TC_CASE3(7)
+#undef LP_TC_CASE3
 #undef LP_TC_CASE
     default:
       return cudaErrorInvalidValue;
