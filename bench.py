@@ -60,6 +60,15 @@ WORKLOADS = {
                               cksum="mod|xor", frac=0.05, store="quad_cas", weak=False),
     "tmm16384_quad_lock": dict(kind="tmm", M=16384, N=16384, K=16384, in_dt="bf16", out_dt="bf16", region=128,
                                cksum="mod|xor", frac=0.05, store="quad_lock", weak=False),
+    "tmm16384_r32_array": dict(kind="tmm", M=16384, N=16384, K=16384, in_dt="bf16", out_dt="bf16", region=32,
+                               cksum="mod|xor", frac=0.05, store="array", weak=False),
+    "tmm16384_r32_quad_cas": dict(kind="tmm", M=16384, N=16384, K=16384, in_dt="bf16", out_dt="bf16", region=32,
+                                  cksum="mod|xor", frac=0.05, store="quad_cas", weak=False),
+    "tmm16384_r32_quad_lock": dict(kind="tmm", M=16384, N=16384, K=16384, in_dt="bf16", out_dt="bf16", region=32,
+                                   cksum="mod|xor", frac=0.05, store="quad_lock", weak=False),
+    # BASELINE configs[1] fp32 variant: the SIMT fp32 body (paper-shaped), 128x128 regions
+    "tmm8192_f32_simt": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="f32", out_dt="f32", region=128,
+                             cksum="mod|xor", frac=0.05, store="array", weak=True),
     # BASELINE configs[4]: 65536^3 bf16 region-sharded across ranks (strong scaling)
     "tmm65536_bf16": dict(kind="tmm", M=65536, N=65536, K=65536, in_dt="bf16", out_dt="bf16", region=128,
                           cksum="mod|xor", frac=0.05, store="array", weak=False),
@@ -328,6 +337,12 @@ def run_ours(args):
         (tp if i % 2 == 0 else tu).append(e0.elapsed_time(e1))
     t_prot, t_unprot = report.median(tp), report.median(tu)
     clocks = clk.stop()
+    # hash-store statistics of one fresh protected run (collisions = sum of extra probes, Table II analog)
+    d_stats = torch.zeros(2, dtype=torch.int64, device=dev)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    h.stats(wl, ck, d_stats)
+    hash_stats = [int(x) for x in d_stats.tolist()]
     clocks["window"] = "warm-up + timed steps + validate/overhead reps"
     assert torch.equal(out_twin, out), "protected and unprotected twin outputs differ"
 
@@ -417,6 +432,8 @@ def run_ours(args):
             "t_recovery_phase_ms": round(sum_vr / args.steps, 4),
             "n_failed_per_step": n_failed,
             "n_failed_after_recover": n_after,
+            "hash_collisions": hash_stats[0] if W["store"] != "array" else None,
+            "hash_error": hash_stats[1] if W["store"] != "array" else None,
             "bytes_recovery_phase": int(bytes_vr_total),
             "roofline": roof,
             "roofline_validate": {"bound": "hbm", "kernel": "validate_kernel", "achieved": round(vach, 1),

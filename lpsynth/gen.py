@@ -37,19 +37,20 @@ def splitmix64(z: np.ndarray) -> np.ndarray:
         return z ^ (z >> np.uint64(31))
 
 
-def raw(seed: int, rows: int, cols: int, row0: int = 0, ncols_global: int | None = None) -> np.ndarray:
-    """uint64 x for rows [row0, row0+rows) x cols [0, cols) of a matrix with ncols_global columns."""
+def raw(seed: int, rows: int, cols: int, row0: int = 0, ncols_global: int | None = None,
+        col0: int = 0) -> np.ndarray:
+    """uint64 x for rows [row0, row0+rows) x cols [col0, col0+cols) of a matrix with ncols_global columns."""
     ncg = cols if ncols_global is None else ncols_global
     r = np.arange(row0, row0 + rows, dtype=np.uint64)[:, None]
-    c = np.arange(cols, dtype=np.uint64)[None, :]
+    c = np.arange(col0, col0 + cols, dtype=np.uint64)[None, :]
     with np.errstate(over="ignore"):
         state = np.uint64(seed) * GOLDEN + r * np.uint64(ncg) + c
     return splitmix64(state)
 
 
 def values_f32(seed: int, rows: int, cols: int, kind: str = "uniform", row0: int = 0,
-               ncols_global: int | None = None) -> np.ndarray:
-    x = raw(seed, rows, cols, row0, ncols_global)
+               ncols_global: int | None = None, col0: int = 0) -> np.ndarray:
+    x = raw(seed, rows, cols, row0, ncols_global, col0)
     if kind == "uniform":
         return ((x >> np.uint64(40)).astype(np.float64) * 2.0 ** -23 - 1.0).astype(np.float32)
     if kind == "int5":
@@ -67,17 +68,18 @@ def f32_to_bf16_bits(v: np.ndarray) -> np.ndarray:
 
 
 def generate(seed: int, rows: int, cols: int, kind: str, dtype: str, row0: int = 0,
-             ncols_global: int | None = None) -> np.ndarray:
-    """Host copy of the synthetic matrix. f32 -> float32, bf16 -> uint16 bits, u32 -> uint32."""
+             ncols_global: int | None = None, col0: int = 0) -> np.ndarray:
+    """Host copy of the synthetic matrix (block at row0/col0 of a matrix with ncols_global columns).
+    f32 -> float32, bf16 -> uint16 bits, u32 -> uint32."""
     if kind == "bits":
-        x = raw(seed, rows, cols, row0, ncols_global)
+        x = raw(seed, rows, cols, row0, ncols_global, col0)
         bits = (x & np.uint64(0xFFFFFFFF)).astype(np.uint32)
         if dtype == "u32" or dtype == "f32":
             return bits if dtype == "u32" else bits.view(np.float32)
         if dtype == "bf16":
             return (bits & np.uint32(0xFFFF)).astype(np.uint16)
         raise ValueError(dtype)
-    v = values_f32(seed, rows, cols, kind, row0, ncols_global)
+    v = values_f32(seed, rows, cols, kind, row0, ncols_global, col0)
     if dtype == "f32":
         return v
     if dtype == "bf16":

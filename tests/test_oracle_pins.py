@@ -334,3 +334,9 @@ def test_synth_value_ranges_and_shard_invariance():
     full = gen.generate(3, 32, 48, "uniform", "bf16")
     shard = gen.generate(3, 8, 48, "uniform", "bf16", row0=16, ncols_global=48)
     assert np.array_equal(full[16:24], shard)
+
+
+def test_synth_column_block_matches_full():
+    full = gen.generate(4, 16, 40, "int5", "bf16")
+    blk = gen.generate(4, 16, 8, "int5", "bf16", ncols_global=40, col0=24)
+    assert np.array_equal(full[:, 24:32], blk)
