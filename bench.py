@@ -262,7 +262,7 @@ def run_ours(args):
         counts[0:1].copy_(d_n)
         counts[1:2].copy_(d_n)
         shard.allreduce_counts(counts[0:2])
-        h.recover(wl, out, ck, failed, d_n)
+        h.recover(wl, out, ck, failed, d_n, ws)
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[2:3].copy_(d_n)
         shard.allreduce_counts(counts[2:3])
@@ -302,7 +302,7 @@ def run_ours(args):
     h.validate(wl, out, ck, failed, d_n, ws)
     k_local = int(d_n.item())
     rec_rids = (failed[:k_local].cpu().numpy() - sh.rid_offset).tolist()
-    h.recover(wl, out, ck, failed, d_n)
+    h.recover(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     bytes_vr_local = 2 * (out_bytes + ck_bytes) + recover_bytes(rec_rids)
     sum_vr = sum(t_vr)
@@ -365,7 +365,7 @@ def run_ours(args):
         counts[0:1].copy_(d_n)
         counts[1:2].copy_(d_n)
         shard.allreduce_counts(counts[0:2])
-        h.recover(wl, out, ck, failed, d_n)
+        h.recover(wl, out, ck, failed, d_n, ws)
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[2:3].copy_(d_n)
         shard.allreduce_counts(counts[2:3])

@@ -160,9 +160,13 @@ LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* o
 
 /* Selective re-execution (eager recovery, L85): re-runs the region body for
  * exactly the regions in failed_list[0 .. *d_n_failed) (global rids of this
- * shard), rewriting their data AND records.  The count is read on the device. */
+ * shard), rewriting their data AND records.  The count is read on the device.
+ * `workspace` (optional, lp_workspace_bytes bytes, may be NULL) lets liblp
+ * de-duplicate failed regions that share one tensor-core tile (32x32 regions:
+ * 16 per 128x128 tile) so each tile is recomputed once; with NULL every listed
+ * region recomputes its tile (same final state, more work). */
 LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
-                     const int64_t* d_n_failed, lp_stream_t stream);
+                            const int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 
 /* Records of every region of `out` (uint32 [R][selem], order MOD, XOR, ADLER)
  * without comparing -- for parity tests against the oracle. */

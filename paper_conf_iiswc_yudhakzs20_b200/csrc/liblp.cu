@@ -151,14 +151,32 @@ size_t cksum_bytes(const lp_ctx* h, const lp::RegionGeom& g) {
   return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R) * 4u * (size_t)(1 + h->selem);
 }
 
-size_t workspace_bytes(const lp::RegionGeom& g) {
-  const size_t flags = ((size_t)g.R + 255) & ~(size_t)255;
-  return flags + lp::compact_scratch_bytes(g.R) + 256;
+// 128x128 tensor-core tiles covering the output (recovery de-duplication of 32x32 regions)
+int64_t dedupe_tiles(const lp::RegionGeom& g) { return (g.RM == 32 && g.RN == 32) ? (g.M / 128) * (g.N / 128) : 0; }
+
+struct WsLayout {
+  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, total;
+};
+
+WsLayout ws_layout(const lp::RegionGeom& g) {
+  auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
+  const int64_t T = dedupe_tiles(g);
+  WsLayout w;
+  w.flags = 0;
+  w.counts = al((size_t)g.R);
+  w.tile_flags = w.counts + al(lp::compact_scratch_bytes(g.R));
+  w.tile_counts = w.tile_flags + al((size_t)T);
+  w.tile_list = w.tile_counts + al(lp::compact_scratch_bytes(T));
+  w.d_ntiles = w.tile_list + al((size_t)T * 8);
+  w.total = w.d_ntiles + 256;
+  return w;
 }
+
+size_t workspace_bytes(const lp::RegionGeom& g) { return ws_layout(g).total; }
 
 // Body dispatch shared by run_protected and recover (list = null for a full run).
 lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
-                   const int64_t* list, const int64_t* d_n, cudaStream_t st) {
+                   const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr) {
   const lp::HashInfo hi = hash_info(h, g);
   if (wl->kind == LP_WL_STENCIL5) {
     if (!lp::stencil_supported(g.RM, g.RN)) return fail(LP_ERR_UNSUPPORTED, "stencil supports 128x128 regions");
@@ -206,6 +224,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.rid_offset = g.rid_offset;
   a.list = list;
   a.d_n = d_n;
+  a.list_is_tiles = 0;
   a.sm_count = h->sm_count;
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
@@ -216,6 +235,18 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
       return fail(LP_ERR_UNSUPPORTED,
                   "tcgen05 body needs bf16 input, m%%128 == 0, n%%256 == 0, k%%64 == 0, region 128x128 or 32x32 "
                   "dividing the 128x256 tile, 16-B aligned pitches");
+    if (list && workspace && dedupe_tiles(g) > 0) {
+      // several failed 32x32 regions may share one 128x128 tile: recompute each tile once
+      const WsLayout w = ws_layout(g);
+      uint8_t* ws = (uint8_t*)workspace;
+      cudaError_t e0 = lp::launch_tiles_of_failed(g, list, d_n, ws + w.tile_flags, dedupe_tiles(g),
+                                                  (uint32_t*)(ws + w.tile_counts), (int64_t*)(ws + w.tile_list),
+                                                  (int64_t*)(ws + w.d_ntiles), st);
+      if (e0 != cudaSuccess) return cuda_fail(e0, "tile de-duplication");
+      a.list = (const int64_t*)(ws + w.tile_list);
+      a.d_n = (const int64_t*)(ws + w.d_ntiles);
+      a.list_is_tiles = 1;
+    }
     const char* why = nullptr;
     cudaError_t e = lp::launch_tmm_tc(a, st, &why);
     if (e != cudaSuccess) return why ? fail(LP_ERR_CUDA, "tcgen05 launch: %s", why) : cuda_fail(e, "tcgen05 launch");
@@ -337,8 +368,9 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
   }
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
-  uint8_t* flags = (uint8_t*)workspace;
-  uint32_t* counts = (uint32_t*)((uint8_t*)workspace + (((size_t)g.R + 255) & ~(size_t)255));
+  const WsLayout w = ws_layout(g);
+  uint8_t* flags = (uint8_t*)workspace + w.flags;
+  uint32_t* counts = (uint32_t*)((uint8_t*)workspace + w.counts);
   cudaStream_t st = (cudaStream_t)stream;
   cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st);
   if (e != cudaSuccess) return cuda_fail(e, "validate launch");
@@ -347,7 +379,7 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
 }
 
 lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
-                     const int64_t* d_n_failed, lp_stream_t stream) {
+                     const int64_t* d_n_failed, void* workspace, lp_stream_t stream) {
   lp::RegionGeom g;
   lp_status s = check_wl(h, wl, &g);
   if (s) return s;
@@ -355,7 +387,8 @@ lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksu
   if (h->mask && !cksum) return fail(LP_ERR_INVALID_ARG, "null cksum");
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
-  return run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream);
+  if (workspace && !aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
+  return run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace);
 }
 
 lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,

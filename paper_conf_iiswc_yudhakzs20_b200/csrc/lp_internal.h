@@ -35,6 +35,10 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
                           const void* stale, const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed,
                           cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
+// failed 32x32 regions -> unique 128x128 tile ids (tile = (p/4)*(N/128) + q/4), ascending
+cudaError_t launch_tiles_of_failed(const RegionGeom& g, const int64_t* list, const int64_t* d_n, uint8_t* tile_flags,
+                                   int64_t T, uint32_t* block_counts, int64_t* tile_list, int64_t* d_ntiles,
+                                   cudaStream_t st);
 
 // ---- tmm_simt.cu : SIMT region body (CTA tile == region), paper-shaped
 struct TmmArgs {
@@ -53,6 +57,7 @@ struct TmmArgs {
   int64_t rid_offset;
   const int64_t* list;  // list mode (recovery) when non-null
   const int64_t* d_n;
+  int list_is_tiles;    // list holds 128x128 tile ids (de-duplicated recovery of 32x32 regions)
   int sm_count;
 };
 bool tmm_simt_supported(int RM, int RN, int in_bf16, int out_bf16);

@@ -221,6 +221,17 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
 }
 
 // ---------------------------------------------------------------------------
+__global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t* __restrict__ d_n,
+                                 int64_t rid_offset, int64_t Q, int64_t tiles_per_row, int per,
+                                 uint8_t* __restrict__ tile_flags) {
+  const int64_t n = *d_n;
+  for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t rid = list[i] - rid_offset;
+    const int64_t p = rid / Q, q = rid - p * Q;
+    tile_flags[(p / per) * tiles_per_row + q / per] = 1;  // idempotent plain store
+  }
+}
+
 __global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed) {
   HashHeader* h = reinterpret_cast<HashHeader*>(ck);
   h->cap = cap;
@@ -369,6 +380,22 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
   else LP_ICASE(3);
 #undef LP_ICASE
   return cudaGetLastError();
+}
+
+cudaError_t launch_tiles_of_failed(const RegionGeom& g, const int64_t* list, const int64_t* d_n, uint8_t* tile_flags,
+                                   int64_t T, uint32_t* block_counts, int64_t* tile_list, int64_t* d_ntiles,
+                                   cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(tile_flags, 0, (size_t)T, st);
+  if (e != cudaSuccess) return e;
+  const int per = 128 / g.RM;
+  tile_mark_kernel<<<(unsigned)(g.R < 148 * 4 * 256 ? (g.R + 255) / 256 : 148 * 4), 256, 0, st>>>(
+      list, d_n, g.rid_offset, g.Q, g.N / 128, per, tile_flags);
+  e = cudaGetLastError();
+  if (e != cudaSuccess) return e;
+  RegionGeom tg = g;
+  tg.R = T;
+  tg.rid_offset = 0;
+  return launch_compact(tg, tile_flags, block_counts, tile_list, d_ntiles, st);
 }
 
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st) {

@@ -124,11 +124,17 @@ struct TileSrc {
   int64_t rid_offset;
   int64_t Qr;                 // regions per output row band
   int reg;                    // region edge (32 or 128)
+  int list_is_tiles;          // list holds tile ids (already de-duplicated)
   __device__ __forceinline__ int64_t count() const { return list ? *d_n : num_m * num_n; }
   template <int BN>
   __device__ __forceinline__ void coords(int64_t t, int64_t& mb, int64_t& nb) const {
     if (!list) {
       tile_coords(t, num_m, num_n, mb, nb);
+      return;
+    }
+    if (list_is_tiles) {
+      mb = list[t] / num_n;
+      nb = list[t] - mb * num_n;
       return;
     }
     const int64_t rid = list[t] - rid_offset;
@@ -375,6 +381,7 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   src.rid_offset = a.rid_offset;
   src.Qr = a.N / REG;
   src.reg = REG;
+  src.list_is_tiles = a.list_is_tiles;
   const int64_t R = (a.M / REG) * (a.N / REG);
   int64_t grid = a.list ? (R < a.sm_count ? R : a.sm_count) : src.num_m * src.num_n;
   if (grid > a.sm_count) grid = a.sm_count;
@@ -410,8 +417,9 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
 
 template <typename OutT, int REG>
 cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
-  // list mode with 128x128 regions re-executes exactly one region per tile (BN = 128)
-  const bool bn256 = (a.N % 256 == 0) && !(a.list && REG == 128);
+  // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
+  // 16 32x32 regions of a de-duplicated tile
+  const bool bn256 = (a.N % 256 == 0) && !a.list;
   return bn256 ? launch_cfg<OutT, REG, 256>(a, st, why) : launch_cfg<OutT, REG, 128>(a, st, why);
 }
 

@@ -92,7 +92,7 @@ def lib():
             "lp_cksum_init": [P, pw, P, P],
             "lp_run_protected": [P, pw, P, P, P],
             "lp_validate": [P, pw, P, P, P, I64, P, P, P],
-            "lp_recover": [P, pw, P, P, P, P, P],
+            "lp_recover": [P, pw, P, P, P, P, P, P],
             "lp_region_checksums": [P, pw, P, P, P],
             "lp_inject": [P, pw, P, P, P, P, I64, U32, U64, P],
             "lp_stats": [P, pw, P, P, P],
@@ -244,9 +244,9 @@ class LP:
         _check(lib().lp_validate(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), failed.numel(),
                                  _ptr(d_n), _ptr(workspace), _stream(stream)))
 
-    def recover(self, wl, out, ck, failed, d_n, stream=None):
+    def recover(self, wl, out, ck, failed, d_n, workspace=None, stream=None):
         _check(lib().lp_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), _ptr(d_n),
-                                _stream(stream)))
+                                _ptr(workspace), _stream(stream)))
 
     def region_checksums(self, wl, out, records, stream=None):
         _check(lib().lp_region_checksums(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(records), _stream(stream)))

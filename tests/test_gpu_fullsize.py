@@ -84,7 +84,7 @@ def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, globa
                                           h.mask, rid_offset=rid0)
     assert np.array_equal(got_failed, exp_failed)
     assert set(got_failed.tolist()) <= set(inj.cpu().numpy().tolist()) and nf > 0
-    h.recover(wl, out, ck, failed, d_n)
+    h.recover(wl, out, ck, failed, d_n, ws)
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0
@@ -108,6 +108,11 @@ def test_c2_tmm8192_f32_out():
 def test_c3_tmm16384_quad_cas_full():
     """configs[2]: 16384^3, lock-free quadratic-probing store; every rid looked up in the GPU's table."""
     _tmm_full(16384, 16384, 16384, 128, "mod|xor", "quad_cas", "int5", "bf16", nsample=2, seed=5)
+
+
+def test_c3_tmm16384_r32_array_full():
+    """configs[2] with 32x32 regions (R = 262144): records of every region, de-duplicated tile recovery."""
+    _tmm_full(16384, 16384, 16384, 32, "mod|xor", "array", "int5", "bf16", nsample=4, seed=9)
 
 
 def test_c5_tmm65536_rank3_of_8_shard():
@@ -152,7 +157,7 @@ def test_c4_stencil32768_full():
         exp_failed = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * 2], 128, 128, 3)
         assert np.array_equal(failed[:nf].cpu().numpy(), exp_failed)
         assert nf == inj.numel()
-        h.recover(wl, out, ck, failed, d_n)
+        h.recover(wl, out, ck, failed, d_n, ws)
         h.validate(wl, out, ck, failed, d_n, ws)
         torch.cuda.synchronize()
         assert int(d_n.item()) == 0 and torch.equal(out, gold_dev)

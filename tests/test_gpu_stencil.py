@@ -46,7 +46,7 @@ def stencil_cycle(H, W, kind, mask, mode, frac, seed=2, store="array"):
     assert set(got.tolist()) <= set(inj.cpu().numpy().tolist())
     if mode == "stale_region":
         assert nf == inj.numel()
-    h.recover(wl, out, ck, failed, d_n)
+    h.recover(wl, out, ck, failed, d_n, ws)
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0

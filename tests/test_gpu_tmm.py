@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
-              store="array", check_values=True):
+              store="array", check_values=True, recover_ws=True):
     h = lp.LP(RM, RN, cksum=mask, store=store, body=body)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
@@ -81,7 +81,7 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     if mode in ("bitflip",):
         assert set(got_failed.tolist()) == injected          # a bit flip always changes MOD and XOR
     # (8) recover -> out == golden byte-for-byte, records == golden, re-validate == 0
-    h.recover(wl, out, ck, failed, d_n)
+    h.recover(wl, out, ck, failed, d_n, ws if recover_ws else None)
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0
@@ -139,6 +139,13 @@ def test_simt_hash_stores(store):
 @pytest.mark.parametrize("reg", [128, 32])
 def test_tc_cycle(kind, out_dt, reg):
     run_cycle(256, 512, 256, reg, reg, "bf16", out_dt, kind, "mod|xor", "tcgen05", mode="stale_words", frac=0.2)
+
+
+@pytest.mark.parametrize("recover_ws", [True, False])
+def test_tc_r32_recovery_tile_dedup(recover_ws):
+    """32x32 regions: many failed regions share a 128x128 tile; with the workspace each tile is recomputed once."""
+    run_cycle(512, 768, 128, 32, 32, "bf16", "bf16", "uniform", "mod|xor", "tcgen05", mode="stale_region",
+              frac=0.3, recover_ws=recover_ws)
 
 
 @pytest.mark.parametrize("mask", ["mod", "xor", "adler", "mod|xor|adler"])
