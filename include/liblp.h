@@ -106,8 +106,13 @@ typedef struct {
   int32_t device;             /* CUDA device ordinal */
   int32_t body;               /* lp_body */
   uint32_t hash_seed;         /* seed of the hash function for QUAD stores (Reading R14) */
-  int32_t reserved;
+  uint32_t flags;             /* OR of lp_config_flags (A/B switches); 0 = defaults */
 } lp_config_t;
+
+/* lp_config_t.flags */
+typedef enum {
+  LP_FLAG_TC_1CTA = 1u /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
+} lp_config_flags;
 
 typedef struct {
   int32_t kind;      /* lp_wl_kind */

@@ -225,6 +225,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.list = list;
   a.d_n = d_n;
   a.list_is_tiles = 0;
+  a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
   a.sm_count = h->sm_count;
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
@@ -276,6 +277,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->store != LP_STORE_ARRAY && cfg->cksum == 0) return fail(LP_ERR_INVALID_ARG, "a hash store needs a checksum");
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
+  if (cfg->flags & ~(uint32_t)LP_FLAG_TC_1CTA) return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((int64_t)cfg->region_m * cfg->region_n * 4 > (16ll << 20))
     return fail(LP_ERR_UNSUPPORTED, "regions larger than 16 MiB are not supported");
   lp_ctx* h = new lp_ctx();

@@ -144,6 +144,95 @@ struct TileSrc {
   }
 };
 
+// ---------------------------------------------------------------------------- epilogue pieces
+// Store one 128-row x BN-column accumulator (this warp's 32 TMEM lanes) to C and
+// fold the exact stored words into the LP checksum (L192).  m128 = index of the
+// 128-row block of C, n0 = first column.  32x32 regions are finished here (one
+// warp-wide redux per checksum, Listing 4); 128x128 regions leave one partial
+// per warp in srec for epi_finish_128.
+template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
+__device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, int64_t ldc, int64_t m128, int64_t n0,
+                                          int wq, int lane, CkRecord* srec_acc, uint32_t* __restrict__ ck, int64_t Qr,
+                                          int64_t rid_offset) {
+  constexpr int ES = (int)sizeof(OutT);
+  constexpr int NCH = BN / 32;
+  const int row_in_tile = wq * 32 + lane;
+  OutT* crow = C + (m128 * kBM + row_in_tile) * ldc + n0;
+  CkPartial<MASK> part;
+#pragma unroll 1
+  for (int ch = 0; ch < NCH; ++ch) {
+    uint32_t r[32];
+    LP_TMEM_LD32(t_row + ch * 32, r);
+    tc_wait_ld();
+    if constexpr (ES == 2) {
+      uint32_t w[16];
+#pragma unroll
+      for (int i = 0; i < 16; ++i) {
+        __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
+        w[i] = *reinterpret_cast<uint32_t*>(&h);  // even column in the low half (Reading R6)
+      }
+      uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+      if constexpr (MASK != 0) {
+        // byte position of word 0 of this chunk inside its region's stream
+        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+                                         : (uint32_t)(lane * 32 * ES + 1);
+#pragma unroll
+        for (int i = 0; i < 16; ++i) part.add(w[i], pos0 + 4 * i);
+      }
+    } else {
+      uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
+#pragma unroll
+      for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
+      if constexpr (MASK != 0) {
+        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+                                         : (uint32_t)(lane * 32 * ES + 1);
+#pragma unroll
+        for (int i = 0; i < 32; ++i) part.add(r[i], pos0 + 4 * i);
+      }
+    }
+    if constexpr (MASK != 0) {
+      if constexpr (REG == 32) {
+        // one 32x32 region = this warp's 32 rows x this 32-column chunk
+        const CkRecord rec = warp_reduce<MASK>(part);
+        if (lane == 0) {
+          const int64_t p = m128 * (kBM / 32) + wq, q = (n0 + ch * 32) / 32;
+          const int64_t rid = p * Qr + q;
+          uint32_t words[3];
+          record_words<MASK>(rec, (uint64_t)32 * 32 * ES, words);
+          store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+        }
+        part = CkPartial<MASK>();
+      } else if ((ch & 3) == 3) {
+        // end of a 128-column region: warp partial -> shared slot
+        const CkRecord rec = warp_reduce<MASK>(part);
+        if (lane == 0) srec_acc[(ch / 4) * 4 + wq] = rec;
+        part = CkPartial<MASK>();
+      }
+    }
+  }
+}
+
+// 128x128 regions: after the epilogue warps' named barrier, combine the 4 warp
+// partials of each region (Listing 3's block combine) and store the record.
+template <typename OutT, uint32_t MASK, int BN, int STORE>
+__device__ __forceinline__ void epi_finish_128(int warp, int lane, const CkRecord* srec_acc, uint32_t* __restrict__ ck,
+                                               int64_t m128, int64_t n0, int64_t Qr, int64_t rid_offset) {
+  constexpr int ES = (int)sizeof(OutT);
+  named_bar_epi();
+  if (warp == kEpiWarp0 && lane < BN / 128) {
+    const int j = lane;
+    CkRecord rr = srec_acc[j * 4 + 0];
+#pragma unroll
+    for (int w = 1; w < 4; ++w) rr = combine(rr, srec_acc[j * 4 + w]);
+    const int64_t rid = m128 * Qr + n0 / 128 + j;
+    uint32_t words[3];
+    record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
+    store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+  }
+}
+
 template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
 __global__ void __launch_bounds__(kThreads, 1)
     tmm_tc_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
@@ -259,7 +348,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else {
     // ===================== epilogue (4 warps, 128 threads) =====================
     const int wq = warp & 3;              // TMEM lane quarter owned by this warp
-    const int row_in_tile = wq * 32 + lane;
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -268,78 +356,15 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
-      OutT* crow = C + (mb * kBM + row_in_tile) * ldc + nb * BN;
-      CkPartial<MASK> part;
-#pragma unroll 1
-      for (int ch = 0; ch < NCH; ++ch) {
-        uint32_t r[32];
-        LP_TMEM_LD32(t_row + ch * 32, r);
-        tc_wait_ld();
-        if constexpr (ES == 2) {
-          uint32_t w[16];
-#pragma unroll
-          for (int i = 0; i < 16; ++i) {
-            __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
-            w[i] = *reinterpret_cast<uint32_t*>(&h);
-          }
-          uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
-          if constexpr (MASK != 0) {
-            // byte position of word 0 of this chunk inside its region's stream
-            const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
-                                             : (uint32_t)(lane * 32 * ES + 1);
-#pragma unroll
-            for (int i = 0; i < 16; ++i) part.add(w[i], pos0 + 4 * i);
-          }
-        } else {
-          uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
-#pragma unroll
-          for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
-          if constexpr (MASK != 0) {
-            const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
-                                             : (uint32_t)(lane * 32 * ES + 1);
-#pragma unroll
-            for (int i = 0; i < 32; ++i) part.add(r[i], pos0 + 4 * i);
-          }
-        }
-        if constexpr (MASK != 0) {
-          if constexpr (REG == 32) {
-            // one 32x32 region = this warp's 32 rows x this 32-column chunk
-            const CkRecord rec = warp_reduce<MASK>(part);
-            if (lane == 0) {
-              const int64_t p = mb * (kBM / 32) + wq, q = (nb * BN + ch * 32) / 32;
-              const int64_t rid = p * src.Qr + q;
-              uint32_t words[3];
-              record_words<MASK>(rec, (uint64_t)32 * 32 * ES, words);
-              store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + src.rid_offset), words);
-            }
-            part = CkPartial<MASK>();
-          } else if ((ch & 3) == 3) {
-            // end of a 128-column region: warp partial -> smem slot
-            const CkRecord rec = warp_reduce<MASK>(part);
-            if (lane == 0) srec[(acc * (BN / 128) + ch / 4) * 4 + wq] = rec;
-            part = CkPartial<MASK>();
-          }
-        }
-      }
-      // all TMEM reads of this accumulator are complete (wait::ld above): release it
+      CkRecord* srec_acc = srec + acc * (BN / 128) * 4;
+      epi_store<OutT, MASK, REG, BN, STORE>(t_row, C, ldc, mb, nb * BN, wq, lane, srec_acc, ck, src.Qr,
+                                            src.rid_offset);
+      // all TMEM reads of this accumulator are complete (wait::ld): release it
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[acc]);
-      if constexpr (MASK != 0 && REG == 128) {
-        named_bar_epi();
-        if (warp == kEpiWarp0 && lane < BN / 128) {
-          const int j = lane;
-          CkRecord rr = srec[(acc * (BN / 128) + j) * 4 + 0];
-#pragma unroll
-          for (int w = 1; w < 4; ++w) rr = combine(rr, srec[(acc * (BN / 128) + j) * 4 + w]);
-          const int64_t rid = mb * src.Qr + nb * (BN / 128) + j;
-          uint32_t words[3];
-          record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
-          store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + src.rid_offset), words);
-        }
-      }
+      if constexpr (MASK != 0 && REG == 128)
+        epi_finish_128<OutT, MASK, BN, STORE>(warp, lane, srec_acc, ck, mb, nb * BN, src.Qr, src.rid_offset);
       if (++acc == 2) {
         acc = 0;
         acc_phase ^= 1;
@@ -354,6 +379,212 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
                  "r"((uint32_t)Cfg::kTmemCols)
                  : "memory");
+  }
+}
+
+// ---------------------------------------------------------------------------- CTA-pair kernel
+// Full (non-list) runs with M % 256 == 0 and N % 256 == 0 use a 2-SM CTA pair
+// (cluster of 2): one tcgen05.mma.cta_group::2 computes a 256x256x16 step with
+// A split by rows (128 per CTA) and B split by columns (128 per CTA), so each
+// SM stages only half of B: 32 KiB per stage, a 6-deep TMA ring, and half the
+// per-SM operand traffic of the 1-CTA 128x256 tile.  The leader CTA (rank 0)
+// owns the smem-full barriers (both CTAs' TMA complete_tx on it) and issues the
+// MMAs; commits multicast to both CTAs' barriers.  Each CTA's TMEM holds its
+// 128 rows x 256 fp32 columns, double-buffered, and its 4 epilogue warps run the
+// same LP epilogue as the 1-CTA kernel on its own 128 rows.
+constexpr int kStages2 = 6;
+constexpr int kA2Bytes = kBM * kBK * 2;   // 16 KiB: this CTA's 128 rows of A
+constexpr int kB2Bytes = kBK * 128 * 2;   // 16 KiB: this CTA's 128 columns of B
+constexpr int kStage2Bytes = kA2Bytes + kB2Bytes;
+constexpr int kSmem2Bytes = kStages2 * kStage2Bytes + 1024 + 1024;
+
+__device__ __forceinline__ uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+// shared::cluster address of the same variable in CTA rank 0 of the cluster
+__device__ __forceinline__ uint32_t mapa_rank0(const void* p) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(r) : "r"(smem_u32(p)));
+  return r;
+}
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap* map, uint32_t mbar_rank0, void* dst, int c0,
+                                                 int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
+      "%4}], [%2];" ::"r"(smem_u32(dst)),
+      "l"((uint64_t)map), "r"(mbar_rank0), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void tc_mma_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                            uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          smem_u32(bar)),
+      "h"((uint16_t)3)
+      : "memory");
+}
+
+template <typename OutT, uint32_t MASK, int REG, int STORE>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+    tmm_tc2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+                   OutT* __restrict__ C, int64_t ldc, int64_t K, int64_t num_m, int64_t num_n, int64_t Qr,
+                   int64_t rid_offset, uint32_t* __restrict__ ck) {
+  constexpr int BN = 256;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + kStages2 * kA2Bytes;
+  uint64_t* full = (uint64_t*)(smem + kStages2 * kStage2Bytes);
+  uint64_t* empty = full + kStages2;
+  uint64_t* tfull = empty + kStages2;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_holder = (uint32_t*)(tempty + 2);
+  CkRecord* srec = (CkRecord*)(tmem_holder + 4);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const int64_t pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&tmap_a);
+    prefetch_tmap(&tmap_b);
+    for (int s = 0; s < kStages2; ++s) {
+      mbar_init(&full[s], 2);   // one arrival per CTA's producer (+ both CTAs' TMA bytes), used in rank 0
+      mbar_init(&empty[s], 1);  // leader's MMA commit (multicast)
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&tfull[s], 1);
+      mbar_init(&tempty[s], 8);  // 4 epilogue warps x 2 CTAs, used in rank 0
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_holder)),
+                 "r"(512u)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_holder;
+  const int64_t ntiles = num_m * num_n;
+  const int nkb = (int)(K / kBK);
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int64_t t = pair; t < ntiles; t += npairs) {
+        int64_t mb, nb;
+        tile_coords(t, num_m, num_n, mb, nb);
+        const int m0 = (int)(mb * 256 + rank * 128), n0 = (int)(nb * 256 + rank * 128);
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          const uint32_t full0 = mapa_rank0(&full[stage]);
+          if (rank == 0)
+            mbar_expect_tx(&full[stage], 2 * kStage2Bytes);
+          else
+            mbar_arrive_remote(full0);
+          tma_load_2d_pair(&tmap_a, full0, sA + stage * kA2Bytes, kb * kBK, m0);
+          tma_load_2d_pair(&tmap_b, full0, sB + stage * kB2Bytes, n0, kb * kBK);
+          tma_load_2d_pair(&tmap_b, full0, sB + stage * kB2Bytes + kBK * 128, n0 + 64, kb * kBK);
+          if (++stage == kStages2) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {
+      // M = 256 (cta_group::2), N = 256
+      constexpr uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) |
+                                 ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int64_t t = pair; t < ntiles; t += npairs) {
+        mbar_wait(&tempty[acc], acc_phase ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_addr = smem_u32(sA + stage * kA2Bytes);
+          const uint32_t b_addr = smem_u32(sB + stage * kB2Bytes);
+#pragma unroll
+          for (int k = 0; k < kBK / kUmmaK; ++k) {
+            const uint64_t ad = smem_desc(a_addr + k * kUmmaK * 2, 16, 1024);
+            const uint64_t bd = smem_desc(b_addr + k * kUmmaK * 128, kBK * 128, 1024);
+            tc_mma_pair(d_tmem, ad, bd, idesc, (kb | k) ? 1u : 0u);
+          }
+          tc_commit_pair(&empty[stage]);
+          if (++stage == kStages2) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc_commit_pair(&tfull[acc]);
+        if (++acc == 2) {
+          acc = 0;
+          acc_phase ^= 1;
+        }
+      }
+    }
+  } else {
+    const int wq = warp & 3;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int64_t t = pair; t < ntiles; t += npairs) {
+      int64_t mb, nb;
+      tile_coords(t, num_m, num_n, mb, nb);
+      mbar_wait(&tfull[acc], acc_phase);
+      tc_fence_after();
+      const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
+      CkRecord* srec_acc = srec + acc * 2 * 4;
+      const int64_t m128 = mb * 2 + rank;
+      epi_store<OutT, MASK, REG, BN, STORE>(t_row, C, ldc, m128, nb * BN, wq, lane, srec_acc, ck, Qr, rid_offset);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) {
+        if (rank == 0)
+          mbar_arrive(&tempty[acc]);
+        else
+          mbar_arrive_remote(mapa_rank0(&tempty[acc]));
+      }
+      if constexpr (MASK != 0 && REG == 128)
+        epi_finish_128<OutT, MASK, BN, STORE>(warp, lane, srec_acc, ck, m128, nb * BN, Qr, rid_offset);
+      if (++acc == 2) {
+        acc = 0;
+        acc_phase ^= 1;
+      }
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync_all();  // the peer's remote arrivals and the leader's MMAs into both TMEMs are done
+  tc_fence_after();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(512u) : "memory");
   }
 }
 
@@ -416,7 +647,51 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
 }
 
 template <typename OutT, int REG>
+cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
+  CUtensorMap ma, mb;
+  if (!make_map_2d(&ma, a.A, (uint64_t)a.K, (uint64_t)a.M, (uint64_t)a.lda, kBK, kBM) ||
+      !make_map_2d(&mb, a.B, (uint64_t)a.N, (uint64_t)a.K, (uint64_t)a.ldb, 64, kBK)) {
+    *why = "cuTensorMapEncodeTiled failed";
+    return cudaErrorInvalidValue;
+  }
+  const int64_t num_m = a.M / 256, num_n = a.N / 256;
+  int64_t grid = 2 * num_m * num_n;
+  const int64_t cap = a.sm_count & ~1;
+  if (grid > cap) grid = cap;
+  if (grid < 2) grid = 2;
+  const int64_t Qr = a.N / REG;
+  const int sk = a.mask ? a.hash.store : 0;
+  cudaError_t e = cudaSuccess;
+  switch (a.mask * 3 + sk) {
+#define LP_TC2_CASE(M, S)                                                                                   \
+  case M * 3 + S: {                                                                                         \
+    auto kfn = tmm_tc2_kernel<OutT, M, REG, S>;                                                            \
+    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2Bytes);                \
+    if (e != cudaSuccess) return e;                                                                         \
+    kfn<<<(unsigned)grid, kThreads, kSmem2Bytes, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr,    \
+                                                       a.rid_offset, a.ck);                                 \
+    break;                                                                                                  \
+  }
+#define LP_TC2_CASE3(M) LP_TC2_CASE(M, 0) LP_TC2_CASE(M, 1) LP_TC2_CASE(M, 2)
+    LP_TC2_CASE(0, 0)
+    LP_TC2_CASE3(1)
+    LP_TC2_CASE3(2)
+    LP_TC2_CASE3(3)
+    LP_TC2_CASE3(4)
+    LP_TC2_CASE3(5)
+    LP_TC2_CASE3(6)
+    LP_TC2_CASE3(7)
+#undef LP_TC2_CASE3
+#undef LP_TC2_CASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+template <typename OutT, int REG>
 cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
+  if (!a.list && a.M % 256 == 0 && a.N % 256 == 0 && !a.force_1cta) return launch_pair<OutT, REG>(a, st, why);
   // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
   // 16 32x32 regions of a de-duplicated tile
   const bool bn256 = (a.N % 256 == 0) && !a.list;

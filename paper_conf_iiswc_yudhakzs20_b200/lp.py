@@ -26,6 +26,7 @@ STORE_ARRAY, STORE_QUAD_CAS, STORE_QUAD_LOCK = 0, 1, 2
 F32, BF16 = 0, 1
 WL_TMM, WL_STENCIL5 = 0, 1
 BODY_AUTO, BODY_SIMT, BODY_TCGEN05 = 0, 1, 2
+FLAG_TC_1CTA = 1
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
@@ -61,7 +62,7 @@ class LPError(RuntimeError):
 class Config(ctypes.Structure):
     _fields_ = [("region_m", ctypes.c_int32), ("region_n", ctypes.c_int32), ("cksum", ctypes.c_uint32),
                 ("store", ctypes.c_int32), ("device", ctypes.c_int32), ("body", ctypes.c_int32),
-                ("hash_seed", ctypes.c_uint32), ("reserved", ctypes.c_int32)]
+                ("hash_seed", ctypes.c_uint32), ("flags", ctypes.c_uint32)]
 
 
 class CWorkload(ctypes.Structure):
@@ -193,13 +194,15 @@ class LP:
     """One liblp handle: region shape + checksum type + store (lp_config)."""
 
     def __init__(self, region_m: int, region_n: int, cksum="mod|xor", store="array", device: int = 0,
-                 body="auto", hash_seed: int = 0x9747B28C):
+                 body="auto", hash_seed: int = 0x9747B28C,
+                 tc_pair: bool = True):
         self.mask = parse_cksum(cksum)
         self.store = STORE_NAMES[store] if isinstance(store, str) else int(store)
         self.body = BODY_NAMES[body] if isinstance(body, str) else int(body)
         self.region = (region_m, region_n)
         self.device = device
-        self.cfg = Config(region_m, region_n, self.mask, self.store, device, self.body, hash_seed, 0)
+        self.cfg = Config(region_m, region_n, self.mask, self.store, device, self.body, hash_seed,
+                          0 if tc_pair else FLAG_TC_1CTA)
         h = ctypes.c_void_p()
         _check(lib().lp_config(ctypes.byref(self.cfg), ctypes.byref(h)))
         self._h = h

@@ -7,8 +7,8 @@ a = torch.empty((M,K), dtype=torch.bfloat16, device='cuda'); b = torch.empty((K,
 lpsynth.device_fill(a, 1, 'uniform', 'bf16'); lpsynth.device_fill(b, 2, 'uniform', 'bf16')
 flush = torch.empty(512<<20, dtype=torch.uint8, device='cuda')
 res = {}
-for name, mask, reg in [('unprot',0,128),('mod',1,128),('xor',2,128),('modxor',3,128),('adler',4,128),('all',7,128),('modxor32',3,32)]:
-    h = lp.LP(reg,reg,cksum=mask,body='tcgen05')
+for name, mask, reg, pair in [('unprot',0,128,True),('modxor',3,128,True),('adler',4,128,True),('all',7,128,True),('modxor32',3,32,True),('unprot_1cta',0,128,False),('modxor_1cta',3,128,False)]:
+    h = lp.LP(reg,reg,cksum=mask,body='tcgen05',tc_pair=pair)
     wl = lp.Workload.tmm(a,b,out_dtype='bf16')
     out,ck,failed,d_n,ws = h.alloc(wl)
     if mask: h.cksum_init(wl,ck)

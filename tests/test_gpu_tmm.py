@@ -18,8 +18,8 @@ pytestmark = pytest.mark.gpu
 
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
-              store="array", check_values=True, recover_ws=True):
-    h = lp.LP(RM, RN, cksum=mask, store=store, body=body)
+              store="array", check_values=True, recover_ws=True, tc_pair=True):
+    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -137,8 +137,11 @@ def test_simt_hash_stores(store):
 @pytest.mark.parametrize("kind", ["int5", "uniform"])
 @pytest.mark.parametrize("out_dt", ["bf16", "f32"])
 @pytest.mark.parametrize("reg", [128, 32])
-def test_tc_cycle(kind, out_dt, reg):
-    run_cycle(256, 512, 256, reg, reg, "bf16", out_dt, kind, "mod|xor", "tcgen05", mode="stale_words", frac=0.2)
+@pytest.mark.parametrize("tc_pair", [True, False])
+def test_tc_cycle(kind, out_dt, reg, tc_pair):
+    """M, N multiples of 256: the CTA-pair kernel (tc_pair) or the 1-SM kernel; recovery = 1-SM list mode."""
+    run_cycle(256, 512, 256, reg, reg, "bf16", out_dt, kind, "mod|xor", "tcgen05", mode="stale_words", frac=0.2,
+              tc_pair=tc_pair)
 
 
 @pytest.mark.parametrize("recover_ws", [True, False])
@@ -157,10 +160,11 @@ def test_tc_n_not_multiple_of_256():
     run_cycle(256, 384, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", mode="stale_region", frac=0.5)
 
 
-def test_tc_many_tiles_persistent():
+@pytest.mark.parametrize("tc_pair", [True, False])
+def test_tc_many_tiles_persistent(tc_pair):
     # more tiles than SMs: persistent scheduling + TMEM double buffering across tiles
     run_cycle(2048, 2048, 512, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", mode="stale_words",
-              frac=0.05, check_values=True)
+              frac=0.05, check_values=True, tc_pair=tc_pair)
 
 
 @pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
