@@ -59,6 +59,8 @@ def main(rdir):
         out.append("")
         wl = WL["stencil" if "stencil" in tag else "tmm"]
         kern = name.split("<")[0].split("::")[-1].replace("void ", "").strip()
+        if "recover" in tag:
+            kern += "_list_mode"
         traffic.setdefault(wl, {})[kern] = int(rd + wr)
     for f in sorted(glob.glob(os.path.join(rdir, "launches_*.csv"))):
         rows = [r for r in csv.reader(open(f)) if len(r) > 5]
