@@ -151,8 +151,10 @@ size_t cksum_bytes(const lp_ctx* h, const lp::RegionGeom& g) {
   return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R) * 4u * (size_t)(1 + h->selem);
 }
 
-// 128x128 tensor-core tiles covering the output (recovery de-duplication of 32x32 regions)
-int64_t dedupe_tiles(const lp::RegionGeom& g) { return (g.RM == 32 && g.RN == 32) ? (g.M / 128) * (g.N / 128) : 0; }
+// Tensor-core tiles covering the output, for recovery de-duplication: 128x128 tiles of
+// 32x32 regions (bf16 1-SM list mode) or 256x256 tiles (fp32 3xTF32 CTA-pair list mode).
+int64_t dedupe_tiles(const lp::RegionGeom& g, int E) { return (g.M % E || g.N % E) ? 0 : (g.M / E) * (g.N / E); }
+int64_t dedupe_capacity(const lp::RegionGeom& g) { return dedupe_tiles(g, 128); }
 
 struct WsLayout {
   size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, total;
@@ -160,7 +162,7 @@ struct WsLayout {
 
 WsLayout ws_layout(const lp::RegionGeom& g) {
   auto al = [](size_t x) { return (x + 255) & ~(size_t)255; };
-  const int64_t T = dedupe_tiles(g);
+  const int64_t T = dedupe_capacity(g);
   WsLayout w;
   w.flags = 0;
   w.counts = al((size_t)g.R);
@@ -229,18 +231,22 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.sm_count = h->sm_count;
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
+  const bool tf_ok = lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, a.out_bf16, wl->lda,
+                                            wl->ldb, wl->ldc, wl->a, wl->b, out);
   int body = h->cfg.body;
-  if (body == LP_BODY_AUTO) body = tc_ok ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
+  if (body == LP_BODY_AUTO) body = (tc_ok || tf_ok) ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
   if (body == LP_BODY_TCGEN05) {
-    if (!tc_ok)
+    if (!tc_ok && !tf_ok)
       return fail(LP_ERR_UNSUPPORTED,
-                  "tcgen05 body needs bf16 input, m%%128 == 0, n%%256 == 0, k%%64 == 0, region 128x128 or 32x32 "
-                  "dividing the 128x256 tile, 16-B aligned pitches");
-    if (list && workspace && dedupe_tiles(g) > 0) {
-      // several failed 32x32 regions may share one 128x128 tile: recompute each tile once
+                  "tcgen05 body needs 16-B aligned pitches, region 128x128 or 32x32, and either bf16 input with "
+                  "m%%128 == 0, n%%128 == 0, k%%64 == 0, or fp32 input/output with m, n %% 256 == 0, k %% 32 == 0");
+    const int E = tc_ok ? 128 : 256;  // tile edge of the list-mode kernel
+    const bool need_dedupe = tf_ok ? true : (g.RM == 32);
+    if (list && workspace && need_dedupe && dedupe_tiles(g, E) > 0) {
+      // several failed regions may share one tensor-core tile: recompute each tile once
       const WsLayout w = ws_layout(g);
       uint8_t* ws = (uint8_t*)workspace;
-      cudaError_t e0 = lp::launch_tiles_of_failed(g, list, d_n, ws + w.tile_flags, dedupe_tiles(g),
+      cudaError_t e0 = lp::launch_tiles_of_failed(g, E, list, d_n, ws + w.tile_flags, dedupe_tiles(g, E),
                                                   (uint32_t*)(ws + w.tile_counts), (int64_t*)(ws + w.tile_list),
                                                   (int64_t*)(ws + w.d_ntiles), st);
       if (e0 != cudaSuccess) return cuda_fail(e0, "tile de-duplication");
@@ -249,7 +255,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
       a.list_is_tiles = 1;
     }
     const char* why = nullptr;
-    cudaError_t e = lp::launch_tmm_tc(a, st, &why);
+    cudaError_t e = tc_ok ? lp::launch_tmm_tc(a, st, &why) : lp::launch_tmm_tf32(a, st, &why);
     if (e != cudaSuccess) return why ? fail(LP_ERR_CUDA, "tcgen05 launch: %s", why) : cuda_fail(e, "tcgen05 launch");
     return ok();
   }

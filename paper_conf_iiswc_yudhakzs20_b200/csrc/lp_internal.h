@@ -35,10 +35,10 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
                           const void* stale, const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed,
                           cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
-// failed 32x32 regions -> unique 128x128 tile ids (tile = (p/4)*(N/128) + q/4), ascending
-cudaError_t launch_tiles_of_failed(const RegionGeom& g, const int64_t* list, const int64_t* d_n, uint8_t* tile_flags,
-                                   int64_t T, uint32_t* block_counts, int64_t* tile_list, int64_t* d_ntiles,
-                                   cudaStream_t st);
+// failed regions -> unique tile ids of an E x E tile grid (tile = (p*RM/E)*(N/E) + q*RN/E), ascending
+cudaError_t launch_tiles_of_failed(const RegionGeom& g, int E, const int64_t* list, const int64_t* d_n,
+                                   uint8_t* tile_flags, int64_t T, uint32_t* block_counts, int64_t* tile_list,
+                                   int64_t* d_ntiles, cudaStream_t st);
 
 // ---- tmm_simt.cu : SIMT region body (CTA tile == region), paper-shaped
 struct TmmArgs {
@@ -68,6 +68,11 @@ cudaError_t launch_tmm_simt(const TmmArgs& a, cudaStream_t st);
 bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int64_t lda, int64_t ldb,
                       int64_t ldc, const void* A, const void* B, const void* C);
 cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why);
+
+// ---- tmm_tf32.cu : fp32 in/out via 3xTF32 on tcgen05 (CTA pair)
+bool tmm_tf32_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int out_bf16, int64_t lda,
+                        int64_t ldb, int64_t ldc, const void* A, const void* B, const void* C);
+cudaError_t launch_tmm_tf32(const TmmArgs& a, cudaStream_t st, const char** why);
 
 // ---- stencil.cu : 5-point stencil region body
 struct StencilArgs {

@@ -382,14 +382,14 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
   return cudaGetLastError();
 }
 
-cudaError_t launch_tiles_of_failed(const RegionGeom& g, const int64_t* list, const int64_t* d_n, uint8_t* tile_flags,
-                                   int64_t T, uint32_t* block_counts, int64_t* tile_list, int64_t* d_ntiles,
-                                   cudaStream_t st) {
+cudaError_t launch_tiles_of_failed(const RegionGeom& g, int E, const int64_t* list, const int64_t* d_n,
+                                   uint8_t* tile_flags, int64_t T, uint32_t* block_counts, int64_t* tile_list,
+                                   int64_t* d_ntiles, cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(tile_flags, 0, (size_t)T, st);
   if (e != cudaSuccess) return e;
-  const int per = 128 / g.RM;
+  const int per = E / g.RM;
   tile_mark_kernel<<<(unsigned)(g.R < 148 * 4 * 256 ? (g.R + 255) / 256 : 148 * 4), 256, 0, st>>>(
-      list, d_n, g.rid_offset, g.Q, g.N / 128, per, tile_flags);
+      list, d_n, g.rid_offset, g.Q, g.N / E, per, tile_flags);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   RegionGeom tg = g;

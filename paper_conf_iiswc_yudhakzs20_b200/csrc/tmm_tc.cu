@@ -35,15 +35,14 @@
 #include "lp_internal.h"
 #include "lp_ptx.cuh"
 #include "lp_tma.h"
+#include "tc_common.cuh"
 
 namespace lp {
 namespace {
 
-constexpr int kBM = 128;
 constexpr int kBK = 64;      // 64 bf16 = 128 B = one swizzle atom row
 constexpr int kUmmaK = 16;   // K per tcgen05.mma kind::f16
 constexpr int kThreads = 192;
-constexpr int kEpiWarp0 = 2;
 
 template <int BN>
 struct TcCfg {
@@ -55,182 +54,12 @@ struct TcCfg {
   static constexpr int kSmemBytes = kStages * kStageBytes + 1024 /*barriers etc.*/ + 1024 /*align slack*/;
 };
 
-__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
-__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
-
-__device__ __forceinline__ void tc_mma(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
-                                       uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-
-__device__ __forceinline__ void tc_commit(uint64_t* bar) {
-  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
-               : "memory");
-}
-
-#define LP_TMEM_LD32(taddr, r)                                                                                       \
-  asm volatile(                                                                                                      \
-      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,%17,%18,"   \
-      "%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"                                                 \
-      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),  \
-        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),       \
-        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),      \
-        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])                    \
-      : "r"(taddr))
-
-__device__ __forceinline__ void tc_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
-
-// Shared-memory matrix descriptor (sm_100 UMMA): start>>4 [0,14), LBO>>4 [16,30),
-// SBO>>4 [32,46), version 1 [46,48), layout SWIZZLE_128B = 2 at [61,64).
-__device__ __forceinline__ uint64_t smem_desc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
-  uint64_t d = 0;
-  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
-  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
-  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
-  d |= (uint64_t)1 << 46;
-  d |= (uint64_t)2 << 61;
-  return d;
-}
-
 // Instruction descriptor kind::f16: D fp32 [4,6)=1, A bf16 [7,10)=1, B bf16 [10,13)=1,
 // A K-major (bit 15 = 0), B MN-major (bit 16 = 1), N>>3 at [17,23), M>>4 at [24,29).
 template <int BN>
 __host__ __device__ constexpr uint32_t instr_desc() {
   return (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
          ((uint32_t)(kBM >> 4) << 24);
-}
-
-__device__ __forceinline__ void named_bar_epi() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
-
-// Tile order: groups of 16 M-blocks, M fastest inside a group (L2 reuse of B panels).
-__device__ __forceinline__ void tile_coords(int64_t t, int64_t num_m, int64_t num_n, int64_t& mb, int64_t& nb) {
-  constexpr int64_t G = 16;
-  const int64_t per_group = G * num_n;
-  const int64_t g = t / per_group, w = t - g * per_group;
-  const int64_t rows = (num_m - g * G) < G ? (num_m - g * G) : G;
-  mb = g * G + w % rows;
-  nb = w / rows;
-}
-
-struct TileSrc {
-  int64_t num_m, num_n;       // tile grid
-  const int64_t* list;        // list mode: failed global rids
-  const int64_t* d_n;
-  int64_t rid_offset;
-  int64_t Qr;                 // regions per output row band
-  int reg;                    // region edge (32 or 128)
-  int list_is_tiles;          // list holds tile ids (already de-duplicated)
-  __device__ __forceinline__ int64_t count() const { return list ? *d_n : num_m * num_n; }
-  template <int BN>
-  __device__ __forceinline__ void coords(int64_t t, int64_t& mb, int64_t& nb) const {
-    if (!list) {
-      tile_coords(t, num_m, num_n, mb, nb);
-      return;
-    }
-    if (list_is_tiles) {
-      mb = list[t] / num_n;
-      nb = list[t] - mb * num_n;
-      return;
-    }
-    const int64_t rid = list[t] - rid_offset;
-    const int64_t p = rid / Qr, q = rid - p * Qr;
-    mb = p * reg / kBM;
-    nb = q * reg / BN;
-  }
-};
-
-// ---------------------------------------------------------------------------- epilogue pieces
-// Store one 128-row x BN-column accumulator (this warp's 32 TMEM lanes) to C and
-// fold the exact stored words into the LP checksum (L192).  m128 = index of the
-// 128-row block of C, n0 = first column.  32x32 regions are finished here (one
-// warp-wide redux per checksum, Listing 4); 128x128 regions leave one partial
-// per warp in srec for epi_finish_128.
-template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
-__device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, int64_t ldc, int64_t m128, int64_t n0,
-                                          int wq, int lane, CkRecord* srec_acc, uint32_t* __restrict__ ck, int64_t Qr,
-                                          int64_t rid_offset) {
-  constexpr int ES = (int)sizeof(OutT);
-  constexpr int NCH = BN / 32;
-  const int row_in_tile = wq * 32 + lane;
-  OutT* crow = C + (m128 * kBM + row_in_tile) * ldc + n0;
-  CkPartial<MASK> part;
-#pragma unroll 1
-  for (int ch = 0; ch < NCH; ++ch) {
-    uint32_t r[32];
-    LP_TMEM_LD32(t_row + ch * 32, r);
-    tc_wait_ld();
-    if constexpr (ES == 2) {
-      uint32_t w[16];
-#pragma unroll
-      for (int i = 0; i < 16; ++i) {
-        __nv_bfloat162 h = __floats2bfloat162_rn(__uint_as_float(r[2 * i]), __uint_as_float(r[2 * i + 1]));
-        w[i] = *reinterpret_cast<uint32_t*>(&h);  // even column in the low half (Reading R6)
-      }
-      uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
-#pragma unroll
-      for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
-      if constexpr (MASK != 0) {
-        // byte position of word 0 of this chunk inside its region's stream
-        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
-                                         : (uint32_t)(lane * 32 * ES + 1);
-#pragma unroll
-        for (int i = 0; i < 16; ++i) part.add(w[i], pos0 + 4 * i);
-      }
-    } else {
-      uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
-#pragma unroll
-      for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
-      if constexpr (MASK != 0) {
-        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
-                                         : (uint32_t)(lane * 32 * ES + 1);
-#pragma unroll
-        for (int i = 0; i < 32; ++i) part.add(r[i], pos0 + 4 * i);
-      }
-    }
-    if constexpr (MASK != 0) {
-      if constexpr (REG == 32) {
-        // one 32x32 region = this warp's 32 rows x this 32-column chunk
-        const CkRecord rec = warp_reduce<MASK>(part);
-        if (lane == 0) {
-          const int64_t p = m128 * (kBM / 32) + wq, q = (n0 + ch * 32) / 32;
-          const int64_t rid = p * Qr + q;
-          uint32_t words[3];
-          record_words<MASK>(rec, (uint64_t)32 * 32 * ES, words);
-          store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
-        }
-        part = CkPartial<MASK>();
-      } else if ((ch & 3) == 3) {
-        // end of a 128-column region: warp partial -> shared slot
-        const CkRecord rec = warp_reduce<MASK>(part);
-        if (lane == 0) srec_acc[(ch / 4) * 4 + wq] = rec;
-        part = CkPartial<MASK>();
-      }
-    }
-  }
-}
-
-// 128x128 regions: after the epilogue warps' named barrier, combine the 4 warp
-// partials of each region (Listing 3's block combine) and store the record.
-template <typename OutT, uint32_t MASK, int BN, int STORE>
-__device__ __forceinline__ void epi_finish_128(int warp, int lane, const CkRecord* srec_acc, uint32_t* __restrict__ ck,
-                                               int64_t m128, int64_t n0, int64_t Qr, int64_t rid_offset) {
-  constexpr int ES = (int)sizeof(OutT);
-  named_bar_epi();
-  if (warp == kEpiWarp0 && lane < BN / 128) {
-    const int j = lane;
-    CkRecord rr = srec_acc[j * 4 + 0];
-#pragma unroll
-    for (int w = 1; w < 4; ++w) rr = combine(rr, srec_acc[j * 4 + w]);
-    const int64_t rid = m128 * Qr + n0 / 128 + j;
-    uint32_t words[3];
-    record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
-    store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
-  }
 }
 
 template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
@@ -397,48 +226,6 @@ constexpr int kA2Bytes = kBM * kBK * 2;   // 16 KiB: this CTA's 128 rows of A
 constexpr int kB2Bytes = kBK * 128 * 2;   // 16 KiB: this CTA's 128 columns of B
 constexpr int kStage2Bytes = kA2Bytes + kB2Bytes;
 constexpr int kSmem2Bytes = kStages2 * kStage2Bytes + 1024 + 1024;
-
-__device__ __forceinline__ uint32_t cluster_ctarank() {
-  uint32_t r;
-  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-  return r;
-}
-__device__ __forceinline__ void cluster_sync_all() {
-  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-// shared::cluster address of the same variable in CTA rank 0 of the cluster
-__device__ __forceinline__ uint32_t mapa_rank0(const void* p) {
-  uint32_t r;
-  asm volatile("mapa.shared::cluster.u32 %0, %1, 0;" : "=r"(r) : "r"(smem_u32(p)));
-  return r;
-}
-__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
-__device__ __forceinline__ void tma_load_2d_pair(const CUtensorMap* map, uint32_t mbar_rank0, void* dst, int c0,
-                                                 int c1) {
-  asm volatile(
-      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, "
-      "%4}], [%2];" ::"r"(smem_u32(dst)),
-      "l"((uint64_t)map), "r"(mbar_rank0), "r"(c0), "r"(c1)
-      : "memory");
-}
-__device__ __forceinline__ void tc_mma_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
-                                            uint32_t accumulate) {
-  asm volatile(
-      "{\n\t.reg .pred p;\n\t"
-      "setp.ne.b32 p, %4, 0;\n\t"
-      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate)
-      : "memory");
-}
-__device__ __forceinline__ void tc_commit_pair(uint64_t* bar) {
-  asm volatile(
-      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
-          smem_u32(bar)),
-      "h"((uint16_t)3)
-      : "memory");
-}
 
 template <typename OutT, uint32_t MASK, int REG, int STORE>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)

@@ -20,12 +20,14 @@ from tests.gpu_util import dev_to_host
 pytestmark = pytest.mark.gpu
 
 
-def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, global_m=None, frac=0.05, seed=1):
+def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, global_m=None, frac=0.05, seed=1,
+              in_dt="bf16"):
     global_m = global_m or M
-    a = torch.empty((M, K), dtype=torch.bfloat16, device="cuda")
-    b = torch.empty((K, N), dtype=torch.bfloat16, device="cuda")
-    lpsynth.device_fill(a, seed, kind, "bf16", row0=row0, ncols_global=K)
-    lpsynth.device_fill(b, seed + 1, kind, "bf16")
+    tdt = torch.bfloat16 if in_dt == "bf16" else torch.float32
+    a = torch.empty((M, K), dtype=tdt, device="cuda")
+    b = torch.empty((K, N), dtype=tdt, device="cuda")
+    lpsynth.device_fill(a, seed, kind, in_dt, row0=row0, ncols_global=K)
+    lpsynth.device_fill(b, seed + 1, kind, in_dt)
     h = lp.LP(region, region, cksum=mask, store=store)                 # body AUTO = tcgen05, as in bench.py
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt, row_offset=row0, global_m=global_m)
     out, ck, failed, d_n, ws = h.alloc(wl)
@@ -58,8 +60,8 @@ def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, globa
     rng = np.random.default_rng(seed)
     for rid in rng.choice(R, nsample, replace=False):
         p, q = divmod(int(rid), Q)
-        A_rows = gen.generate(seed, region, K, kind, "bf16", row0=row0 + p * region, ncols_global=K)
-        B_cols = gen.generate(seed + 1, K, region, kind, "bf16", ncols_global=N, col0=q * region)
+        A_rows = gen.generate(seed, region, K, kind, in_dt, row0=row0 + p * region, ncols_global=K)
+        B_cols = gen.generate(seed + 1, K, region, kind, in_dt, ncols_global=N, col0=q * region)
         ref = oracle.gemm_block_f64(A_rows, B_cols, 0, 0, region, region)
         got = gold[p * region:(p + 1) * region, q * region:(q + 1) * region]
         if kind != "uniform":
@@ -103,6 +105,15 @@ def test_c2_tmm8192_integer_valued_bit_exact():
 
 def test_c2_tmm8192_f32_out():
     _tmm_full(8192, 8192, 8192, 128, "mod|xor", "array", "uniform", "f32", nsample=4, seed=11)
+
+
+def test_c2_tmm8192_fp32_3xtf32_full():
+    """configs[1] fp32 -> fp32 on the tensor cores (3xTF32): max rel. error <= 1e-5 on sampled regions."""
+    _tmm_full(8192, 8192, 8192, 128, "mod|xor", "array", "uniform", "f32", nsample=4, seed=13, in_dt="f32")
+
+
+def test_c2_tmm8192_fp32_integer_valued_bit_exact():
+    _tmm_full(8192, 8192, 8192, 128, "mod|xor", "array", "int5", "f32", nsample=4, seed=17, in_dt="f32")
 
 
 def test_c3_tmm16384_quad_cas_full():

@@ -207,3 +207,30 @@ def test_tc_matches_simt_integer_valued():
         torch.cuda.synchronize()
         res.append((dev_to_host(out), dev_to_host(ck)))
     assert np.array_equal(res[0][0], res[1][0]) and np.array_equal(res[0][1], res[1][1])
+
+
+# ----------------------------------------------------------------------------- fp32 via 3xTF32 (CTA pair)
+@pytest.mark.parametrize("kind", ["int5", "uniform"])
+@pytest.mark.parametrize("reg", [128, 32])
+@pytest.mark.parametrize("recover_ws", [True, False])
+def test_tf32x3_cycle(kind, reg, recover_ws):
+    run_cycle(512, 768, 256, reg, reg, "f32", "f32", kind, "mod|xor", "tcgen05", mode="stale_words", frac=0.1,
+              recover_ws=recover_ws)
+
+
+def test_tf32x3_matches_simt_integer_valued():
+    """3xTF32 tensor-core body and the SIMT FFMA body are both exact on integer-valued fp32 inputs: same bits."""
+    import numpy as np
+    from tests.gpu_util import make_inputs
+    A, B = make_inputs(6, 512, 512, 512, "int5", "f32")
+    a, b = host_to_dev(A, "f32"), host_to_dev(B, "f32")
+    res = []
+    for body in ["simt", "tcgen05"]:
+        h = lp.LP(128, 128, cksum="mod|xor|adler", body=body)
+        wl = lp.Workload.tmm(a, b, out_dtype="f32")
+        out, ck, *_ = h.alloc(wl)
+        h.cksum_init(wl, ck)
+        h.run_protected(wl, out, ck)
+        torch.cuda.synchronize()
+        res.append((dev_to_host(out), dev_to_host(ck)))
+    assert np.array_equal(res[0][0], res[1][0]) and np.array_equal(res[0][1], res[1][1])
