@@ -48,6 +48,17 @@ WORKLOADS = {
     # BASELINE configs[1] (N=1 default); weak-scaled by rows under torchrun
     "tmm8192_bf16": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=128,
                          cksum="mod|xor", frac=0.05, store="array", weak=True),
+    # C2 checksum-type sweep (L192, L587: parity vs modular vs both vs Adler-32)
+    "tmm8192_bf16_mod": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=128,
+                             cksum="mod", frac=0.05, store="array", weak=True),
+    "tmm8192_bf16_xor": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=128,
+                             cksum="xor", frac=0.05, store="array", weak=True),
+    "tmm8192_bf16_adler": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=128,
+                               cksum="adler", frac=0.05, store="array", weak=True),
+    "tmm8192_bf16_all": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=128,
+                             cksum="mod|xor|adler", frac=0.05, store="array", weak=True),
+    "tmm8192_bf16_r32": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="bf16", region=32,
+                             cksum="mod|xor", frac=0.05, store="array", weak=True),
     "tmm8192_bf16_f32out": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="f32", region=128,
                                 cksum="mod|xor", frac=0.05, store="array", weak=True),
     # BASELINE configs[3]: stencil 32768^2 fp32, 128x128 regions, 10% injection
@@ -340,6 +351,9 @@ def run_ours(args):
         torch.cuda.synchronize()
         (tp if i % 2 == 0 else tu).append(e0.elapsed_time(e1))
     t_prot, t_unprot = report.median(tp), report.median(tu)
+    # overhead from adjacent (protected, unprotected) pairs: robust to clock drift under the power cap
+    pair_ratios = [a / b for a, b in zip(tp, tu)]
+    overhead_pairs = 100.0 * (report.median(pair_ratios) - 1.0)
     clocks = clk.stop()
     # hash-store statistics of one fresh protected run (collisions = sum of extra probes, Table II analog)
     d_stats = torch.zeros(2, dtype=torch.int64, device=dev)
@@ -410,19 +424,25 @@ def run_ours(args):
             elif W["in_dt"] == "bf16":
                 kname = "tmm_tc2_kernel" if (M % 256 == 0 and N % 256 == 0) else "tmm_tc_kernel"
                 achieved = body_flops / (t_prot * 1e-3) / 1e12
+                # kernels of several ms run back to back under the 1 kW cap: sustained peak
+                long_kernel = t_prot > 2.0 and bf16_s is not None
+                pk = bf16_s if long_kernel else bf16
                 roof = {"bound": "tensor", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 1),
-                        "peak": bf16, "unit": "TFLOP/s", "frac": round(achieved / bf16, 4),
-                        "peak_source": f"{peak_src} bf16 burst (kernel timed alone)",
+                        "peak": pk, "unit": "TFLOP/s", "frac": round(achieved / pk, 4),
+                        "peak_source": f"{peak_src} bf16 " + ("sustained (multi-ms kernel, power-capped)" if long_kernel
+                                                              else "burst (kernel timed alone)"),
                         "algorithmic_per_launch": f"2*M*N*K = {body_flops:.4g} flop",
                         "traffic": ncu_traffic(kname, args.workload)}
             else:
                 kname = "tmm_tf32x3_kernel"
-                tf32_peak = bf16 * (1.125 / 2.25)   # measured bf16 x nominal tf32/bf16 dense ratio (guide table)
+                base = bf16_s if (t_prot > 2.0 and bf16_s is not None) else bf16
+                tf32_peak = base * (1.125 / 2.25)   # measured bf16 x nominal tf32/bf16 dense ratio (guide table)
                 achieved = 3.0 * body_flops / (t_prot * 1e-3) / 1e12   # 3 tf32 MMAs per fp32 MAC
                 roof = {"bound": "tensor", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 1),
                         "peak": round(tf32_peak, 1), "unit": "TFLOP/s (tf32 tensor work)",
                         "frac": round(achieved / tf32_peak, 4),
-                        "peak_source": f"{peak_src} bf16 burst x 0.5 (nominal tf32/bf16 dense ratio)",
+                        "peak_source": f"{peak_src} bf16 {'sustained' if base != bf16 else 'burst'} x 0.5 "
+                                       "(nominal tf32/bf16 dense ratio)",
                         "algorithmic_per_launch": f"3 x 2*M*N*K = {3 * body_flops:.4g} tf32 flop "
                                                   f"(fp32-equivalent {body_flops / (t_prot * 1e-3) / 1e12:.1f} TFLOP/s)",
                         "traffic": ncu_traffic(kname, args.workload)}
@@ -452,7 +472,10 @@ def run_ours(args):
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write) before every recovery phase and every isolated kernel rep"},
-            "lp_overhead_pct": round(report.overhead_pct(t_prot, t_unprot), 3),
+            "lp_overhead_pct": round(overhead_pairs, 3),
+            "lp_overhead_pct_of_medians": round(report.overhead_pct(t_prot, t_unprot), 3),
+            "lp_overhead_method": f"median over {len(pair_ratios)} adjacent (protected, unprotected) run pairs of "
+                                  "t_prot/t_unprot - 1, L2 flushed before every run",
             "t_protected_ms": round(t_prot, 4),
             "t_unprotected_ms": round(t_unprot, 4),
             "t_validate_ms": round(t_validate, 4),

@@ -166,7 +166,9 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   WsLayout w;
   w.flags = 0;
   w.counts = al((size_t)g.R);
-  w.tile_flags = w.counts + al(lp::compact_scratch_bytes(g.R));
+  const size_t counts_bytes = lp::compact_scratch_bytes(g.R) > (size_t)148 * 16 * 4 * 4 ? lp::compact_scratch_bytes(g.R)
+                                                                                         : (size_t)148 * 16 * 4 * 4;
+  w.tile_flags = w.counts + al(counts_bytes);
   w.tile_counts = w.tile_flags + al((size_t)T);
   w.tile_list = w.tile_counts + al(lp::compact_scratch_bytes(T));
   w.d_ntiles = w.tile_list + al((size_t)T * 8);
@@ -380,10 +382,9 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
   uint8_t* flags = (uint8_t*)workspace + w.flags;
   uint32_t* counts = (uint32_t*)((uint8_t*)workspace + w.counts);
   cudaStream_t st = (cudaStream_t)stream;
-  cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st);
-  if (e != cudaSuccess) return cuda_fail(e, "validate launch");
-  e = lp::launch_compact(g, flags, counts, failed_list, d_n_failed, st);
-  return e == cudaSuccess ? ok() : cuda_fail(e, "compact launch");
+  cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st, counts,
+                                      failed_list, d_n_failed);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "validate launch");
 }
 
 lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
@@ -413,8 +414,8 @@ lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* 
   }
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
-  cudaError_t e =
-      lp::launch_validate(g, h->mask, hash_info(h, g), out, nullptr, nullptr, records, h->sm_count, (cudaStream_t)stream);
+  cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, nullptr, nullptr, records, h->sm_count,
+                                      (cudaStream_t)stream, nullptr, nullptr, nullptr);
   return e == cudaSuccess ? ok() : cuda_fail(e, "records launch");
 }
 

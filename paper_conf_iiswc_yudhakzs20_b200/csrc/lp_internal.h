@@ -25,9 +25,13 @@ struct HashInfo {
 
 // ---- lp_kernels.cu
 cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaStream_t st);
+// Validation + ordered compaction (2 launches): flags[R], per-CTA failure counts,
+// ascending failed list + device count.  records != null => records mode (no compare,
+// no compaction).
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
-                            uint8_t* flags, uint32_t* records /* non-null => records mode */, int sm_count,
-                            cudaStream_t st);
+                            uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
+                            int64_t* list, int64_t* d_n);
+size_t validate_counts_bytes(const RegionGeom& g, int sm_count);
 cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* block_counts, int64_t* list,
                            int64_t* d_n, cudaStream_t st);
 size_t compact_scratch_bytes(int64_t R);

@@ -17,37 +17,54 @@ namespace lp {
 namespace {
 
 constexpr int kValThreads = 256;
+constexpr int64_t kMaxValCtas = 148 * 16 * 4;
 constexpr int kValUnroll = 8;
 
-// One warp per region.  MODE 0 = compare with array table, 1 = compare with a
-// quad hash table (lookup by global rid), 2 = write records (no compare).
-template <uint32_t MASK, int MODE>
+// W warps per region (W = 1, 2, 4, 8; chosen so each warp streams ~2-8 batches of
+// 4 KiB), 8/W regions in flight per CTA, each CTA a contiguous range of regions so
+// it can count its failures for the ordered compaction (no separate count pass).
+// A region's W warp partials are combined through double-buffered shared slots
+// behind a named barrier of the W warps (Listing 3's block combine, per region).
+// MODE 0 = compare with array table, 1 = compare with a quad hash table (lookup
+// by global rid), 2 = write records (no compare).
+template <uint32_t MASK, int MODE, int W>
 __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
                                                                 int64_t Q, int64_t R, int RM, int row_bytes,
                                                                 int cpr_log2, const uint32_t* __restrict__ ck,
                                                                 int64_t rid_offset, uint8_t* __restrict__ flags,
-                                                                uint32_t* __restrict__ records) {
+                                                                uint32_t* __restrict__ records, int64_t rpc,
+                                                                uint32_t* __restrict__ cta_counts) {
   constexpr int S = selem_of(MASK);
-  const int lane = threadIdx.x & 31;
-  const int64_t nwarps = (int64_t)gridDim.x * (kValThreads / 32);
+  constexpr int GROUPS = (kValThreads / 32) / W;
+  __shared__ CkRecord slots[2][GROUPS][W];
+  __shared__ uint32_t s_fail;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int g = warp / W, wi = warp - g * W;
   const int cpr_mask = (1 << cpr_log2) - 1;
   const int chunks = RM << cpr_log2;
+  const int my_chunks = chunks / W, c_begin = wi * my_chunks;
   const uint64_t nbytes = (uint64_t)RM * (uint64_t)row_bytes;
-  for (int64_t r = (int64_t)blockIdx.x * (kValThreads / 32) + (threadIdx.x >> 5); r < R; r += nwarps) {
+  if (threadIdx.x == 0) s_fail = 0;
+  __syncthreads();
+  const int64_t r0 = (int64_t)blockIdx.x * rpc;
+  const int64_t r1 = r0 + rpc < R ? r0 + rpc : R;
+  int parity = 0;
+  for (int64_t r = r0 + g; r < r1; r += GROUPS) {
     const int64_t p = r / Q, q = r - p * Q;
     const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
     CkPartial<MASK> part;
-    for (int c0 = 0; c0 < chunks; c0 += 32 * kValUnroll) {
+    for (int c0 = c_begin; c0 < c_begin + my_chunks; c0 += 32 * kValUnroll) {
       uint4 v[kValUnroll];
 #pragma unroll
       for (int u = 0; u < kValUnroll; ++u) {
         const int c = c0 + u * 32 + lane;
-        if (c < chunks) v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cpr_mask) << 4));
+        if (c < c_begin + my_chunks)
+          v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cpr_mask) << 4));
       }
 #pragma unroll
       for (int u = 0; u < kValUnroll; ++u) {
         const int c = c0 + u * 32 + lane;
-        if (c < chunks) {
+        if (c < c_begin + my_chunks) {
           const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cpr_mask) << 4) + 1);
           part.add(v[u].x, pos);
           part.add(v[u].y, pos + 4);
@@ -56,43 +73,88 @@ __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __
         }
       }
     }
-    const CkRecord rec = warp_reduce<MASK>(part);
-    if (lane == 0) {
+    CkRecord rec = warp_reduce<MASK>(part);
+    bool finisher = true;
+    if constexpr (W > 1) {
+      if (lane == 0) slots[parity][g][wi] = rec;
+      asm volatile("bar.sync %0, %1;" ::"r"(1 + g), "r"(W * 32) : "memory");
+      finisher = (wi == 0);
+      if (finisher) {
+        rec = slots[parity][g][0];
+#pragma unroll
+        for (int w = 1; w < W; ++w) rec = combine(rec, slots[parity][g][w]);
+      }
+      parity ^= 1;
+    }
+    if (finisher && lane == 0) {
       uint32_t w[3];
       record_words<MASK>(rec, nbytes, w);
       if constexpr (MODE == 2) {
 #pragma unroll
         for (int s = 0; s < S; ++s) records[r * S + s] = w[s];
-      } else if constexpr (MODE == 0) {
-        bool bad = false;
-#pragma unroll
-        for (int s = 0; s < S; ++s) bad |= (ck[r * S + s] != w[s]);
-        flags[r] = bad ? 1 : 0;
       } else {
-        uint32_t stored[3];
-        bool bad = !quad_lookup<S>(ck, (uint32_t)(r + rid_offset), stored);
+        bool bad = false;
+        if constexpr (MODE == 0) {
 #pragma unroll
-        for (int s = 0; s < S; ++s) bad |= (!bad && stored[s] != w[s]);
+          for (int s = 0; s < S; ++s) bad |= (ck[r * S + s] != w[s]);
+        } else {
+          uint32_t stored[3];
+          bad = !quad_lookup<S>(ck, (uint32_t)(r + rid_offset), stored);
+#pragma unroll
+          for (int s = 0; s < S; ++s) bad |= (!bad && stored[s] != w[s]);
+        }
         flags[r] = bad ? 1 : 0;
+        if (bad) atomicAdd(&s_fail, 1u);
       }
     }
   }
+  if constexpr (MODE != 2) {
+    __syncthreads();
+    if (threadIdx.x == 0) cta_counts[blockIdx.x] = s_fail;
+  }
+}
+
+struct ValLaunch {
+  dim3 grid;
+  int W;
+  int64_t rpc;
+};
+
+template <uint32_t MASK, int W>
+cudaError_t validate_dispatch_w(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out, int64_t ldc_bytes,
+                                int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2, const uint32_t* ck,
+                                int64_t rid_offset, uint8_t* flags, uint32_t* records, uint32_t* counts) {
+  if (mode == 0)
+    validate_kernel<MASK, 0, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                                rid_offset, flags, records, L.rpc, counts);
+  else if (mode == 1)
+    validate_kernel<MASK, 1, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                                rid_offset, flags, records, L.rpc, counts);
+  else
+    validate_kernel<MASK, 2, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                                rid_offset, flags, records, L.rpc, counts);
+  return cudaGetLastError();
 }
 
 template <uint32_t MASK>
-cudaError_t validate_dispatch_mode(int mode, dim3 grid, cudaStream_t st, const uint8_t* out, int64_t ldc_bytes,
-                                   int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2, const uint32_t* ck,
-                                   int64_t rid_offset, uint8_t* flags, uint32_t* records) {
-  if (mode == 0)
-    validate_kernel<MASK, 0><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                           rid_offset, flags, records);
-  else if (mode == 1)
-    validate_kernel<MASK, 1><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                           rid_offset, flags, records);
-  else
-    validate_kernel<MASK, 2><<<grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                           rid_offset, flags, records);
-  return cudaGetLastError();
+cudaError_t validate_dispatch_mode(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
+                                   int64_t ldc_bytes, int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2,
+                                   const uint32_t* ck, int64_t rid_offset, uint8_t* flags, uint32_t* records,
+                                   uint32_t* counts) {
+  switch (L.W) {
+    case 8:
+      return validate_dispatch_w<MASK, 8>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
+                                          flags, records, counts);
+    case 4:
+      return validate_dispatch_w<MASK, 4>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
+                                          flags, records, counts);
+    case 2:
+      return validate_dispatch_w<MASK, 2>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
+                                          flags, records, counts);
+    default:
+      return validate_dispatch_w<MASK, 1>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
+                                          flags, records, counts);
+  }
 }
 
 // ---------------------------------------------------------------------------
@@ -167,57 +229,63 @@ __global__ void __launch_bounds__(kCompactThreads) compact_count_kernel(const ui
 
 __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const uint8_t* __restrict__ flags, int64_t R,
                                                                           const uint32_t* __restrict__ block_counts,
-                                                                          int nblocks, int64_t rid_offset,
+                                                                          int nblocks, int64_t chunk, int per_block,
+                                                                          int64_t rid_offset,
                                                                           int64_t* __restrict__ list,
                                                                           int64_t* __restrict__ d_n) {
+  // counting block i (i < nblocks) owns flags [i*chunk, (i+1)*chunk); this scatter block
+  // owns counting blocks [b*per_block, (b+1)*per_block).  Its output offset is the sum of
+  // the counts before its first counting block (block 0 also publishes the total).
   __shared__ int warp_s[kCompactThreads / 32];
+  __shared__ long long red[2][kCompactThreads / 32];
   __shared__ long long s_base;
-  // base offset of this block = sum of the counts of the blocks before it
+  const int first = (int)blockIdx.x * per_block;
   long long mine = 0, all = 0;
   for (int b = threadIdx.x; b < nblocks; b += kCompactThreads) {
     const long long c = block_counts[b];
-    all += c;
-    if (b < (int)blockIdx.x) mine += c;
+    if (b < first) mine += c;
+    if (blockIdx.x == 0) all += c;
+    else if (b >= first) break;
   }
-  {
-    // block-reduce two values through shuffles + smem
-    for (int o = 16; o > 0; o >>= 1) {
-      mine += __shfl_xor_sync(0xFFFFFFFFu, mine, o);
-      all += __shfl_xor_sync(0xFFFFFFFFu, all, o);
-    }
-    __shared__ long long red[2][kCompactThreads / 32];
-    if ((threadIdx.x & 31) == 0) {
-      red[0][threadIdx.x >> 5] = mine;
-      red[1][threadIdx.x >> 5] = all;
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      long long m = 0, a = 0;
-      for (int w = 0; w < kCompactThreads / 32; ++w) {
-        m += red[0][w];
-        a += red[1][w];
-      }
-      s_base = m;
-      if (blockIdx.x == 0) *d_n = a;
-    }
-    __syncthreads();
+  for (int o = 16; o > 0; o >>= 1) {
+    mine += __shfl_xor_sync(0xFFFFFFFFu, mine, o);
+    all += __shfl_xor_sync(0xFFFFFFFFu, all, o);
   }
-  const int64_t idx0 = (int64_t)blockIdx.x * kCompactChunk + (int64_t)threadIdx.x * kCompactPerThread;
-  uint32_t f[8];
-  load_flags(flags, R, idx0, f);
-  int c = 0;
-#pragma unroll
-  for (int i = 0; i < 8; ++i) c += __popc(f[i]);
-  int total;
-  const int off = block_exclusive_scan(c, warp_s, &total);
-  int64_t o = s_base + off;
-#pragma unroll
-  for (int i = 0; i < 8; ++i) {
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      if ((f[i] >> (8 * j)) & 0xFFu) list[o++] = rid_offset + idx0 + i * 4 + j;
-    }
+  if ((threadIdx.x & 31) == 0) {
+    red[0][threadIdx.x >> 5] = mine;
+    red[1][threadIdx.x >> 5] = all;
   }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    long long m = 0, a = 0;
+    for (int w = 0; w < kCompactThreads / 32; ++w) {
+      m += red[0][w];
+      a += red[1][w];
+    }
+    s_base = m;
+    if (blockIdx.x == 0) *d_n = a;
+  }
+  __syncthreads();
+  long long base = s_base;
+  const int64_t lo = (int64_t)first * chunk;
+  int64_t hi = (int64_t)(first + per_block) * chunk;
+  if (hi > R) hi = R;
+  for (int64_t i0 = lo; i0 < hi; i0 += kCompactThreads) {
+    const int64_t i = i0 + threadIdx.x;
+    const int f = (i < hi && flags[i]) ? 1 : 0;
+    int total;
+    const int off = block_exclusive_scan(f, warp_s, &total);
+    if (f) list[base + off] = rid_offset + i;
+    base += total;
+    __syncthreads();  // warp_s reuse
+  }
+}
+
+static void scatter_grid(int64_t nblocks, int& grid, int& per_block) {
+  grid = (int)(nblocks < 64 ? nblocks : 64);
+  if (grid < 1) grid = 1;
+  per_block = (int)((nblocks + grid - 1) / grid);
+  grid = (int)((nblocks + per_block - 1) / per_block);
 }
 
 // ---------------------------------------------------------------------------
@@ -315,26 +383,54 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
   return e;
 }
 
+static ValLaunch plan_validate(const RegionGeom& g, int sm_count) {
+  ValLaunch L;
+  const int chunks = g.RM * ((g.RN * g.es) / 16);
+  const int64_t resident_warps = (int64_t)sm_count * 32;  // ~4 CTAs of 8 warps per SM
+  // enough warps per region that each warp streams only a few 4-KiB batches when regions are few
+  // Splitting a region over W > 1 warps was measured slower (validate of 128 MiB /
+  // 4096 regions: 45 us at W = 4 vs 25 us at W = 1): one warp streams one region.
+  int W = 1;
+  (void)resident_warps;
+  (void)chunks;
+  L.W = W;
+  const int groups = 8 / W;
+  int64_t max_ctas = (int64_t)sm_count * 16;
+  if (max_ctas > kMaxValCtas) max_ctas = kMaxValCtas;  // per-CTA counts live in the caller's workspace
+  int64_t ctas = (g.R + groups - 1) / groups;
+  if (ctas > max_ctas) ctas = max_ctas;
+  if (ctas < 1) ctas = 1;
+  int64_t rpc = (g.R + ctas - 1) / ctas;
+  rpc = (rpc + groups - 1) / groups * groups;
+  ctas = (g.R + rpc - 1) / rpc;
+  L.rpc = rpc;
+  L.grid = dim3((unsigned)(ctas < 1 ? 1 : ctas));
+  return L;
+}
+
+size_t validate_counts_bytes(const RegionGeom& g, int sm_count) {
+  (void)g;
+  return (size_t)sm_count * 16 * sizeof(uint32_t) + 256;
+}
+
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
-                            uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st) {
+                            uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
+                            int64_t* list, int64_t* d_n) {
   const int row_bytes = g.RN * g.es;
   const int cpr = row_bytes / 16;
   int cpr_log2 = 0;
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
-  const int64_t warps_needed = g.R;
-  int64_t blocks = (warps_needed + (kValThreads / 32) - 1) / (kValThreads / 32);
-  const int64_t cap_blocks = (int64_t)sm_count * 8;  // 8 x 256 threads = 2048 threads/SM
-  if (blocks > cap_blocks) blocks = cap_blocks;
-  if (blocks < 1) blocks = 1;
+  const ValLaunch L = plan_validate(g, sm_count);
   const int mode = records ? 2 : (hi.store == 0 ? 0 : 1);
   const uint8_t* o = (const uint8_t*)out;
   const int64_t ldcb = g.ldc * g.es;
-  dim3 grid((unsigned)blocks);
+  cudaError_t e;
   switch (mask) {
 #define LP_VCASE(M)                                                                                          \
   case M:                                                                                                    \
-    return validate_dispatch_mode<M>(mode, grid, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,          \
-                                     (const uint32_t*)ck, g.rid_offset, flags, records);
+    e = validate_dispatch_mode<M>(mode, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                \
+                                  (const uint32_t*)ck, g.rid_offset, flags, records, counts);               \
+    break;
     LP_VCASE(1)
     LP_VCASE(2)
     LP_VCASE(3)
@@ -346,6 +442,13 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
     default:
       return cudaErrorInvalidValue;
   }
+  if (e != cudaSuccess || records) return e;
+  // ordered compaction: one pass, offsets from the validate kernel's per-CTA counts
+  int sg, per;
+  scatter_grid(L.grid.x, sg, per);
+  compact_scatter_kernel<<<sg, kCompactThreads, 0, st>>>(flags, g.R, counts, (int)L.grid.x, L.rpc, per, g.rid_offset,
+                                                         list, d_n);
+  return cudaGetLastError();
 }
 
 size_t compact_scratch_bytes(int64_t R) {
@@ -360,8 +463,10 @@ cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* 
   compact_count_kernel<<<(unsigned)nb, kCompactThreads, 0, st>>>(flags, g.R, block_counts);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return e;
-  compact_scatter_kernel<<<(unsigned)nb, kCompactThreads, 0, st>>>(flags, g.R, block_counts, (int)nb, g.rid_offset,
-                                                                   list, d_n);
+  int sg, per;
+  scatter_grid(nb, sg, per);
+  compact_scatter_kernel<<<sg, kCompactThreads, 0, st>>>(flags, g.R, block_counts, (int)nb, kCompactChunk, per,
+                                                         g.rid_offset, list, d_n);
   return cudaGetLastError();
 }
 
