@@ -79,7 +79,9 @@ typedef enum { LP_CK_NONE = 0u, LP_CK_MOD = 1u, LP_CK_XOR = 2u, LP_CK_ADLER32 = 
  * insert inside one global spin lock (L81-83, L341 Table III, Reading R15). */
 typedef enum { LP_STORE_ARRAY = 0, LP_STORE_QUAD_CAS = 1, LP_STORE_QUAD_LOCK = 2 } lp_store;
 
-typedef enum { LP_F32 = 0, LP_BF16 = 1 } lp_dtype;
+/* Element types.  LP_I32 (in = out = int32, wrapping integer multiply-add) is the
+ * paper's own TMM type (Listing 2: int *a, *b, *c); SIMT body only. */
+typedef enum { LP_F32 = 0, LP_BF16 = 1, LP_I32 = 2 } lp_dtype;
 
 /* Region bodies.  TMM = tiled matrix multiply (Listing 2, Listing 6
  * L546-554), C = A*B, idempotent.  STENCIL5 = 5-point stencil, out-of-place

@@ -11,6 +11,7 @@ produce the same inputs independently. The recipe is DESIGN.md "Input recipe"
     int5    : v = (x mod 5) - 2                 TMM integer-valued inputs
     int17   : v = (x mod 17) - 8                stencil integer-valued inputs
     bits    : u32 = low 32 bits of x            "stale" pre-image of the output
+    int32 ("i32") inputs take the integer-valued kinds as int32 (the paper's TMM, Listing 2)
 
 global_index = row * ncols_global + col over the *global* matrix, so a row shard
 sees the same values it would see inside the unsharded matrix.
@@ -25,7 +26,7 @@ _M1 = np.uint64(0xBF58476D1CE4E5B9)
 _M2 = np.uint64(0x94D049BB133111EB)
 
 KINDS = {"uniform": 0, "int5": 1, "int17": 2, "bits": 3}
-DTYPES = {"f32": 0, "bf16": 1, "u32": 2}
+DTYPES = {"f32": 0, "bf16": 1, "u32": 2, "i32": 3}
 
 
 def splitmix64(z: np.ndarray) -> np.ndarray:
@@ -74,14 +75,18 @@ def generate(seed: int, rows: int, cols: int, kind: str, dtype: str, row0: int =
     if kind == "bits":
         x = raw(seed, rows, cols, row0, ncols_global, col0)
         bits = (x & np.uint64(0xFFFFFFFF)).astype(np.uint32)
-        if dtype == "u32" or dtype == "f32":
-            return bits if dtype == "u32" else bits.view(np.float32)
+        if dtype in ("u32", "f32", "i32"):
+            return {"u32": bits, "f32": bits.view(np.float32), "i32": bits.view(np.int32)}[dtype]
         if dtype == "bf16":
             return (bits & np.uint32(0xFFFF)).astype(np.uint16)
         raise ValueError(dtype)
     v = values_f32(seed, rows, cols, kind, row0, ncols_global, col0)
     if dtype == "f32":
         return v
+    if dtype == "i32":
+        if kind == "uniform":
+            raise ValueError("int32 inputs are integer-valued kinds (int5, int17)")
+        return v.astype(np.int32)
     if dtype == "bf16":
         return f32_to_bf16_bits(v)
     raise ValueError(dtype)

@@ -41,6 +41,7 @@ __global__ void synth_fill_kernel(void* dst, int64_t rows, int64_t cols, int64_t
     }
     const float v = value_of(x, kind);
     if (dtype == 1) ((__nv_bfloat16*)dst)[off] = __float2bfloat16_rn(v);
+    else if (dtype == 3) ((int32_t*)dst)[off] = (int32_t)v;
     else ((float*)dst)[off] = v;
   }
 }
@@ -49,7 +50,8 @@ __global__ void synth_fill_kernel(void* dst, int64_t rows, int64_t cols, int64_t
 
 extern "C" int synth_fill(void* dst, int64_t rows, int64_t cols, int64_t ld, int64_t row0,
                           int64_t ncols_global, uint64_t seed, int kind, int dtype, void* stream) {
-  if (!dst || rows < 0 || cols < 0 || ld < cols || kind < 0 || kind > 3 || dtype < 0 || dtype > 2) return 1;
+  if (!dst || rows < 0 || cols < 0 || ld < cols || kind < 0 || kind > 3 || dtype < 0 || dtype > 3) return 1;
+  if (dtype == 3 && kind == 0) return 1;  // int32 inputs are integer-valued kinds
   if (rows == 0 || cols == 0) return 0;
   const int64_t total = rows * cols;
   int64_t blocks = (total + 255) / 256;

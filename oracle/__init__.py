@@ -86,7 +86,7 @@ def _ptr(a: np.ndarray):
 
 
 def _es(out: np.ndarray) -> int:
-    if out.dtype == np.float32 or out.dtype == np.uint32:
+    if out.dtype == np.float32 or out.dtype == np.uint32 or out.dtype == np.int32:
         return 4
     if out.dtype == np.uint16:
         return 2
@@ -172,11 +172,11 @@ def validate_quad(out: np.ndarray, table: np.ndarray, cap: int, seed: int, RM: i
 
 
 def gemm_block_f64(A: np.ndarray, B: np.ndarray, row0: int, col0: int, rows: int, cols: int) -> np.ndarray:
-    """fp64 C[row0:row0+rows, col0:col0+cols] of A @ B (A, B float32 or bf16-bits uint16)."""
+    """fp64 C[row0:row0+rows, col0:col0+cols] of A @ B (A, B float32, bf16-bits uint16 or int32)."""
     A = np.ascontiguousarray(A)
     B = np.ascontiguousarray(B)
     assert A.dtype == B.dtype and A.shape[1] == B.shape[0]
-    is_bf16 = 1 if A.dtype == np.uint16 else 0
+    is_bf16 = {np.dtype(np.uint16): 1, np.dtype(np.float32): 0, np.dtype(np.int32): 2}[A.dtype]
     C = np.zeros((rows, cols), dtype=np.float64)
     lib().lpo_gemm_block_f64(_ptr(A), A.shape[1], _ptr(B), B.shape[1], is_bf16, A.shape[1], row0, col0, rows, cols,
                              _ptr(C))

@@ -194,9 +194,16 @@ int64_t lpo_validate_quad(const void* out, const uint32_t* table, uint32_t cap, 
 /* ------------------------------------------------------------------------ */
 /* Region body 1: tiled matrix multiply (Listing 2, Listing 6        */
 /* L546-554): C = A * B, A [M x K] row-major, B [K x N] row-major.  Plain     */
-/* triple loop in fp64 for the RM x RN block at (row0, col0).  a_bf16 /       */
-/* b_bf16 select the storage of the operands (bf16 bits are widened exactly). */
+/* triple loop in fp64 for the RM x RN block at (row0, col0).  is_bf16 selects */
+/* the operand storage: 0 fp32, 1 bf16 bits (widened exactly), 2 int32 (exact */
+/* while |partial sums| < 2^53).                                              */
+/* operand element as fp64: dtype 0 = fp32, 1 = bf16 bits, 2 = int32 (Listing 2's int TMM) */
 static double load_elem(const void* base, int is_bf16, int64_t idx) {
+  if (is_bf16 == 2) {
+    int32_t v;
+    memcpy(&v, (const uint8_t*)base + 4 * idx, 4);
+    return (double)v;
+  }
   if (is_bf16) {
     uint16_t h;
     memcpy(&h, (const uint8_t*)base + 2 * idx, 2);

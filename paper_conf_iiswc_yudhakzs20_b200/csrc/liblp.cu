@@ -74,8 +74,10 @@ lp_status check_wl(const lp_ctx* h, const lp_workload_t* wl, lp::RegionGeom* g) 
   if (!h) return fail(LP_ERR_INVALID_ARG, "null handle");
   if (!wl) return fail(LP_ERR_INVALID_ARG, "null workload");
   if (wl->kind != LP_WL_TMM && wl->kind != LP_WL_STENCIL5) return fail(LP_ERR_INVALID_ARG, "unknown workload kind %d", wl->kind);
-  if ((wl->in_dtype != LP_F32 && wl->in_dtype != LP_BF16) || (wl->out_dtype != LP_F32 && wl->out_dtype != LP_BF16))
+  if (wl->in_dtype < LP_F32 || wl->in_dtype > LP_I32 || wl->out_dtype < LP_F32 || wl->out_dtype > LP_I32)
     return fail(LP_ERR_INVALID_ARG, "unknown dtype");
+  if ((wl->in_dtype == LP_I32) != (wl->out_dtype == LP_I32))
+    return fail(LP_ERR_UNSUPPORTED, "int32 TMM needs int32 input and output");
   if (wl->m <= 0 || wl->n <= 0) return fail(LP_ERR_INVALID_ARG, "m and n must be positive");
   const int RM = h->cfg.region_m, RN = h->cfg.region_n;
   if (wl->m % RM || wl->n % RN)
@@ -220,6 +222,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.K = wl->k;
   a.in_bf16 = wl->in_dtype == LP_BF16;
   a.out_bf16 = wl->out_dtype == LP_BF16;
+  a.i32 = wl->in_dtype == LP_I32;
   a.RM = g.RM;
   a.RN = g.RN;
   a.mask = h->mask;
@@ -233,8 +236,8 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.sm_count = h->sm_count;
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
-  const bool tf_ok = lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, a.out_bf16, wl->lda,
-                                            wl->ldb, wl->ldc, wl->a, wl->b, out);
+  const bool tf_ok = !a.i32 && lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, a.out_bf16,
+                                                       wl->lda, wl->ldb, wl->ldc, wl->a, wl->b, out);
   int body = h->cfg.body;
   if (body == LP_BODY_AUTO) body = (tc_ok || tf_ok) ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
   if (body == LP_BODY_TCGEN05) {

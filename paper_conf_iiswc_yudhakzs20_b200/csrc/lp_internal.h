@@ -54,6 +54,7 @@ struct TmmArgs {
   int64_t ldc;
   int64_t M, N, K;
   int in_bf16, out_bf16;
+  int i32;  // int32 in/out (SIMT body, integer multiply-add)
   int RM, RN;
   uint32_t mask;
   HashInfo hash;

@@ -25,12 +25,50 @@ namespace {
 constexpr int kThreads = 256;
 constexpr int kBK = 16;
 
+// compute type: fp32 for float / bf16 operands (FFMA), int32 for the paper's int TMM (IMAD, wrapping)
 template <typename T>
-__device__ __forceinline__ float to_f(T v);
+struct Acc {
+  using type = float;
+};
 template <>
-__device__ __forceinline__ float to_f<float>(float v) { return v; }
+struct Acc<int32_t> {
+  using type = int32_t;
+};
+template <typename T>
+__device__ __forceinline__ typename Acc<T>::type to_acc(T v) {
+  return v;
+}
 template <>
-__device__ __forceinline__ float to_f<__nv_bfloat16>(__nv_bfloat16 v) { return __bfloat162float(v); }
+__device__ __forceinline__ float to_acc<__nv_bfloat16>(__nv_bfloat16 v) {
+  return __bfloat162float(v);
+}
+__device__ __forceinline__ float mac(float a, float b, float c) { return fmaf(a, b, c); }
+__device__ __forceinline__ int32_t mac(int32_t a, int32_t b, int32_t c) {
+  return (int32_t)((uint32_t)a * (uint32_t)b + (uint32_t)c);
+}
+// Fragment loads from shared memory, explicitly vectorised so the protected kernel
+// and its unprotected twin compile to the same mainloop (the overhead denominator).
+template <int U, typename TA>
+__device__ __forceinline__ void load_frag(TA* dst, const TA* src) {
+  static_assert(sizeof(TA) == 4, "32-bit compute types");
+  if constexpr (U % 4 == 0) {
+#pragma unroll
+    for (int i = 0; i < U; i += 4) *reinterpret_cast<uint4*>(dst + i) = *reinterpret_cast<const uint4*>(src + i);
+  } else if constexpr (U % 2 == 0) {
+#pragma unroll
+    for (int i = 0; i < U; i += 2) *reinterpret_cast<uint2*>(dst + i) = *reinterpret_cast<const uint2*>(src + i);
+  } else {
+#pragma unroll
+    for (int i = 0; i < U; ++i) dst[i] = src[i];
+  }
+}
+
+template <typename T>
+__device__ __forceinline__ uint32_t word_of(T v);
+template <>
+__device__ __forceinline__ uint32_t word_of<float>(float v) { return __float_as_uint(v); }
+template <>
+__device__ __forceinline__ uint32_t word_of<int32_t>(int32_t v) { return (uint32_t)v; }
 
 template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE>
 __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
@@ -47,9 +85,10 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
   constexpr int B_PER = BN * kBK / kThreads;
   static_assert(A_PER >= 1 && B_PER >= 1, "tile too small");
   constexpr int ES = (int)sizeof(TOut);
+  using TA = typename Acc<TIn>::type;
 
-  __shared__ float As[2][kBK][BM + 4];
-  __shared__ float Bs[2][kBK][BN + 4];
+  __shared__ __align__(16) TA As[2][kBK][BM + 4];
+  __shared__ __align__(16) TA Bs[2][kBK][BN + 4];
   __shared__ CkRecord warp_rec[kThreads / 32];
 
   const int tid = threadIdx.x;
@@ -61,25 +100,25 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
     const int64_t p = rid / Q, q = rid - p * Q;
     const int64_t row0 = p * BM, col0 = q * BN;
 
-    float acc[UM][UN];
+    TA acc[UM][UN];
 #pragma unroll
     for (int i = 0; i < UM; ++i)
 #pragma unroll
-      for (int j = 0; j < UN; ++j) acc[i][j] = 0.f;
+      for (int j = 0; j < UN; ++j) acc[i][j] = TA(0);
 
-    float ra[A_PER], rb[B_PER];
+    TA ra[A_PER], rb[B_PER];
     auto gload = [&](int64_t k0) {
 #pragma unroll
       for (int i = 0; i < A_PER; ++i) {
         const int e = tid + i * kThreads;
         const int m = e / kBK, k = e % kBK;
-        ra[i] = to_f(A[(row0 + m) * lda + k0 + k]);
+        ra[i] = to_acc(A[(row0 + m) * lda + k0 + k]);
       }
 #pragma unroll
       for (int i = 0; i < B_PER; ++i) {
         const int e = tid + i * kThreads;
         const int k = e / BN, n = e % BN;
-        rb[i] = to_f(B[(k0 + k) * ldb + col0 + n]);
+        rb[i] = to_acc(B[(k0 + k) * ldb + col0 + n]);
       }
     };
     auto sstore = [&](int buf) {
@@ -105,15 +144,13 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
       if (kt + 1 < nk) gload((kt + 1) * kBK);
 #pragma unroll
       for (int k = 0; k < kBK; ++k) {
-        float a[UM], b[UN];
-#pragma unroll
-        for (int i = 0; i < UM; ++i) a[i] = As[buf][k][ty * UM + i];
-#pragma unroll
-        for (int j = 0; j < UN; ++j) b[j] = Bs[buf][k][tx * UN + j];
+        TA a[UM], b[UN];
+        load_frag<UM>(a, &As[buf][k][ty * UM]);
+        load_frag<UN>(b, &Bs[buf][k][tx * UN]);
 #pragma unroll
         for (int i = 0; i < UM; ++i)
 #pragma unroll
-          for (int j = 0; j < UN; ++j) acc[i][j] = fmaf(a[i], b[j], acc[i][j]);
+          for (int j = 0; j < UN; ++j) acc[i][j] = mac(a[i], b[j], acc[i][j]);
       }
       if (kt + 1 < nk) sstore(buf ^ 1);
       __syncthreads();
@@ -129,9 +166,10 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
       for (int j = 0; j < UN; j += 2) {
         uint32_t w0, w1 = 0;
         if constexpr (ES == 4) {
-          w0 = __float_as_uint(acc[i][j]);
-          w1 = __float_as_uint(acc[i][j + 1]);
-          *reinterpret_cast<float2*>(crow + j) = make_float2(acc[i][j], acc[i][j + 1]);
+          const TOut o0 = (TOut)acc[i][j], o1 = (TOut)acc[i][j + 1];
+          w0 = word_of<TOut>(o0);
+          w1 = word_of<TOut>(o1);
+          *reinterpret_cast<uint2*>(crow + j) = make_uint2(w0, w1);
         } else {
           __nv_bfloat162 h = __floats2bfloat162_rn(acc[i][j], acc[i][j + 1]);  // .x (even col) -> low half
           w0 = *reinterpret_cast<uint32_t*>(&h);
@@ -208,6 +246,7 @@ bool tmm_simt_supported(int RM, int RN, int, int) {
 }
 
 cudaError_t launch_tmm_simt(const TmmArgs& a, cudaStream_t st) {
+  if (a.i32) return launch_shape<int32_t, int32_t>(a, st);
   if (a.in_bf16) {
     return a.out_bf16 ? launch_shape<__nv_bfloat16, __nv_bfloat16>(a, st) : launch_shape<__nv_bfloat16, float>(a, st);
   }

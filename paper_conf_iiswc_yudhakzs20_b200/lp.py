@@ -23,7 +23,7 @@ LIB_PATH = os.path.join(_HERE, "liblp.so")
 LP_OK, LP_ERR_INVALID_ARG, LP_ERR_UNSUPPORTED, LP_ERR_CUDA, LP_ERR_CAPACITY, LP_ERR_STATE = range(6)
 CK_NONE, CK_MOD, CK_XOR, CK_ADLER32 = 0, 1, 2, 4
 STORE_ARRAY, STORE_QUAD_CAS, STORE_QUAD_LOCK = 0, 1, 2
-F32, BF16 = 0, 1
+F32, BF16, I32 = 0, 1, 2
 WL_TMM, WL_STENCIL5 = 0, 1
 BODY_AUTO, BODY_SIMT, BODY_TCGEN05 = 0, 1, 2
 FLAG_TC_1CTA = 1
@@ -134,7 +134,7 @@ def _stream(stream) -> Optional[int]:
     return stream.cuda_stream
 
 
-_DT = {"f32": F32, "fp32": F32, "float32": F32, "bf16": BF16, "bfloat16": BF16}
+_DT = {"f32": F32, "fp32": F32, "float32": F32, "bf16": BF16, "bfloat16": BF16, "i32": I32, "int32": I32}
 
 
 def _dt_of(x) -> int:
@@ -143,7 +143,7 @@ def _dt_of(x) -> int:
     if isinstance(x, str):
         return _DT[x]
     import torch
-    return {torch.float32: F32, torch.bfloat16: BF16}[x]
+    return {torch.float32: F32, torch.bfloat16: BF16, torch.int32: I32}[x]
 
 
 @dataclass
@@ -267,7 +267,7 @@ class LP:
         """Allocate out, cksum, failed list, d_n (int64[1]) and workspace on the device."""
         import torch
         dev = torch.device("cuda", self.device if device is None else device)
-        dt = torch.bfloat16 if wl.out_dtype == BF16 else torch.float32
+        dt = {BF16: torch.bfloat16, F32: torch.float32, I32: torch.int32}[wl.out_dtype]
         R = self.num_regions(wl)
         out = torch.empty((wl.m, wl.ldc), dtype=dt, device=dev)[:, :wl.n]
         ckb = max(self.cksum_bytes(wl), 16)

@@ -13,6 +13,8 @@ def host_to_dev(arr: np.ndarray, dtype: str, device="cuda"):
         t = torch.from_numpy(np.ascontiguousarray(arr).view(np.int16)).view(torch.bfloat16)
     elif dtype == "f32":
         t = torch.from_numpy(np.ascontiguousarray(arr, dtype=np.float32))
+    elif dtype == "i32":
+        t = torch.from_numpy(np.ascontiguousarray(arr, dtype=np.int32))
     else:
         raise ValueError(dtype)
     return t.to(device)

@@ -49,7 +49,9 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
             p, q = divmod(int(rid), Q)
             ref = oracle.gemm_block_f64(A, B, p * RM, q * RN, RM, RN)
             got = golden[p * RM:(p + 1) * RM, q * RN:(q + 1) * RN]
-            if kind != "uniform":                       # integer-valued: bit-exact (Reading R18)
+            if out_dt == "i32":                         # the paper's int TMM (Listing 2): exact
+                assert np.array_equal(got.view(np.int32), ref.astype(np.int64).astype(np.int32)), rid
+            elif kind != "uniform":                     # integer-valued: bit-exact (Reading R18)
                 exp = ref.astype(np.float32) if out_dt == "f32" else oracle.round_bf16(ref)
                 assert np.array_equal(got, exp), rid
             else:
@@ -234,3 +236,12 @@ def test_tf32x3_matches_simt_integer_valued():
         torch.cuda.synchronize()
         res.append((dev_to_host(out), dev_to_host(ck)))
     assert np.array_equal(res[0][0], res[1][0]) and np.array_equal(res[0][1], res[1][1])
+
+
+
+# ----------------------------------------------------------------------------- int32 (the paper's TMM type)
+@pytest.mark.parametrize("mask", ["mod|xor", "mod|xor|adler"])
+@pytest.mark.parametrize("mode", ["stale_words", "bitflip"])
+def test_int32_tmm_paper_shape(mask, mode):
+    """Listing 2's int TMM with 32x32 thread-block regions (Table III: TMM = 32x32 blocks)."""
+    run_cycle(256, 320, 192, 32, 32, "i32", "i32", "int17", mask, "simt", mode=mode, frac=0.1)

@@ -340,3 +340,12 @@ def test_synth_column_block_matches_full():
     full = gen.generate(4, 16, 40, "int5", "bf16")
     blk = gen.generate(4, 16, 8, "int5", "bf16", ncols_global=40, col0=24)
     assert np.array_equal(full[:, 24:32], blk)
+
+
+def test_gemm_int32_operands_vs_numpy_int64():
+    A = gen.generate(3, 32, 128, "int17", "i32")
+    B = gen.generate(4, 128, 48, "int5", "i32")
+    assert A.dtype == np.int32
+    ref = A.astype(np.int64) @ B.astype(np.int64)
+    got = oracle.gemm_block_f64(A, B, 0, 16, 32, 32)
+    assert np.array_equal(got.astype(np.int64), ref[:, 16:48])
