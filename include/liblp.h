@@ -192,6 +192,19 @@ LP_API lp_status lp_inject(lp_handle h, const lp_workload_t* wl, void* out, void
  * ARRAY store: {0, 0}. */
 LP_API lp_status lp_stats(lp_handle h, const lp_workload_t* wl, const void* cksum, int64_t* d_stats, lp_stream_t stream);
 
+/* False-negative study (NEXT row N3, L53/L192 "random error injection"): run `trials`
+ * seeded corruption trials of a region of `region_words` 32-bit words under
+ * `model` (0 random words, 1 bit flips, 2 adversarial same-bit pair, 3 zeroed
+ * words; k in [1, kmax] corruptions, kmax <= 8) and count, in device
+ * d_counts (uint64[7]): {trials that changed the region, undetected by MOD, XOR,
+ * MOD|XOR, ADLER32, MOD|XOR|ADLER32, no-op trials}.  The first dump_trials trials
+ * are written to device dump (uint32[dump_trials][26]: k, positions[8], old
+ * words[8], new words[8], detected bits MOD=1 XOR=2 ADLER=4, changed=8) for
+ * re-checking against the CPU oracle; dump may be NULL. */
+LP_API lp_status lp_fn_study(lp_handle h, uint32_t model, int32_t kmax, int64_t region_words, uint64_t seed,
+                             int64_t trials, uint64_t* d_counts, uint32_t* dump, int64_t dump_trials,
+                             lp_stream_t stream);
+
 /* Number of SMs / cached device properties are queried lazily; this returns
  * the device's SM count (0 if no device). */
 LP_API int32_t lp_device_sm_count(lp_handle h);

@@ -453,4 +453,18 @@ lp_status lp_stats(lp_handle h, const lp_workload_t* wl, const void* cksum, int6
   return e == cudaSuccess ? ok() : cuda_fail(e, "stats launch");
 }
 
+lp_status lp_fn_study(lp_handle h, uint32_t model, int32_t kmax, int64_t region_words, uint64_t seed, int64_t trials,
+                      uint64_t* d_counts, uint32_t* dump, int64_t dump_trials, lp_stream_t stream) {
+  if (!h || !d_counts) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (model > 3 || kmax < 1 || kmax > 8 || region_words < 2 || trials < 0 || dump_trials < 0)
+    return fail(LP_ERR_INVALID_ARG, "model 0..3, kmax 1..8, region_words >= 2");
+  if (dump_trials > 0 && !dump) return fail(LP_ERR_INVALID_ARG, "null dump");
+  lp_status s;
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e = lp::launch_fn_study(seed, trials, region_words, (int)model, kmax, (unsigned long long*)d_counts,
+                                      dump, dump_trials, h->sm_count, (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "fn_study launch");
+}
+
 }  // extern "C"

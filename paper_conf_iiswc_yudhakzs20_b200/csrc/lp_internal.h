@@ -98,4 +98,9 @@ struct StencilArgs {
 bool stencil_supported(int RM, int RN);
 cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st);
 
+// ---- fn_study.cu : false-negative study (N3)
+cudaError_t launch_fn_study(uint64_t seed, int64_t trials, int64_t nwords, int mode, int kmax,
+                            unsigned long long* counts, uint32_t* dump, int64_t dump_trials, int sm_count,
+                            cudaStream_t st);
+
 }  // namespace lp

@@ -35,7 +35,7 @@ BODY_NAMES = {"auto": 0, "simt": 1, "tcgen05": 2}
 INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 3}
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",
             "lp_run_protected", "lp_validate", "lp_recover", "lp_region_checksums", "lp_inject", "lp_stats",
-            "lp_device_sm_count", "lp_last_error", "lp_abi_version"]
+            "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study"]
 
 
 def parse_cksum(spec) -> int:
@@ -97,6 +97,7 @@ def lib():
             "lp_region_checksums": [P, pw, P, P, P],
             "lp_inject": [P, pw, P, P, P, P, I64, U32, U64, P],
             "lp_stats": [P, pw, P, P, P],
+            "lp_fn_study": [P, U32, ctypes.c_int32, I64, U64, I64, P, P, I64, P],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -261,6 +262,13 @@ class LP:
 
     def stats(self, wl, ck, d_stats, stream=None):
         _check(lib().lp_stats(self._h, ctypes.byref(wl.c()), _ptr(ck), _ptr(d_stats), _stream(stream)))
+
+    def fn_study(self, model, kmax, region_words, seed, trials, d_counts, dump=None, dump_trials=0, stream=None):
+        """False-negative study (N3): see lp_fn_study in include/liblp.h."""
+        m = {"random_words": 0, "bitflips": 1, "adversarial": 2, "zeroed": 3}[model] if isinstance(model, str) \
+            else int(model)
+        _check(lib().lp_fn_study(self._h, m, kmax, region_words, seed, trials, _ptr(d_counts), _ptr(dump),
+                                 dump_trials, _stream(stream)))
 
     # ---- buffer helper (torch allocations; the caller owns them)
     def alloc(self, wl: Workload, device=None):
