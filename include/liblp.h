@@ -175,6 +175,15 @@ LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* o
 LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
                             const int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 
+/* The paper's own recovery form (Listing 7; NEXT row N2): ONE kernel
+ * with the grid of the original kernel, in which every CTA validates its region
+ * and, if the check fails, re-executes the region in place (data and record).
+ * *d_n_recovered (device int64, zeroed by the call) receives the number of
+ * re-executed regions.  No failed list is produced.  STENCIL5 workloads only
+ * (LP_ERR_UNSUPPORTED otherwise). */
+LP_API lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
+                                  int64_t* d_n_recovered, lp_stream_t stream);
+
 /* Records of every region of `out` (uint32 [R][selem], order MOD, XOR, ADLER)
  * without comparing -- for parity tests against the oracle. */
 LP_API lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,

@@ -403,6 +403,38 @@ lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksu
   return run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace);
 }
 
+lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, int64_t* d_n_recovered,
+                           lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (wl->kind != LP_WL_STENCIL5) return fail(LP_ERR_UNSUPPORTED, "same-grid check-and-recover: STENCIL5 only");
+  if (h->mask == 0) return fail(LP_ERR_STATE, "check-and-recover needs a checksum (cfg.cksum != 0)");
+  if (!out || !cksum || !d_n_recovered || !wl->a) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (!lp::stencil_supported(g.RM, g.RN)) return fail(LP_ERR_UNSUPPORTED, "stencil supports 128x128 regions");
+  if (!aligned16(wl->a) || !aligned16(out) || (wl->lda * 4) % 16) return fail(LP_ERR_INVALID_ARG, "stencil buffers must be 16-B aligned");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  lp::StencilArgs a;
+  a.in = (const float*)wl->a;
+  a.ldi = wl->lda;
+  a.out = (float*)out;
+  a.ldo = wl->ldc;
+  a.H = wl->m;
+  a.W = wl->n;
+  a.RM = g.RM;
+  a.RN = g.RN;
+  a.mask = h->mask;
+  a.hash = hash_info(h, g);
+  a.ck = (uint32_t*)cksum;
+  a.rid_offset = g.rid_offset;
+  a.list = nullptr;
+  a.d_n = nullptr;
+  a.sm_count = h->sm_count;
+  cudaError_t e = lp::launch_stencil_check_recover(a, d_n_recovered, (cudaStream_t)stream);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "check-and-recover launch");
+}
+
 lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,
                               lp_stream_t stream) {
   lp::RegionGeom g;

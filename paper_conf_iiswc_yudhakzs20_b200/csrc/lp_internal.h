@@ -97,6 +97,9 @@ struct StencilArgs {
 };
 bool stencil_supported(int RM, int RN);
 cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st);
+// Listing 7's same-grid check-and-recover (N2): one CTA per region validates and, on
+// mismatch, re-executes in place; *d_recovered (zeroed here) counts re-executed regions.
+cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recovered, cudaStream_t st);
 
 // ---- fn_study.cu : false-negative study (N3)
 cudaError_t launch_fn_study(uint64_t seed, int64_t trials, int64_t nwords, int mode, int kmax,

@@ -66,12 +66,52 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
     if (threadIdx.x < 5) s_acc[threadIdx.x] = 0u;
     __syncthreads();
   }
-  const int64_t ntiles = list ? *d_n : R;
+  __shared__ int s_bad;
+  const int64_t ntiles = (list && COMBINE != 2) ? *d_n : R;
   for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-    const int64_t rid = list ? (list[t] - rid_offset) : t;
+    const int64_t rid = (list && COMBINE != 2) ? (list[t] - rid_offset) : t;
     const int64_t p = rid / Q, q = rid - p * Q;
     const int i0 = (int)(p * kRM) + wid * kRowsW;
     const int j = (int)(q * kRN) + lane * 4;
+    if constexpr (COMBINE == 2) {
+      // Listing 7 (L565-578): check-and-recover in the same grid as the original kernel --
+      // validate this region from memory (L183), re-execute it only if the check fails.
+      CkPartial<MASK> vp;
+#pragma unroll
+      for (int r = 0; r < kRowsW; ++r) {
+        const uint4 w4 = ld_stream_u4(out + (int64_t)(i0 + r) * ldo + j);
+        const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
+        vp.add(w4.x, pos);
+        vp.add(w4.y, pos + 4);
+        vp.add(w4.z, pos + 8);
+        vp.add(w4.w, pos + 12);
+      }
+      const CkRecord vr = warp_reduce<MASK>(vp);
+      if (lane == 0) warp_rec[wid] = vr;
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        CkRecord rr = warp_rec[0];
+#pragma unroll
+        for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
+        uint32_t words[3];
+        record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
+        constexpr int S = selem_of(MASK);
+        bool bad = false;
+        if constexpr (STORE == 0) {
+#pragma unroll
+          for (int s2 = 0; s2 < S; ++s2) bad |= (ck[rid * S + s2] != words[s2]);
+        } else {
+          uint32_t stored[3];
+          bad = !quad_lookup<S>(ck, (uint32_t)(rid + rid_offset), stored);
+#pragma unroll
+          for (int s2 = 0; s2 < S; ++s2) bad |= (!bad && stored[s2] != words[s2]);
+        }
+        s_bad = bad ? 1 : 0;
+        if (bad) atomicAdd(reinterpret_cast<unsigned long long*>(const_cast<int64_t*>(d_n)), 1ull);
+      }
+      __syncthreads();
+      if (!s_bad) continue;  // uniform across the CTA
+    }
     const int je = lane == 0 ? j - 1 : j + 4;
     const bool eok = (lane == 0 || lane == 31) && je >= 0 && je < W;
     float4 v[kRowsW + 2];
@@ -129,6 +169,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       }
     } else if constexpr (MASK != 0) {
       const CkRecord wr = warp_reduce<MASK>(part);
+      __syncthreads();  // warp_rec may still be read by the check phase (COMBINE == 2)
       if (lane == 0) warp_rec[wid] = wr;
       __syncthreads();
       if (threadIdx.x == 0) {
@@ -139,7 +180,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
         record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
         store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
       }
-      if (list) __syncthreads();
+      if (list || COMBINE == 2) __syncthreads();
     }
   }
 }
@@ -180,6 +221,34 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
     LP_LCASE3(7)
 #undef LP_LCASE3
 #undef LP_LCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recovered, cudaStream_t st) {
+  const int64_t Q = a.W / kRN, R = (a.H / kRM) * Q;
+  if (a.H > (int64_t)INT32_MAX / 2 || a.W > (int64_t)INT32_MAX / 2 || a.mask == 0) return cudaErrorInvalidValue;
+  cudaError_t e = cudaMemsetAsync(d_recovered, 0, sizeof(int64_t), st);
+  if (e != cudaSuccess) return e;
+  const int sk = a.hash.store;
+  switch (a.mask * 3 + sk) {
+#define LP_CCASE(M, S)                                                                                          \
+  case M * 3 + S:                                                                                               \
+    stencil5_ldg_kernel<M, S, 2><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H, (int)a.W, Q,  \
+                                                              R, a.ck, a.rid_offset, nullptr, d_recovered);     \
+    break;
+#define LP_CCASE3(M) LP_CCASE(M, 0) LP_CCASE(M, 1) LP_CCASE(M, 2)
+    LP_CCASE3(1)
+    LP_CCASE3(2)
+    LP_CCASE3(3)
+    LP_CCASE3(4)
+    LP_CCASE3(5)
+    LP_CCASE3(6)
+    LP_CCASE3(7)
+#undef LP_CCASE3
+#undef LP_CCASE
     default:
       return cudaErrorInvalidValue;
   }

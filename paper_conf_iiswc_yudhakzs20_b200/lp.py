@@ -35,7 +35,7 @@ BODY_NAMES = {"auto": 0, "simt": 1, "tcgen05": 2}
 INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 3}
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",
             "lp_run_protected", "lp_validate", "lp_recover", "lp_region_checksums", "lp_inject", "lp_stats",
-            "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study"]
+            "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study", "lp_check_recover"]
 
 
 def parse_cksum(spec) -> int:
@@ -98,6 +98,7 @@ def lib():
             "lp_inject": [P, pw, P, P, P, P, I64, U32, U64, P],
             "lp_stats": [P, pw, P, P, P],
             "lp_fn_study": [P, U32, ctypes.c_int32, I64, U64, I64, P, P, I64, P],
+            "lp_check_recover": [P, pw, P, P, P, P],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -251,6 +252,11 @@ class LP:
     def recover(self, wl, out, ck, failed, d_n, workspace=None, stream=None):
         _check(lib().lp_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), _ptr(d_n),
                                 _ptr(workspace), _stream(stream)))
+
+    def check_recover(self, wl, out, ck, d_n_recovered, stream=None):
+        """Listing 7's same-grid check-and-recover (N2): validate + in-place re-execution in one kernel."""
+        _check(lib().lp_check_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(d_n_recovered),
+                                      _stream(stream)))
 
     def region_checksums(self, wl, out, records, stream=None):
         _check(lib().lp_region_checksums(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(records), _stream(stream)))

@@ -68,3 +68,41 @@ def test_stencil_checksums_and_modes(mask, mode):
 
 def test_stencil_quad_store():
     stencil_cycle(512, 512, "uniform", "mod|xor", "stale_words", 0.25, store="quad_cas")
+
+
+
+@pytest.mark.parametrize("frac", [0.01, 0.10, 0.50])
+@pytest.mark.parametrize("store", ["array", "quad_cas"])
+def test_same_grid_check_and_recover(frac, store):
+    """Listing 7 (N2): one kernel validates every region and re-executes the failed ones in place;
+    the result equals the golden output and the count equals the oracle's failed set."""
+    H, W = 1024, 768
+    h = lp.LP(128, 128, cksum="mod|xor", store=store)
+    X = gen.generate(3, H, W, "uniform", "f32")
+    x = host_to_dev(X, "f32")
+    wl = lp.Workload.stencil(x)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = host_to_dev(gen.generate(503, H, W, "bits", "f32"), "f32")
+    out.copy_(stale)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    torch.cuda.synchronize()
+    golden = dev_to_host(out)
+    R = h.num_regions(wl)
+    inj = torch.from_numpy(lp.choose_regions(R, frac, 1003)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=1003)
+    torch.cuda.synchronize()
+    if store == "array":
+        exp = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * 2], 128, 128, 3)
+    else:
+        ckh = dev_to_host(ck)
+        cap = int(ckh[0])
+        exp = oracle.validate_quad(dev_to_host(out), ckh[16:16 + cap * 3], cap, int(ckh[1]), 128, 128, 3)
+    d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+    h.check_recover(wl, out, ck, d_rec)
+    torch.cuda.synchronize()
+    assert int(d_rec.item()) == len(exp) == inj.numel()
+    assert np.array_equal(dev_to_host(out).view(np.uint32), golden.view(np.uint32))
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
