@@ -76,8 +76,17 @@ typedef enum { LP_CK_NONE = 0u, LP_CK_MOD = 1u, LP_CK_XOR = 2u, LP_CK_ADLER32 = 
 /* Checksum store.  ARRAY is the paper's hash-table-less global array indexed
  * by region id (L349, §V).  QUAD_CAS is the lock-free quadratic-probing table
  * (atomicCAS on the key slot, L267-272); QUAD_LOCK the same table with every
- * insert inside one global spin lock (L81-83, L341 Table III, Reading R15). */
-typedef enum { LP_STORE_ARRAY = 0, LP_STORE_QUAD_CAS = 1, LP_STORE_QUAD_LOCK = 2 } lp_store;
+ * insert inside one global spin lock (L81-83, L341 Table III, Reading R15).
+ * CUCKOO is the two-table cuckoo table with atomicExch inserts (L269-274;
+ * 16-byte entries moved by one 128-bit exchange, Reading R24); CUCKOO_LOCK the
+ * same under the global lock.  Hash stores are built for MOD and MOD|XOR. */
+typedef enum {
+  LP_STORE_ARRAY = 0,
+  LP_STORE_QUAD_CAS = 1,
+  LP_STORE_QUAD_LOCK = 2,
+  LP_STORE_CUCKOO = 3,
+  LP_STORE_CUCKOO_LOCK = 4
+} lp_store;
 
 /* Element types.  LP_I32 (in = out = int32, wrapping integer multiply-add) is the
  * paper's own TMM type (Listing 2: int *a, *b, *c); SIMT body only. */
@@ -142,7 +151,9 @@ LP_API lp_status lp_num_regions(lp_handle h, const lp_workload_t* wl, int64_t* r
 
 /* Bytes of the checksum buffer.  ARRAY: R * 4 * selem (selem = popcount(cksum),
  * L528 "number of checksums in an element").  QUAD_*: 64-byte header + cap *
- * 4 * (1 + selem) with cap = smallest prime >= ceil(R / 0.7) (L267 load <= 70%). */
+ * 4 * (1 + selem) with cap = smallest prime >= ceil(R / 0.7) (L267 load <= 70%).
+ * CUCKOO*: 64-byte header + 2 tables * cap * 16 with cap = smallest prime >= R
+ * (total load <= 50%, L270). */
 LP_API lp_status lp_cksum_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
 
 /* Bytes of the scratch `workspace` lp_validate needs (flags + scan counters). */

@@ -71,6 +71,14 @@ def lib():
         L.lpo_quad_insert.argtypes = [_p, _u32, _i, _u32, _u32, _p]
         L.lpo_validate_quad.restype = _i64
         L.lpo_validate_quad.argtypes = [_p, _p, _u32, _u32, _i64, _i64, _i64, _i, _i, _i, _u32, _i64, _p]
+        L.lpo_cuckoo_hash.restype = _u32
+        L.lpo_cuckoo_hash.argtypes = [_i, _u32, _u32, _u32]
+        L.lpo_cuckoo_lookup.restype = _i
+        L.lpo_cuckoo_lookup.argtypes = [_p, _u32, _i, _u32, _u32, _p]
+        L.lpo_cuckoo_insert.restype = _u32
+        L.lpo_cuckoo_insert.argtypes = [_p, _u32, _i, _u32, _u32, _p, _i]
+        L.lpo_validate_cuckoo.restype = _i64
+        L.lpo_validate_cuckoo.argtypes = [_p, _p, _u32, _u32, _i64, _i64, _i64, _i, _i, _i, _u32, _i64, _p]
         L.lpo_gemm_block_f64.restype = None
         L.lpo_gemm_block_f64.argtypes = [_p, _i64, _p, _i64, _i, _i64, _i64, _i64, _i64, _i64, _p]
         L.lpo_round_bf16.restype = None
@@ -168,6 +176,38 @@ def validate_quad(out: np.ndarray, table: np.ndarray, cap: int, seed: int, RM: i
     failed = np.zeros(R, dtype=np.int64)
     nf = lib().lpo_validate_quad(_ptr(out), _ptr(table), cap, seed, M, N, N, _es(out), RM, RN, mask, rid_offset,
                                  _ptr(failed))
+    return failed[:nf].copy()
+
+
+def cuckoo_hash(t: int, key: int, seed: int, cap: int) -> int:
+    return int(lib().lpo_cuckoo_hash(t, key, seed, cap))
+
+
+def cuckoo_lookup(table: np.ndarray, cap: int, sel: int, key: int, seed: int):
+    """table: uint32 [2*cap*4] (T1 then T2, 16-byte entries {key, rec0, rec1, rec2})."""
+    table = np.ascontiguousarray(table, dtype=np.uint32).reshape(-1)
+    rec = np.zeros(max(sel, 1), dtype=np.uint32)
+    ok = lib().lpo_cuckoo_lookup(_ptr(table), cap, sel, key, seed, _ptr(rec))
+    return rec[:sel].copy() if ok else None
+
+
+def cuckoo_insert(table: np.ndarray, cap: int, sel: int, key: int, seed: int, rec, max_evict: int = 128) -> int:
+    assert table.flags.c_contiguous and table.dtype == np.uint32
+    r = np.ascontiguousarray(np.asarray(rec, dtype=np.uint32).reshape(-1))
+    if r.size == 0:
+        r = np.zeros(1, dtype=np.uint32)
+    return int(lib().lpo_cuckoo_insert(_ptr(table), cap, sel, key, seed, _ptr(r), max_evict))
+
+
+def validate_cuckoo(out: np.ndarray, table: np.ndarray, cap: int, seed: int, RM: int, RN: int, mask: int,
+                    rid_offset: int = 0) -> np.ndarray:
+    out = np.ascontiguousarray(out)
+    table = np.ascontiguousarray(table, dtype=np.uint32).reshape(-1)
+    M, N = out.shape
+    R = (M // RM) * (N // RN)
+    failed = np.zeros(R, dtype=np.int64)
+    nf = lib().lpo_validate_cuckoo(_ptr(out), _ptr(table), cap, seed, M, N, N, _es(out), RM, RN, mask, rid_offset,
+                                   _ptr(failed))
     return failed[:nf].copy()
 
 

@@ -192,6 +192,65 @@ int64_t lpo_validate_quad(const void* out, const uint32_t* table, uint32_t cap, 
 }
 
 /* ------------------------------------------------------------------------ */
+/* Cuckoo hashing (L269-270, Fig. 4): tables T1, T2 with hash functions H1, H2. */
+/* Insert puts the key at T1[H1(k)]; an occupant is evicted to the other table */
+/* (T2[H2(.)], then T1[H1(.)], ...); L270 "The lookup process ... find all    */
+/* possible indices pointed by all hashing functions".  Hash functions are     */
+/* unstated: Reading R24 = H1 = fmix32(k ^ seed) mod cap, H2 = fmix32(k ^      */
+/* (seed * 0x9E3779B9 + 0x7F4A7C15)) mod cap.  Entry = 4 u32: key, 3 record    */
+/* words (unused words 0).  Table t starts at entry t * cap.                  */
+uint32_t lpo_cuckoo_hash(int t, uint32_t key, uint32_t seed, uint32_t cap) {
+  return t == 0 ? lpo_quad_hash(key, seed, cap) : lpo_quad_hash(key, seed * 0x9E3779B9u + 0x7F4A7C15u, cap);
+}
+
+int lpo_cuckoo_lookup(const uint32_t* tab, uint32_t cap, int selem, uint32_t key, uint32_t seed, uint32_t* rec) {
+  for (int t = 0; t < 2; ++t) {
+    const uint32_t* e = tab + 4 * ((uint64_t)t * cap + lpo_cuckoo_hash(t, key, seed, cap));
+    if (e[0] == key) {
+      for (int s = 0; s < selem; ++s) rec[s] = e[1 + s];
+      return 1;
+    }
+  }
+  return 0;
+}
+
+/* Sequential insert; returns the number of placements (1 = no eviction), 0 if */
+/* the chain exceeds max_evict (the paper would rehash).                       */
+uint32_t lpo_cuckoo_insert(uint32_t* tab, uint32_t cap, int selem, uint32_t key, uint32_t seed, const uint32_t* rec,
+                           int max_evict) {
+  uint32_t e[4] = {key, 0, 0, 0};
+  for (int s = 0; s < selem; ++s) e[1 + s] = rec[s];
+  int t = 0;
+  for (int i = 0; i < max_evict; ++i) {
+    uint32_t* slot = tab + 4 * ((uint64_t)t * cap + lpo_cuckoo_hash(t, e[0], seed, cap));
+    uint32_t old[4];
+    memcpy(old, slot, 16);
+    memcpy(slot, e, 16);
+    if (old[0] == 0xFFFFFFFFu || old[0] == e[0]) return (uint32_t)i + 1;
+    memcpy(e, old, 16);
+    t ^= 1;
+  }
+  return 0;
+}
+
+int64_t lpo_validate_cuckoo(const void* out, const uint32_t* tab, uint32_t cap, uint32_t seed, int64_t M, int64_t N,
+                            int64_t ldc, int es, int RM, int RN, uint32_t mask, int64_t rid_offset, int64_t* failed) {
+  const int selem = lpo_selem(mask);
+  const int64_t P = M / RM, Q = N / RN;
+  int64_t nf = 0;
+  uint32_t rec[3], stored[3];
+  for (int64_t p = 0; p < P; ++p)
+    for (int64_t q = 0; q < Q; ++q) {
+      const int64_t rid = p * Q + q + rid_offset;
+      lpo_region_record(out, ldc, es, p, q, RM, RN, mask, rec);
+      int bad = !lpo_cuckoo_lookup(tab, cap, selem, (uint32_t)rid, seed, stored);
+      for (int s = 0; !bad && s < selem; ++s) bad |= (rec[s] != stored[s]);
+      if (bad) failed[nf++] = rid;
+    }
+  return nf;
+}
+
+/* ------------------------------------------------------------------------ */
 /* Region body 1: tiled matrix multiply (Listing 2, Listing 6        */
 /* L546-554): C = A * B, A [M x K] row-major, B [K x N] row-major.  Plain     */
 /* triple loop in fp64 for the RM x RN block at (row0, col0).  is_bf16 selects */

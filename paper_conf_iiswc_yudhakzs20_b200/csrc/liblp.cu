@@ -60,8 +60,9 @@ bool is_prime(uint64_t n) {
   return true;
 }
 
-uint32_t hash_cap(int64_t R) {
-  uint64_t c = (uint64_t)std::ceil((double)R / 0.7);
+// quadratic probing: load <= 70% (L267); cuckoo: per-table capacity, total load <= 50% (L270)
+uint32_t hash_cap(int64_t R, int store) {
+  uint64_t c = store >= LP_STORE_CUCKOO ? (uint64_t)R : (uint64_t)std::ceil((double)R / 0.7);
   if (c < 2) c = 2;
   while (!is_prime(c)) ++c;
   return (uint32_t)c;
@@ -143,14 +144,15 @@ struct DeviceGuard {
 lp::HashInfo hash_info(const lp_ctx* h, const lp::RegionGeom& g) {
   lp::HashInfo hi;
   hi.store = h->cfg.store;
-  hi.cap = h->cfg.store == LP_STORE_ARRAY ? 0u : hash_cap(g.R);
+  hi.cap = h->cfg.store == LP_STORE_ARRAY ? 0u : hash_cap(g.R, h->cfg.store);
   hi.seed = h->cfg.hash_seed;
   return hi;
 }
 
 size_t cksum_bytes(const lp_ctx* h, const lp::RegionGeom& g) {
   if (h->cfg.store == LP_STORE_ARRAY) return (size_t)g.R * 4u * (size_t)h->selem;
-  return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R) * 4u * (size_t)(1 + h->selem);
+  if (h->cfg.store >= LP_STORE_CUCKOO) return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R, h->cfg.store) * 2u * 16u;
+  return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R, h->cfg.store) * 4u * (size_t)(1 + h->selem);
 }
 
 // Tensor-core tiles covering the output, for recovery de-duplication: 128x128 tiles of
@@ -284,8 +286,10 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   *out = nullptr;
   if (cfg->region_m <= 0 || cfg->region_n <= 0) return fail(LP_ERR_INVALID_ARG, "region shape must be positive");
   if (cfg->cksum & ~7u) return fail(LP_ERR_INVALID_ARG, "unknown checksum bits 0x%x", cfg->cksum);
-  if (cfg->store < LP_STORE_ARRAY || cfg->store > LP_STORE_QUAD_LOCK) return fail(LP_ERR_INVALID_ARG, "unknown store %d", cfg->store);
+  if (cfg->store < LP_STORE_ARRAY || cfg->store > LP_STORE_CUCKOO_LOCK) return fail(LP_ERR_INVALID_ARG, "unknown store %d", cfg->store);
   if (cfg->store != LP_STORE_ARRAY && cfg->cksum == 0) return fail(LP_ERR_INVALID_ARG, "a hash store needs a checksum");
+  if (cfg->store != LP_STORE_ARRAY && cfg->cksum != LP_CK_MOD && cfg->cksum != (LP_CK_MOD | LP_CK_XOR))
+    return fail(LP_ERR_UNSUPPORTED, "hash stores (the ablation) are built for MOD and MOD|XOR records");
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)LP_FLAG_TC_1CTA) return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);

@@ -226,16 +226,112 @@ __device__ __forceinline__ bool quad_lookup(const uint32_t* ckbuf, uint32_t rid,
   return false;
 }
 
+// ---------------------------------------------------------------------------
+// Cuckoo store (L269-274, Fig. 4): two tables T1/T2 with hash functions H1/H2;
+// an insert puts the key at T1[H1(k)] and carries whatever it evicts to the other
+// table (T2[H2(.)], then T1[H1(.)], ...).  L274: "we use atomic exchange
+// (atomicExch()) ... we will always insert the entry to a hash table entry no
+// matter whether it is occupied or empty".  An entry is 16 bytes {key, rec0,
+// rec1, rec2} exchanged with ONE 128-bit atom.exch so a record always travels with
+// its key.  Per-table capacity = smallest prime >= R: total load <= 50% (L270).
+// A chain longer than kCuckooMaxEvict sets the error flag (the paper rehashes
+// with new functions; Reading R24).  Layout: HashHeader, T1[cap], T2[cap].
+constexpr int kCuckooMaxEvict = 128;
+
+__host__ __device__ __forceinline__ uint32_t cuckoo_h(int t, uint32_t key, uint32_t seed, uint32_t cap) {
+  return (t == 0 ? hash_fmix32(key, seed) : hash_fmix32(key, seed * 0x9E3779B9u + 0x7F4A7C15u)) % cap;
+}
+
+__device__ __forceinline__ uint4 atom_exch_128(uint4* p, uint4 v) {
+  const uint64_t lo = ((uint64_t)v.y << 32) | v.x, hi = ((uint64_t)v.w << 32) | v.z;
+  uint64_t olo, ohi;
+  asm volatile(
+      "{\n\t.reg .b128 d, b;\n\tmov.b128 b, {%2, %3};\n\tatom.global.exch.b128 d, [%4], b;\n\tmov.b128 {%0, %1}, d;\n\t}"
+      : "=l"(olo), "=l"(ohi)
+      : "l"(lo), "l"(hi), "l"(p)
+      : "memory");
+  return make_uint4((uint32_t)olo, (uint32_t)(olo >> 32), (uint32_t)ohi, (uint32_t)(ohi >> 32));
+}
+
+template <uint32_t MASK>
+__device__ __forceinline__ uint4 cuckoo_entry(uint32_t rid, const uint32_t* w) {
+  constexpr int S = selem_of(MASK);
+  return make_uint4(rid, S > 0 ? w[0] : 0u, S > 1 ? w[1] : 0u, S > 2 ? w[2] : 0u);
+}
+
+template <uint32_t MASK>
+__device__ __forceinline__ uint32_t cuckoo_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+  HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
+  uint4* tab = reinterpret_cast<uint4*>(ckbuf + sizeof(HashHeader) / 4);
+  const uint32_t cap = hdr->cap, seed = hdr->seed;
+  uint4 e = cuckoo_entry<MASK>(rid, w);
+  int t = 0;
+  for (int i = 0; i < kCuckooMaxEvict; ++i) {
+    const uint4 old = atom_exch_128(tab + (uint64_t)t * cap + cuckoo_h(t, e.x, seed, cap), e);
+    if (old.x == kEmptyKey || old.x == e.x) {  // empty slot, or the same key's stale entry (dropped)
+      if (i) atomicAdd(&hdr->collisions, (unsigned long long)i);
+      return (uint32_t)i + 1;
+    }
+    e = old;  // carry the evicted entry to its slot in the other table
+    t ^= 1;
+  }
+  atomicExch(&hdr->error, 1u);
+  return 0;
+}
+
+template <uint32_t MASK>
+__device__ __forceinline__ uint32_t cuckoo_insert_locked(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
+  HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
+  while (atomicCAS(&hdr->lock, 0u, 1u) != 0u) __nanosleep(32);
+  __threadfence();
+  const uint32_t r = cuckoo_insert<MASK>(ckbuf, rid, w);
+  __threadfence();
+  atomicExch(&hdr->lock, 0u);
+  return r;
+}
+
+template <int S>
+__device__ __forceinline__ bool cuckoo_lookup(const uint32_t* ckbuf, uint32_t rid, uint32_t* w) {
+  const HashHeader* hdr = reinterpret_cast<const HashHeader*>(ckbuf);
+  const uint4* tab = reinterpret_cast<const uint4*>(ckbuf + sizeof(HashHeader) / 4);
+  const uint32_t cap = hdr->cap, seed = hdr->seed;
+  for (int t = 0; t < 2; ++t) {
+    const uint4 e = tab[(uint64_t)t * cap + cuckoo_h(t, rid, seed, cap)];
+    if (e.x == rid) {
+      if (S > 0) w[0] = e.y;
+      if (S > 1) w[1] = e.z;
+      if (S > 2) w[2] = e.w;
+      return true;
+    }
+  }
+  return false;
+}
+
 // Record store, selected at compile time so the array-store kernels carry no
 // hash-table code (and no register pressure from it).
+// STORE: 0 array, 1 quad CAS, 2 quad + global lock, 3 cuckoo (atomicExch), 4 cuckoo + global lock.
 template <uint32_t MASK, int STORE>
 __device__ __forceinline__ void store_record(uint32_t* ck, int64_t local_rid, uint32_t global_rid, const uint32_t* w) {
   if constexpr (STORE == 0) {
     store_array<MASK>(ck, local_rid, w);
   } else if constexpr (STORE == 1) {
     quad_insert<MASK>(ck, global_rid, w);
-  } else {
+  } else if constexpr (STORE == 2) {
     quad_insert_locked<MASK>(ck, global_rid, w);
+  } else if constexpr (STORE == 3) {
+    cuckoo_insert<MASK>(ck, global_rid, w);
+  } else {
+    cuckoo_insert_locked<MASK>(ck, global_rid, w);
+  }
+}
+
+// Lookup dispatch for validation: returns false if the key is absent.
+template <int S, int STORE>
+__device__ __forceinline__ bool store_lookup(const uint32_t* ck, uint32_t global_rid, uint32_t* w) {
+  if constexpr (STORE == 3 || STORE == 4) {
+    return cuckoo_lookup<S>(ck, global_rid, w);
+  } else {
+    return quad_lookup<S>(ck, global_rid, w);
   }
 }
 

@@ -26,7 +26,7 @@ constexpr int kValUnroll = 8;
 // A region's W warp partials are combined through double-buffered shared slots
 // behind a named barrier of the W warps (Listing 3's block combine, per region).
 // MODE 0 = compare with array table, 1 = compare with a quad hash table (lookup
-// by global rid), 2 = write records (no compare).
+// by global rid), 2 = write records (no compare), 3 = compare with a cuckoo table.
 template <uint32_t MASK, int MODE, int W>
 __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
                                                                 int64_t Q, int64_t R, int RM, int row_bytes,
@@ -99,7 +99,8 @@ __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __
           for (int s = 0; s < S; ++s) bad |= (ck[r * S + s] != w[s]);
         } else {
           uint32_t stored[3];
-          bad = !quad_lookup<S>(ck, (uint32_t)(r + rid_offset), stored);
+          bad = MODE == 3 ? !cuckoo_lookup<S>(ck, (uint32_t)(r + rid_offset), stored)
+                          : !quad_lookup<S>(ck, (uint32_t)(r + rid_offset), stored);
 #pragma unroll
           for (int s = 0; s < S; ++s) bad |= (!bad && stored[s] != w[s]);
         }
@@ -129,6 +130,9 @@ cudaError_t validate_dispatch_w(int mode, const ValLaunch& L, cudaStream_t st, c
                                                                 rid_offset, flags, records, L.rpc, counts);
   else if (mode == 1)
     validate_kernel<MASK, 1, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
+                                                                rid_offset, flags, records, L.rpc, counts);
+  else if (mode == 3)
+    validate_kernel<MASK, 3, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
                                                                 rid_offset, flags, records, L.rpc, counts);
   else
     validate_kernel<MASK, 2, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
@@ -351,6 +355,18 @@ __global__ void inject_kernel(uint8_t* out, int64_t ldc_bytes, int64_t Q, int RM
     if (threadIdx.x == 0) {
       if (store == 0) {
         for (int s = 0; s < S; ++s) ck[r * S + s] = kSentinel;
+      } else if (store >= 3) {
+        const HashHeader* hdr = reinterpret_cast<const HashHeader*>(ck);
+        uint4* tab = reinterpret_cast<uint4*>(ck + sizeof(HashHeader) / 4);
+        for (int t = 0; t < 2; ++t) {
+          uint4* e = tab + (uint64_t)t * hdr->cap + cuckoo_h(t, (uint32_t)grid, hdr->seed, hdr->cap);
+          if (e->x == (uint32_t)grid) {
+            e->y = kSentinel;
+            e->z = kSentinel;
+            e->w = kSentinel;
+            break;
+          }
+        }
       } else {
         const HashHeader* hdr = reinterpret_cast<const HashHeader*>(ck);
         uint32_t* ent = ck + sizeof(HashHeader) / 4;
@@ -421,7 +437,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   int cpr_log2 = 0;
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
   const ValLaunch L = plan_validate(g, sm_count);
-  const int mode = records ? 2 : (hi.store == 0 ? 0 : 1);
+  const int mode = records ? 2 : (hi.store == 0 ? 0 : (hi.store <= 2 ? 1 : 3));
   const uint8_t* o = (const uint8_t*)out;
   const int64_t ldcb = g.ldc * g.es;
   cudaError_t e;

@@ -102,7 +102,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
           for (int s2 = 0; s2 < S; ++s2) bad |= (ck[rid * S + s2] != words[s2]);
         } else {
           uint32_t stored[3];
-          bad = !quad_lookup<S>(ck, (uint32_t)(rid + rid_offset), stored);
+          bad = !store_lookup<S, STORE>(ck, (uint32_t)(rid + rid_offset), stored);
 #pragma unroll
           for (int s2 = 0; s2 < S; ++s2) bad |= (!bad && stored[s2] != words[s2]);
         }
@@ -198,9 +198,9 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   // persistent CTAs over the failed list, barrier combine (accumulators reused)
   int64_t grid = a.list ? (R < a.sm_count * 2 ? R : a.sm_count * 2) : R;
   if (grid < 1) grid = 1;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_LCASE(M, S)                                                                                          \
-  case M * 3 + S:                                                                                               \
+  case M * 5 + S:                                                                                               \
     if (a.list)                                                                                                 \
       stencil5_ldg_kernel<M, S, 0><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H,         \
                                                                    (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
@@ -210,16 +210,18 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
                                                                    (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
                                                                    a.d_n);                                      \
     break;
-#define LP_LCASE3(M) LP_LCASE(M, 0) LP_LCASE(M, 1) LP_LCASE(M, 2)
+#define LP_LCASE3(M) LP_LCASE(M, 0)
+#define LP_LCASE5(M) LP_LCASE(M, 0) LP_LCASE(M, 1) LP_LCASE(M, 2) LP_LCASE(M, 3) LP_LCASE(M, 4)
     LP_LCASE(0, 0)
-    LP_LCASE3(1)
+    LP_LCASE5(1)
     LP_LCASE3(2)
-    LP_LCASE3(3)
+    LP_LCASE5(3)
     LP_LCASE3(4)
     LP_LCASE3(5)
     LP_LCASE3(6)
     LP_LCASE3(7)
 #undef LP_LCASE3
+#undef LP_LCASE5
 #undef LP_LCASE
     default:
       return cudaErrorInvalidValue;
@@ -233,21 +235,23 @@ cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recove
   cudaError_t e = cudaMemsetAsync(d_recovered, 0, sizeof(int64_t), st);
   if (e != cudaSuccess) return e;
   const int sk = a.hash.store;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_CCASE(M, S)                                                                                          \
-  case M * 3 + S:                                                                                               \
+  case M * 5 + S:                                                                                               \
     stencil5_ldg_kernel<M, S, 2><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H, (int)a.W, Q,  \
                                                               R, a.ck, a.rid_offset, nullptr, d_recovered);     \
     break;
-#define LP_CCASE3(M) LP_CCASE(M, 0) LP_CCASE(M, 1) LP_CCASE(M, 2)
-    LP_CCASE3(1)
+#define LP_CCASE3(M) LP_CCASE(M, 0)
+#define LP_CCASE5(M) LP_CCASE(M, 0) LP_CCASE(M, 1) LP_CCASE(M, 2) LP_CCASE(M, 3) LP_CCASE(M, 4)
+    LP_CCASE5(1)
     LP_CCASE3(2)
-    LP_CCASE3(3)
+    LP_CCASE5(3)
     LP_CCASE3(4)
     LP_CCASE3(5)
     LP_CCASE3(6)
     LP_CCASE3(7)
 #undef LP_CCASE3
+#undef LP_CCASE5
 #undef LP_CCASE
     default:
       return cudaErrorInvalidValue;

@@ -208,22 +208,24 @@ cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
   const TIn* B = (const TIn*)a.B;
   TOut* C = (TOut*)a.C;
   const int sk = a.mask ? a.hash.store : 0;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_SCASE(M, S)                                                                                         \
-  case M * 3 + S:                                                                                              \
+  case M * 5 + S:                                                                                              \
     tmm_simt_kernel<TIn, TOut, BM, BN, UM, UN, M, S><<<(unsigned)grid, kThreads, 0, st>>>(                     \
         A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.rid_offset, a.list, a.d_n);                           \
     break;
-#define LP_SCASE3(M) LP_SCASE(M, 0) LP_SCASE(M, 1) LP_SCASE(M, 2)
+#define LP_SCASE3(M) LP_SCASE(M, 0)
+#define LP_SCASE5(M) LP_SCASE(M, 0) LP_SCASE(M, 1) LP_SCASE(M, 2) LP_SCASE(M, 3) LP_SCASE(M, 4)
     LP_SCASE(0, 0)
-    LP_SCASE3(1)
+    LP_SCASE5(1)
     LP_SCASE3(2)
-    LP_SCASE3(3)
+    LP_SCASE5(3)
     LP_SCASE3(4)
     LP_SCASE3(5)
     LP_SCASE3(6)
     LP_SCASE3(7)
 #undef LP_SCASE3
+#undef LP_SCASE5
 #undef LP_SCASE
     default:
       return cudaErrorInvalidValue;

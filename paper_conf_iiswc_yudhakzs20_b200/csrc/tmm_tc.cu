@@ -407,25 +407,27 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   const int smem = Cfg::kSmemBytes;
   cudaError_t e = cudaSuccess;
   const int sk = a.mask ? a.hash.store : 0;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_TC_CASE(M, S)                                                                                    \
-  case M * 3 + S: {                                                                                         \
+  case M * 5 + S: {                                                                                         \
     auto kfn = tmm_tc_kernel<OutT, M, REG, BN, S>;                                                         \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
     if (e != cudaSuccess) return e;                                                                         \
     kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, src, a.ck);                \
     break;                                                                                                  \
   }
-#define LP_TC_CASE3(M) LP_TC_CASE(M, 0) LP_TC_CASE(M, 1) LP_TC_CASE(M, 2)
+#define LP_TC_CASE3(M) LP_TC_CASE(M, 0)
+#define LP_TC_CASE5(M) LP_TC_CASE(M, 0) LP_TC_CASE(M, 1) LP_TC_CASE(M, 2) LP_TC_CASE(M, 3) LP_TC_CASE(M, 4)
     LP_TC_CASE(0, 0)
-    LP_TC_CASE3(1)
+    LP_TC_CASE5(1)
     LP_TC_CASE3(2)
-    LP_TC_CASE3(3)
+    LP_TC_CASE5(3)
     LP_TC_CASE3(4)
     LP_TC_CASE3(5)
     LP_TC_CASE3(6)
     LP_TC_CASE3(7)
 #undef LP_TC_CASE3
+#undef LP_TC_CASE5
 #undef LP_TC_CASE
     default:
       return cudaErrorInvalidValue;
@@ -449,9 +451,9 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
   const int64_t Qr = a.N / REG;
   const int sk = a.mask ? a.hash.store : 0;
   cudaError_t e = cudaSuccess;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_TC2_CASE(M, S)                                                                                   \
-  case M * 3 + S: {                                                                                         \
+  case M * 5 + S: {                                                                                         \
     auto kfn = tmm_tc2_kernel<OutT, M, REG, S>;                                                            \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2Bytes);                \
     if (e != cudaSuccess) return e;                                                                         \
@@ -459,16 +461,18 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
                                                        a.rid_offset, a.ck);                                 \
     break;                                                                                                  \
   }
-#define LP_TC2_CASE3(M) LP_TC2_CASE(M, 0) LP_TC2_CASE(M, 1) LP_TC2_CASE(M, 2)
+#define LP_TC2_CASE3(M) LP_TC2_CASE(M, 0)
+#define LP_TC2_CASE5(M) LP_TC2_CASE(M, 0) LP_TC2_CASE(M, 1) LP_TC2_CASE(M, 2) LP_TC2_CASE(M, 3) LP_TC2_CASE(M, 4)
     LP_TC2_CASE(0, 0)
-    LP_TC2_CASE3(1)
+    LP_TC2_CASE5(1)
     LP_TC2_CASE3(2)
-    LP_TC2_CASE3(3)
+    LP_TC2_CASE5(3)
     LP_TC2_CASE3(4)
     LP_TC2_CASE3(5)
     LP_TC2_CASE3(6)
     LP_TC2_CASE3(7)
 #undef LP_TC2_CASE3
+#undef LP_TC2_CASE5
 #undef LP_TC2_CASE
     default:
       return cudaErrorInvalidValue;

@@ -359,25 +359,27 @@ cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
   const int sk = a.mask ? a.hash.store : 0;
   cudaError_t e = cudaSuccess;
   const int chunk_kb = kFChunkKB;
-  switch (a.mask * 3 + sk) {
+  switch (a.mask * 5 + sk) {
 #define LP_TF_CASE(M, S)                                                                                    \
-  case M * 3 + S: {                                                                                         \
+  case M * 5 + S: {                                                                                         \
     auto kfn = tmm_tf32x3_kernel<M, REG, S>;                                                               \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kFSmemBytes);                \
     if (e != cudaSuccess) return e;                                                                         \
     kfn<<<(unsigned)grid, kFThreads, kFSmemBytes, st>>>(ma, mb, (float*)a.C, a.ldc, a.K, tl, a.ck, chunk_kb); \
     break;                                                                                                  \
   }
-#define LP_TF_CASE3(M) LP_TF_CASE(M, 0) LP_TF_CASE(M, 1) LP_TF_CASE(M, 2)
+#define LP_TF_CASE3(M) LP_TF_CASE(M, 0)
+#define LP_TF_CASE5(M) LP_TF_CASE(M, 0) LP_TF_CASE(M, 1) LP_TF_CASE(M, 2) LP_TF_CASE(M, 3) LP_TF_CASE(M, 4)
     LP_TF_CASE(0, 0)
-    LP_TF_CASE3(1)
+    LP_TF_CASE5(1)
     LP_TF_CASE3(2)
-    LP_TF_CASE3(3)
+    LP_TF_CASE5(3)
     LP_TF_CASE3(4)
     LP_TF_CASE3(5)
     LP_TF_CASE3(6)
     LP_TF_CASE3(7)
 #undef LP_TF_CASE3
+#undef LP_TF_CASE5
 #undef LP_TF_CASE
     default:
       return cudaErrorInvalidValue;

@@ -22,7 +22,7 @@ LIB_PATH = os.path.join(_HERE, "liblp.so")
 # ---- enums (mirror include/liblp.h)
 LP_OK, LP_ERR_INVALID_ARG, LP_ERR_UNSUPPORTED, LP_ERR_CUDA, LP_ERR_CAPACITY, LP_ERR_STATE = range(6)
 CK_NONE, CK_MOD, CK_XOR, CK_ADLER32 = 0, 1, 2, 4
-STORE_ARRAY, STORE_QUAD_CAS, STORE_QUAD_LOCK = 0, 1, 2
+STORE_ARRAY, STORE_QUAD_CAS, STORE_QUAD_LOCK, STORE_CUCKOO, STORE_CUCKOO_LOCK = 0, 1, 2, 3, 4
 F32, BF16, I32 = 0, 1, 2
 WL_TMM, WL_STENCIL5 = 0, 1
 BODY_AUTO, BODY_SIMT, BODY_TCGEN05 = 0, 1, 2
@@ -30,7 +30,7 @@ FLAG_TC_1CTA = 1
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
-STORE_NAMES = {"array": 0, "quad_cas": 1, "quad": 1, "quad_lock": 2}
+STORE_NAMES = {"array": 0, "quad_cas": 1, "quad": 1, "quad_lock": 2, "cuckoo": 3, "cuckoo_lock": 4}
 BODY_NAMES = {"auto": 0, "simt": 1, "tcgen05": 2}
 INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 3}
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",

@@ -15,7 +15,7 @@ import torch
 import lpsynth
 import oracle
 from paper_conf_iiswc_yudhakzs20_b200 import lp, shard
-from tests.gpu_util import dev_to_host
+from tests.gpu_util import check_store_table, dev_to_host, oracle_validate
 
 pytestmark = pytest.mark.gpu
 
@@ -50,10 +50,7 @@ def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, globa
     if store == "array":
         assert np.array_equal(ckh[:R * sel].reshape(R, sel), recs)
     else:
-        cap, hseed = int(ckh[0]), int(ckh[1])
-        table = ckh[16:16 + cap * (1 + sel)]
-        for rid in range(R):
-            assert list(oracle.quad_lookup(table, cap, sel, rid0 + rid, hseed)) == list(recs[rid]), rid
+        check_store_table(ckh, store, R, sel, recs, rid0)
     # sampled values vs the fp64 oracle (inputs regenerated on the host by the shared generator)
     from lpsynth import gen
     Q = N // region
@@ -78,12 +75,7 @@ def _tmm_full(M, N, K, region, mask, store, kind, out_dt, nsample, row0=0, globa
     nf = int(d_n.item())
     got_failed = failed[:nf].cpu().numpy()
     bad, badck = dev_to_host(out), dev_to_host(ck)
-    if store == "array":
-        exp_failed = oracle.validate_array(bad, badck[:R * sel], region, region, h.mask, rid_offset=rid0)
-    else:
-        cap = int(badck[0])
-        exp_failed = oracle.validate_quad(bad, badck[16:16 + cap * (1 + sel)], cap, int(badck[1]), region, region,
-                                          h.mask, rid_offset=rid0)
+    exp_failed = oracle_validate(bad, badck, store, region, region, h.mask, rid_offset=rid0)
     assert np.array_equal(got_failed, exp_failed)
     assert set(got_failed.tolist()) <= set(inj.cpu().numpy().tolist()) and nf > 0
     h.recover(wl, out, ck, failed, d_n, ws)
@@ -119,6 +111,11 @@ def test_c2_tmm8192_fp32_integer_valued_bit_exact():
 def test_c3_tmm16384_quad_cas_full():
     """configs[2]: 16384^3, lock-free quadratic-probing store; every rid looked up in the GPU's table."""
     _tmm_full(16384, 16384, 16384, 128, "mod|xor", "quad_cas", "int5", "bf16", nsample=2, seed=5)
+
+
+def test_c3_tmm16384_cuckoo_full():
+    """configs[2] ablation extended to the paper's cuckoo table (N1)."""
+    _tmm_full(16384, 16384, 16384, 128, "mod|xor", "cuckoo", "int5", "bf16", nsample=2, seed=19)
 
 
 def test_c3_tmm16384_r32_array_full():

@@ -8,7 +8,7 @@ import torch
 import oracle
 from lpsynth import gen
 from paper_conf_iiswc_yudhakzs20_b200 import lp
-from tests.gpu_util import dev_to_host, host_to_dev
+from tests.gpu_util import check_store_table, dev_to_host, host_to_dev, oracle_validate
 
 pytestmark = pytest.mark.gpu
 
@@ -32,6 +32,8 @@ def stencil_cycle(H, W, kind, mask, mode, frac, seed=2, store="array"):
     assert np.array_equal(golden.view(np.uint32), oracle.stencil5(X).view(np.uint32))
     if store == "array":
         assert np.array_equal(ck_golden[:R * sel].reshape(R, sel), oracle.records(golden, 128, 128, h.mask))
+    else:
+        check_store_table(ck_golden, store, R, sel, oracle.records(golden, 128, 128, h.mask))
     h.validate(wl, out, ck, failed, d_n, ws)
     assert int(d_n.item()) == 0
     inj = torch.from_numpy(lp.choose_regions(R, frac, 1000 + seed)).cuda()
@@ -40,9 +42,8 @@ def stencil_cycle(H, W, kind, mask, mode, frac, seed=2, store="array"):
     torch.cuda.synchronize()
     nf = int(d_n.item())
     got = failed[:nf].cpu().numpy()
-    if store == "array":
-        exp = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * sel], 128, 128, h.mask)
-        assert np.array_equal(got, exp)
+    exp = oracle_validate(dev_to_host(out), dev_to_host(ck), store, 128, 128, h.mask)
+    assert np.array_equal(got, exp)
     assert set(got.tolist()) <= set(inj.cpu().numpy().tolist())
     if mode == "stale_region":
         assert nf == inj.numel()
@@ -66,13 +67,14 @@ def test_stencil_checksums_and_modes(mask, mode):
     stencil_cycle(512, 640, "uniform", mask, mode, 0.2)
 
 
-def test_stencil_quad_store():
-    stencil_cycle(512, 512, "uniform", "mod|xor", "stale_words", 0.25, store="quad_cas")
+@pytest.mark.parametrize("store", ["quad_cas", "cuckoo", "cuckoo_lock"])
+def test_stencil_hash_stores(store):
+    stencil_cycle(512, 512, "uniform", "mod|xor", "stale_words", 0.25, store=store)
 
 
 
 @pytest.mark.parametrize("frac", [0.01, 0.10, 0.50])
-@pytest.mark.parametrize("store", ["array", "quad_cas"])
+@pytest.mark.parametrize("store", ["array", "quad_cas", "cuckoo"])
 def test_same_grid_check_and_recover(frac, store):
     """Listing 7 (N2): one kernel validates every region and re-executes the failed ones in place;
     the result equals the golden output and the count equals the oracle's failed set."""
@@ -92,12 +94,7 @@ def test_same_grid_check_and_recover(frac, store):
     inj = torch.from_numpy(lp.choose_regions(R, frac, 1003)).cuda()
     h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=1003)
     torch.cuda.synchronize()
-    if store == "array":
-        exp = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * 2], 128, 128, 3)
-    else:
-        ckh = dev_to_host(ck)
-        cap = int(ckh[0])
-        exp = oracle.validate_quad(dev_to_host(out), ckh[16:16 + cap * 3], cap, int(ckh[1]), 128, 128, 3)
+    exp = oracle_validate(dev_to_host(out), dev_to_host(ck), store, 128, 128, 3)
     d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
     h.check_recover(wl, out, ck, d_rec)
     torch.cuda.synchronize()

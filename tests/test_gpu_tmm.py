@@ -12,7 +12,7 @@ import torch
 
 import oracle
 from paper_conf_iiswc_yudhakzs20_b200 import lp
-from tests.gpu_util import dev_to_host, host_to_dev, make_inputs, stale_image
+from tests.gpu_util import check_store_table, dev_to_host, host_to_dev, make_inputs, oracle_validate, stale_image
 
 pytestmark = pytest.mark.gpu
 
@@ -39,7 +39,7 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     if store == "array":
         assert np.array_equal(ck_golden[:R * sel].reshape(R, sel), recs)
     else:
-        check_hash_table(ck_golden, R, sel, recs)
+        check_store_table(ck_golden, store, R, sel, recs)
     # (5) values vs fp64 oracle
     if check_values:
         to32 = (lambda x: x) if out_dt == "f32" else oracle.bf16_bits_to_f32
@@ -71,12 +71,7 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     nf = int(d_n.item())
     got_failed = failed[:nf].cpu().numpy()
     bad_out, bad_ck = dev_to_host(out), dev_to_host(ck)
-    if store == "array":
-        exp_failed = oracle.validate_array(bad_out, bad_ck[:R * sel], RM, RN, h.mask)
-    else:
-        cap = int(bad_ck[0])
-        exp_failed = oracle.validate_quad(bad_out, bad_ck[16:16 + cap * (1 + sel)], cap, int(bad_ck[1]), RM, RN,
-                                          h.mask)
+    exp_failed = oracle_validate(bad_out, bad_ck, store, RM, RN, h.mask)
     assert np.array_equal(got_failed, exp_failed)
     injected = set(inj.cpu().numpy().tolist())
     assert set(got_failed.tolist()) <= injected
@@ -91,20 +86,8 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     if store == "array":
         assert np.array_equal(dev_to_host(ck)[:R * sel], ck_golden[:R * sel])
     else:
-        check_hash_table(dev_to_host(ck), R, sel, recs)
+        check_store_table(dev_to_host(ck), store, R, sel, recs)
     return h, nf
-
-
-def check_hash_table(ckh, R, sel, recs):
-    """Every rid is found exactly once by the oracle's lookup with its oracle record (SURVEY §4 layer 4)."""
-    cap, seed = int(ckh[0]), int(ckh[1])
-    table = ckh[16:16 + cap * (1 + sel)]
-    keys = table.reshape(cap, 1 + sel)[:, 0]
-    present = keys[keys != oracle.EMPTY_KEY]
-    assert len(present) == R and len(set(present.tolist())) == R
-    for rid in range(R):
-        assert list(oracle.quad_lookup(table, cap, sel, rid, seed)) == list(recs[rid]), rid
-    assert oracle.quad_lookup(table, cap, sel, R + 7, seed) is None
 
 
 @pytest.mark.parametrize("kind", ["uniform", "int5"])
@@ -130,7 +113,7 @@ def test_simt_larger_regions(RM):
     run_cycle(256, 384, 160, RM, RM, "f32", "f32", "uniform", "mod|xor", "simt", frac=0.3)
 
 
-@pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
+@pytest.mark.parametrize("store", ["quad_cas", "quad_lock", "cuckoo", "cuckoo_lock"])
 def test_simt_hash_stores(store):
     h, _ = run_cycle(256, 256, 64, 32, 32, "f32", "f32", "int5", "mod|xor", "simt", store=store, frac=0.1)
 
@@ -169,7 +152,7 @@ def test_tc_many_tiles_persistent(tc_pair):
               frac=0.05, check_values=True, tc_pair=tc_pair)
 
 
-@pytest.mark.parametrize("store", ["quad_cas", "quad_lock"])
+@pytest.mark.parametrize("store", ["quad_cas", "quad_lock", "cuckoo", "cuckoo_lock"])
 def test_tc_hash_stores(store):
     run_cycle(512, 512, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, frac=0.1)
 
@@ -245,3 +228,8 @@ def test_tf32x3_matches_simt_integer_valued():
 def test_int32_tmm_paper_shape(mask, mode):
     """Listing 2's int TMM with 32x32 thread-block regions (Table III: TMM = 32x32 blocks)."""
     run_cycle(256, 320, 192, 32, 32, "i32", "i32", "int17", mask, "simt", mode=mode, frac=0.1)
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "cuckoo", "cuckoo_lock"])
+def test_tf32x3_hash_stores(store):
+    run_cycle(512, 512, 128, 128, 128, "f32", "f32", "int5", "mod|xor", "tcgen05", store=store, frac=0.2)

@@ -349,3 +349,54 @@ def test_gemm_int32_operands_vs_numpy_int64():
     ref = A.astype(np.int64) @ B.astype(np.int64)
     got = oracle.gemm_block_f64(A, B, 0, 16, 32, 32)
     assert np.array_equal(got.astype(np.int64), ref[:, 16:48])
+
+
+
+# --------------------------------------------------------------------------- cuckoo hashing (L269-270)
+def test_cuckoo_hashes_re_derived():
+    def fmix(h):
+        h ^= h >> 16
+        h = (h * 0x85EBCA6B) & 0xFFFFFFFF
+        h ^= h >> 13
+        h = (h * 0xC2B2AE35) & 0xFFFFFFFF
+        h ^= h >> 16
+        return h
+    seed, cap = 0x9747B28C, 1009
+    for key in [0, 7, 123456]:
+        assert oracle.cuckoo_hash(0, key, seed, cap) == fmix(key ^ seed) % cap
+        assert oracle.cuckoo_hash(1, key, seed, cap) == fmix(key ^ ((seed * 0x9E3779B9 + 0x7F4A7C15) & 0xFFFFFFFF)) % cap
+
+
+def test_cuckoo_eviction_moves_occupant_to_other_table():
+    # Fig. 4 step (1)-(2): X hashes onto C's T1 slot -> X takes it, C moves to T2[H2(C)]
+    cap, seed = 101, 5
+    tab = np.full(2 * cap * 4, 0xFFFFFFFF, dtype=np.uint32)
+    c = 3
+    x = next(k for k in range(4, 100000) if oracle.cuckoo_hash(0, k, seed, cap) == oracle.cuckoo_hash(0, c, seed, cap))
+    assert oracle.cuckoo_insert(tab, cap, 1, c, seed, [111]) == 1
+    assert oracle.cuckoo_insert(tab, cap, 1, x, seed, [222]) == 2
+    t1 = tab.reshape(2, cap, 4)
+    assert t1[0, oracle.cuckoo_hash(0, x, seed, cap), 0] == x
+    assert t1[1, oracle.cuckoo_hash(1, c, seed, cap), 0] == c
+    assert list(oracle.cuckoo_lookup(tab, cap, 1, c, seed)) == [111]
+    assert list(oracle.cuckoo_lookup(tab, cap, 1, x, seed)) == [222]
+
+
+def test_cuckoo_roundtrip_at_load_half():
+    R, sel, seed = 1000, 2, 9
+    cap = 1009  # per table -> total load 1000 / 2018 < 50% (L270)
+    tab = np.full(2 * cap * 4, 0xFFFFFFFF, dtype=np.uint32)
+    rng = random.Random(1)
+    recs = {k: [rng.getrandbits(32), rng.getrandbits(32)] for k in range(R)}
+    evictions = 0
+    for k in range(R):
+        n = oracle.cuckoo_insert(tab, cap, sel, k, seed, recs[k])
+        assert n >= 1
+        evictions += n - 1
+    keys = tab.reshape(2 * cap, 4)[:, 0]
+    present = keys[keys != 0xFFFFFFFF]
+    assert len(present) == R and len(set(present.tolist())) == R
+    for k in range(R):
+        assert list(oracle.cuckoo_lookup(tab, cap, sel, k, seed)) == recs[k]
+    assert oracle.cuckoo_lookup(tab, cap, sel, R + 3, seed) is None
+    assert evictions > 0
