@@ -103,6 +103,9 @@ def parse():
     ap.add_argument("--overhead-reps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
+    ap.add_argument("--store", default=None, help="override the workload's checksum store (design-space runs)")
+    ap.add_argument("--cksum", default=None, help="override the workload's checksum set")
+    ap.add_argument("--no-shuffle", action="store_true", help="SIMT body: sequential reduction ablation (L343)")
     return ap.parse_args()
 
 
@@ -206,7 +209,11 @@ def run_ours(args):
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
-    W = WORKLOADS[args.workload]
+    W = dict(WORKLOADS[args.workload])
+    if args.store:
+        W["store"] = args.store
+    if args.cksum:
+        W["cksum"] = args.cksum
     RM = RN = W["region"]
     if W["kind"] == "tmm":
         gM = W["M"] * (world if W["weak"] else 1)
@@ -231,7 +238,8 @@ def run_ours(args):
         b = None
         wl = lp.Workload.stencil(a)
         body_flops = 0.0
-    h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"))
+    h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
+              shuffle=not args.no_shuffle)
     h0 = lp.LP(RM, RN, cksum=0, device=local, body=W.get("body", "auto"))   # unprotected twin (overhead denominator)
     out, ck, failed, d_n, ws = h.alloc(wl)
     out_twin = torch.empty_like(out)
@@ -476,6 +484,7 @@ def run_ours(args):
             "data": "synthetic (counter-based splitmix64 inputs generated in HBM; stale pre-image of out)",
             "config": {"workload": args.workload, "M_global": gM, "N": N, "K": K, "region": [RM, RN],
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
+                       "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write) before every recovery phase and every isolated kernel rep"},
             "lp_overhead_pct": round(overhead_pairs, 3),

@@ -122,7 +122,9 @@ typedef struct {
 
 /* lp_config_t.flags */
 typedef enum {
-  LP_FLAG_TC_1CTA = 1u /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
+  LP_FLAG_TC_1CTA = 1u,    /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
+  LP_FLAG_NO_SHUFFLE = 2u  /* SIMT body, MOD|XOR: sequential shared-memory reduction instead of warp reduction
+                              (the paper's "without parallel reduction" ablation, L343, Table IV) */
 } lp_config_flags;
 
 typedef struct {

@@ -220,6 +220,13 @@ uint32_t lpo_cuckoo_insert(uint32_t* tab, uint32_t cap, int selem, uint32_t key,
                            int max_evict) {
   uint32_t e[4] = {key, 0, 0, 0};
   for (int s = 0; s < selem; ++s) e[1 + s] = rec[s];
+  for (int t2 = 0; t2 < 2; ++t2) { /* an existing key is updated in place (re-insertion on recovery) */
+    uint32_t* slot = tab + 4 * ((uint64_t)t2 * cap + lpo_cuckoo_hash(t2, key, seed, cap));
+    if (slot[0] == key) {
+      memcpy(slot, e, 16);
+      return 1;
+    }
+  }
   int t = 0;
   for (int i = 0; i < max_evict; ++i) {
     uint32_t* slot = tab + 4 * ((uint64_t)t * cap + lpo_cuckoo_hash(t, e[0], seed, cap));

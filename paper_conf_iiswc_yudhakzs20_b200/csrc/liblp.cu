@@ -235,6 +235,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.d_n = d_n;
   a.list_is_tiles = 0;
   a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
+  a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
   a.sm_count = h->sm_count;
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
@@ -292,7 +293,10 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
     return fail(LP_ERR_UNSUPPORTED, "hash stores (the ablation) are built for MOD and MOD|XOR records");
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
-  if (cfg->flags & ~(uint32_t)LP_FLAG_TC_1CTA) return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
+  if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE))
+    return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
+  if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body != LP_BODY_SIMT || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
+    return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT body with MOD|XOR records");
   if ((int64_t)cfg->region_m * cfg->region_n * 4 > (16ll << 20))
     return fail(LP_ERR_UNSUPPORTED, "regions larger than 16 MiB are not supported");
   lp_ctx* h = new lp_ctx();

@@ -265,6 +265,19 @@ __device__ __forceinline__ uint32_t cuckoo_insert(uint32_t* ckbuf, uint32_t rid,
   uint4* tab = reinterpret_cast<uint4*>(ckbuf + sizeof(HashHeader) / 4);
   const uint32_t cap = hdr->cap, seed = hdr->seed;
   uint4 e = cuckoo_entry<MASK>(rid, w);
+  // Re-insertion (recovery): if the key already lives in one of its two slots, replace that
+  // entry in place -- inserting at T1 again could leave a stale duplicate in T2 that a later
+  // eviction chain would write back over the fresh record.
+  for (int t = 0; t < 2; ++t) {
+    uint4* slot = tab + (uint64_t)t * cap + cuckoo_h(t, rid, seed, cap);
+    if (slot->x == rid) {
+      const uint4 old = atom_exch_128(slot, e);
+      if (old.x == rid) return 1;
+      e = old;  // raced with a concurrent move: carry what we displaced
+      if (e.x == kEmptyKey) return 1;
+      break;
+    }
+  }
   int t = 0;
   for (int i = 0; i < kCuckooMaxEvict; ++i) {
     const uint4 old = atom_exch_128(tab + (uint64_t)t * cap + cuckoo_h(t, e.x, seed, cap), e);

@@ -64,6 +64,7 @@ struct TmmArgs {
   const int64_t* d_n;
   int list_is_tiles;    // list holds 128x128 tile ids (de-duplicated recovery of 32x32 regions)
   int force_1cta;       // tcgen05: use the 1-CTA 128x256 kernel even where the CTA-pair kernel applies
+  int no_shuffle;       // SIMT: sequential shared-memory reduction (the paper's "no shuffle" ablation)
   int sm_count;
 };
 bool tmm_simt_supported(int RM, int RN, int in_bf16, int out_bf16);

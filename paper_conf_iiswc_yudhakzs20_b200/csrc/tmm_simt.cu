@@ -70,7 +70,10 @@ __device__ __forceinline__ uint32_t word_of<float>(float v) { return __float_as_
 template <>
 __device__ __forceinline__ uint32_t word_of<int32_t>(int32_t v) { return (uint32_t)v; }
 
-template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE>
+// SEQ = the paper's "no shuffle" ablation (L343, Table IV "+no"): partials go to
+// shared memory and ONE thread folds all 256 of them sequentially, O(N) instead of
+// the O(log N) warp reduction (L220).
+template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE, bool SEQ = false>
 __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
                                                             const TIn* __restrict__ B, int64_t ldb,
                                                             TOut* __restrict__ C, int64_t ldc, int64_t K,
@@ -90,6 +93,7 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
   __shared__ __align__(16) TA As[2][kBK][BM + 4];
   __shared__ __align__(16) TA Bs[2][kBK][BN + 4];
   __shared__ CkRecord warp_rec[kThreads / 32];
+  __shared__ uint32_t seq_part[SEQ ? 4 : 1][SEQ ? kThreads : 1];
 
   const int tid = threadIdx.x;
   const int tx = tid % TX, ty = tid / TX;
@@ -182,7 +186,25 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
         }
       }
     }
-    if constexpr (MASK != 0) {
+    if constexpr (MASK != 0 && SEQ) {
+      seq_part[0][tid] = part.mod;
+      seq_part[1][tid] = part.xr;
+      seq_part[2][tid] = part.s;
+      seq_part[3][tid] = (uint32_t)(part.w % kAdlerBase);
+      __syncthreads();
+      if (tid == 0) {
+        CkRecord r{0u, 0u, 0u, 0u};
+        for (int i = 0; i < kThreads; ++i) {  // sequential, as on the CPU (L81, L220)
+          r.mod += seq_part[0][i];
+          r.xr ^= seq_part[1][i];
+          r.s += seq_part[2][i];
+          r.wmod = (r.wmod + seq_part[3][i]) % kAdlerBase;
+        }
+        uint32_t words[3];
+        record_words<MASK>(r, (uint64_t)BM * BN * ES, words);
+        store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+      }
+    } else if constexpr (MASK != 0) {
       const CkRecord wr = warp_reduce<MASK>(part);
       if ((tid & 31) == 0) warp_rec[tid >> 5] = wr;
       __syncthreads();
@@ -208,6 +230,25 @@ cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
   const TIn* B = (const TIn*)a.B;
   TOut* C = (TOut*)a.C;
   const int sk = a.mask ? a.hash.store : 0;
+  if (a.no_shuffle) {
+    if (a.mask != 3) return cudaErrorInvalidValue;  // the ablation is built for MOD|XOR (Table IV)
+    switch (sk) {
+#define LP_QCASE(S)                                                                                            \
+  case S:                                                                                                      \
+    tmm_simt_kernel<TIn, TOut, BM, BN, UM, UN, 3, S, true><<<(unsigned)grid, kThreads, 0, st>>>(               \
+        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.rid_offset, a.list, a.d_n);                           \
+    break;
+      LP_QCASE(0)
+      LP_QCASE(1)
+      LP_QCASE(2)
+      LP_QCASE(3)
+      LP_QCASE(4)
+#undef LP_QCASE
+      default:
+        return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+  }
   switch (a.mask * 5 + sk) {
 #define LP_SCASE(M, S)                                                                                         \
   case M * 5 + S:                                                                                              \

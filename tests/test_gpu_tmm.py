@@ -18,8 +18,8 @@ pytestmark = pytest.mark.gpu
 
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
-              store="array", check_values=True, recover_ws=True, tc_pair=True):
-    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair)
+              store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True):
+    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -157,6 +157,13 @@ def test_tc_hash_stores(store):
     run_cycle(512, 512, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, frac=0.1)
 
 
+@pytest.mark.parametrize("store", ["quad_cas", "cuckoo"])
+@pytest.mark.parametrize("mode", ["stale_record", "stale_region"])
+def test_hash_store_recovery_modes(store, mode):
+    """Recovery re-inserts records for keys that already exist (sentinel or intact records)."""
+    run_cycle(512, 512, 128, 32, 32, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, mode=mode, frac=0.3)
+
+
 def test_tc_unprotected_twin_same_bits():
     """cksum=0 builds the same body without the epilogue checksum: identical output bits."""
     import numpy as np
@@ -233,3 +240,10 @@ def test_int32_tmm_paper_shape(mask, mode):
 @pytest.mark.parametrize("store", ["quad_cas", "cuckoo", "cuckoo_lock"])
 def test_tf32x3_hash_stores(store):
     run_cycle(512, 512, 128, 128, 128, "f32", "f32", "int5", "mod|xor", "tcgen05", store=store, frac=0.2)
+
+
+
+@pytest.mark.parametrize("store", ["array", "quad_cas", "cuckoo"])
+def test_simt_no_shuffle_ablation(store):
+    """The paper's "without parallel reduction" variant (L343): same records, sequential fold."""
+    run_cycle(256, 256, 128, 32, 32, "i32", "i32", "int17", "mod|xor", "simt", store=store, frac=0.1, shuffle=False)

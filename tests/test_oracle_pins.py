@@ -400,3 +400,17 @@ def test_cuckoo_roundtrip_at_load_half():
         assert list(oracle.cuckoo_lookup(tab, cap, sel, k, seed)) == recs[k]
     assert oracle.cuckoo_lookup(tab, cap, sel, R + 3, seed) is None
     assert evictions > 0
+
+
+
+def test_cuckoo_reinsert_updates_in_place():
+    cap, seed = 53, 2
+    tab = np.full(2 * cap * 4, 0xFFFFFFFF, dtype=np.uint32)
+    for k in range(40):
+        oracle.cuckoo_insert(tab, cap, 2, k, seed, [k, k + 1])
+    for k in range(40):                       # recovery re-inserts every key with a new record
+        oracle.cuckoo_insert(tab, cap, 2, k, seed, [7 * k, 9])
+    keys = tab.reshape(2 * cap, 4)[:, 0]
+    assert np.sum(keys != 0xFFFFFFFF) == 40   # no duplicates
+    for k in range(40):
+        assert list(oracle.cuckoo_lookup(tab, cap, 2, k, seed)) == [7 * k, 9]

@@ -1,0 +1,24 @@
+#!/bin/bash
+# The paper's design space (Fig. 5 / Tables III-IV / V) on its own TMM (int32 4096^2, 32x32 thread-block
+# regions, MOD+XOR), B200: store x lock x reduction.  -> gpurun_out/design/*.json
+mkdir -p gpurun_out/design
+for st in array quad_cas quad_lock cuckoo cuckoo_lock; do
+  for sh in "" "--no-shuffle"; do
+    tag=${st}${sh:+_noshfl}
+    timeout 900 python bench.py --workload tmm4096_i32_paper --store $st $sh --steps 3 --warmup 3 --overhead-reps 10 \
+      --no-cpu-baseline > gpurun_out/design/$tag.json 2> gpurun_out/design/$tag.err || tail -2 gpurun_out/design/$tag.err
+  done
+done
+python - <<'PY'
+import glob, json, os
+print("| store | reduction | t_prot ms | t_unprot ms | LP overhead | slowdown (x) | hash collisions |")
+print("|---|---|---|---|---|---|---|")
+for f in sorted(glob.glob("gpurun_out/design/*.json")):
+    try:
+        d = json.loads(open(f).read().strip().splitlines()[-1])
+    except Exception:
+        continue
+    c = d["config"]
+    print(f"| {c['store']} | {c['reduction']} | {d['t_protected_ms']:.3f} | {d['t_unprotected_ms']:.3f} | "
+          f"{d['lp_overhead_pct']:+.2f}% | {d['t_protected_ms'] / d['t_unprotected_ms']:.2f} | {d.get('hash_collisions')} |")
+PY
