@@ -102,8 +102,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
   uint64_t* cv_empty = cv_full + kFCvStages;
   uint64_t* tfull = cv_empty + kFCvStages;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_holder = (uint32_t*)(tempty + 2);
-  CkRecord* srec = (CkRecord*)(tmem_holder + 4);
+  CkRecord* srec = (CkRecord*)(tempty + 2);                       // [2 acc][2 regions][4 warps] = 256 B
+  uint32_t* tmem_holder = (uint32_t*)((uint8_t*)(tempty + 2) + 256);  // own 128-B line, written by tcgen05.alloc
   auto raw = [&](int s) { return smem + s * kFRawBytes; };
   auto cvs = [&](int s) { return cv_base + s * kFCvBytes; };
 

@@ -1,0 +1,60 @@
+"""Small runs of every kernel family for compute-sanitizer (memcheck / racecheck / synccheck)."""
+import sys
+
+import torch
+
+sys.path.insert(0, ".")
+import lpsynth  # noqa: E402
+from paper_conf_iiswc_yudhakzs20_b200 import lp  # noqa: E402
+
+
+def cycle(h, wl, out, ck, failed, d_n, ws, stale, frac=0.2):
+    out.copy_(stale)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    R = h.num_regions(wl)
+    inj = torch.from_numpy(lp.choose_regions(R, frac, 5)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=5)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    h.recover(wl, out, ck, failed, d_n, ws)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+
+
+def tmm(M, N, K, reg, in_dt, out_dt, body, store="array", shuffle=True):
+    tdt = {"bf16": torch.bfloat16, "f32": torch.float32, "i32": torch.int32}[in_dt]
+    a = torch.empty((M, K), dtype=tdt, device="cuda")
+    b = torch.empty((K, N), dtype=tdt, device="cuda")
+    kind = "int5"
+    lpsynth.device_fill(a, 1, kind, in_dt)
+    lpsynth.device_fill(b, 2, kind, in_dt)
+    h = lp.LP(reg, reg, cksum="mod|xor", store=store, body=body, shuffle=shuffle)
+    wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = torch.zeros_like(out)
+    cycle(h, wl, out, ck, failed, d_n, ws, stale)
+    print("ok", M, N, K, reg, in_dt, out_dt, body, store, shuffle, flush=True)
+
+
+def stencil(store="array"):
+    x = torch.empty((512, 384), dtype=torch.float32, device="cuda")
+    lpsynth.device_fill(x, 1, "uniform", "f32")
+    h = lp.LP(128, 128, cksum="mod|xor", store=store)
+    wl = lp.Workload.stencil(x)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = torch.zeros_like(out)
+    cycle(h, wl, out, ck, failed, d_n, ws, stale)
+    d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+    h.check_recover(wl, out, ck, d_rec)
+    torch.cuda.synchronize()
+    print("ok stencil", store, flush=True)
+
+
+tmm(256, 256, 128, 32, "f32", "f32", "simt")
+tmm(256, 256, 128, 32, "i32", "i32", "simt", store="cuckoo", shuffle=False)
+tmm(256, 512, 128, 128, "bf16", "bf16", "tcgen05")
+tmm(256, 512, 128, 32, "bf16", "f32", "tcgen05", store="quad_cas")
+tmm(256, 512, 64, 128, "f32", "f32", "tcgen05", store="cuckoo")
+stencil()
+stencil("quad_cas")
