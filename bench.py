@@ -106,6 +106,8 @@ def parse():
     ap.add_argument("--store", default=None, help="override the workload's checksum store (design-space runs)")
     ap.add_argument("--cksum", default=None, help="override the workload's checksum set")
     ap.add_argument("--no-shuffle", action="store_true", help="SIMT body: sequential reduction ablation (L343)")
+    ap.add_argument("--no-graph", dest="graph", action="store_false",
+                    help="launch the step eagerly instead of replaying captured CUDA graphs")
     return ap.parse_args()
 
 
@@ -274,24 +276,52 @@ def run_ours(args):
     def ev():
         return torch.cuda.Event(enable_timing=True)
 
-    def step(timed_segments):
-        """One pass of the hot path; returns (t_body, t_inject, t_valrec, n_failed) events-based (ms)."""
-        e = [ev() for _ in range(6)]
-        e[0].record(st)
+    # The step's segments; each is captured once into a CUDA graph after the eager warm-up (all of
+    # liblp's launches are stream-ordered with device-side counts, so a replay re-does the same work on
+    # whatever the buffers hold).  The count all-reduce stays eager between the two recovery graphs.
+    def seg_body():
         h.cksum_init(wl, ck)
         h.run_protected(wl, out, ck)
-        e[1].record(st)
+
+    def seg_inject():
         h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=1000 + rank)
-        e[2].record(st)
-        flush_buf.zero_()             # cold L2 for the recovery phase (not timed)
-        e[3].record(st)
+
+    def seg_validate():
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[0:1].copy_(d_n)
         counts[1:2].copy_(d_n)
-        shard.allreduce_counts(counts[0:2])
+
+    def seg_recover():
         h.recover(wl, out, ck, failed, d_n, ws)
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[2:3].copy_(d_n)
+
+    runners = {"body": seg_body, "inject": seg_inject, "validate": seg_validate, "recover": seg_recover}
+
+    def capture_graphs():
+        graphs = {}
+        for name, fn in list(runners.items()):
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                fn()
+            graphs[name] = g
+        for name, g in graphs.items():
+            runners[name] = g.replay
+        torch.cuda.synchronize()
+
+    def step(timed_segments):
+        """One pass of the hot path; returns the 5 segment events (body, inject, flush, recovery phase)."""
+        e = [ev() for _ in range(6)]
+        e[0].record(st)
+        runners["body"]()
+        e[1].record(st)
+        runners["inject"]()
+        e[2].record(st)
+        flush_buf.zero_()             # cold L2 for the recovery phase (not timed)
+        e[3].record(st)
+        runners["validate"]()
+        shard.allreduce_counts(counts[0:2])
+        runners["recover"]()
         shard.allreduce_counts(counts[2:3])
         e[4].record(st)
         return e
@@ -305,6 +335,11 @@ def run_ours(args):
     clk.wait_first()
     for _ in range(max(args.warmup, 3)):
         e = step(True)
+        torch.cuda.synchronize()
+        finish(e)
+    if args.graph:
+        capture_graphs()
+        e = step(True)                # one untimed replay of the captured graphs
         torch.cuda.synchronize()
         finish(e)
     # ---- timed K steps (barrier + sync on both sides; per-segment device events)
@@ -391,13 +426,9 @@ def run_ours(args):
         e0.record(st)
         out.copy_(out_host, non_blocking=True)
         ck.copy_(ck_host, non_blocking=True)
-        h.validate(wl, out, ck, failed, d_n, ws)
-        counts[0:1].copy_(d_n)
-        counts[1:2].copy_(d_n)
+        runners["validate"]()
         shard.allreduce_counts(counts[0:2])
-        h.recover(wl, out, ck, failed, d_n, ws)
-        h.validate(wl, out, ck, failed, d_n, ws)
-        counts[2:3].copy_(d_n)
+        runners["recover"]()
         shard.allreduce_counts(counts[2:3])
         summary_host.copy_(counts, non_blocking=True)
         e1.record(st)
@@ -486,7 +517,8 @@ def run_ours(args):
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
-                       "l2": "flushed (2x L2 write) before every recovery phase and every isolated kernel rep"},
+                       "l2": "flushed (2x L2 write) before every recovery phase and every isolated kernel rep",
+                       "launch": "CUDA graph replay per step segment" if args.graph else "eager"},
             "lp_overhead_pct": round(overhead_pairs, 3),
             "lp_overhead_pct_of_medians": round(report.overhead_pct(t_prot, t_unprot), 3),
             "lp_overhead_method": f"median over {len(pair_ratios)} adjacent (protected, unprotected) run pairs of "
