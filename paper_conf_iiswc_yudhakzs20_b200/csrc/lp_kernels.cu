@@ -9,6 +9,7 @@
 // recovery re-executes only those.
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "lp_device.cuh"
 #include "lp_internal.h"
@@ -17,55 +18,85 @@ namespace lp {
 namespace {
 
 constexpr int kValThreads = 256;
+constexpr int kValWarps = kValThreads / 32;
 constexpr int64_t kMaxValCtas = 148 * 16 * 4;
 constexpr int kValUnroll = 8;
 
-// W warps per region (W = 1, 2, 4, 8; chosen so each warp streams ~2-8 batches of
-// 4 KiB), 8/W regions in flight per CTA, each CTA a contiguous range of regions so
-// it can count its failures for the ordered compaction (no separate count pass).
-// A region's W warp partials are combined through double-buffered shared slots
-// behind a named barrier of the W warps (Listing 3's block combine, per region).
+// Segmented reduction of the per-lane partials over aligned groups of 2^lg_log2
+// lanes (one group = one region).  A whole-warp group uses one redux.sync per
+// checksum (the B200 form of Listing 4's shfl_down ladder, L244-258); narrower
+// groups use an xor butterfly of log2(group) shuffles.  Adler's W is reduced
+// mod 65521 per lane first so the u32 sums cannot wrap (<= 32 * 65520).
+template <uint32_t MASK>
+__device__ __forceinline__ CkRecord segment_reduce(const CkPartial<MASK>& p, int lg_log2) {
+  if (lg_log2 == 5) return warp_reduce<MASK>(p);
+  CkRecord r{p.mod, p.xr, p.s, 0u};
+  if constexpr ((MASK & kAdler) != 0) r.wmod = (uint32_t)(p.w % kAdlerBase);
+  for (int o = (1 << lg_log2) >> 1; o > 0; o >>= 1) {
+    if constexpr ((MASK & kMod) != 0) r.mod += __shfl_xor_sync(0xFFFFFFFFu, r.mod, o);
+    if constexpr ((MASK & kXor) != 0) r.xr ^= __shfl_xor_sync(0xFFFFFFFFu, r.xr, o);
+    if constexpr ((MASK & kAdler) != 0) {
+      r.s += __shfl_xor_sync(0xFFFFFFFFu, r.s, o);
+      r.wmod += __shfl_xor_sync(0xFFFFFFFFu, r.wmod, o);
+    }
+  }
+  return r;
+}
+
+// Validate (a8): a warp task is a strip of G = 2^g_log2 horizontally adjacent
+// regions (consecutive rids), LG = 32 / G lanes per region.  Lane li of a group
+// reads the 16-byte chunks li, li + LG, ... of its region in row-major order, so
+// the group's lanes cover LG / cpr whole region rows per load instruction (or
+// 1 / (cpr / LG) of a row) and the warp touches G adjacent row segments.  Eight
+// 16-byte non-allocating loads are in flight per lane.  G is chosen on the host
+// (plan_validate) so that enough warps exist to keep ~16 MiB of reads in flight
+// (1 region per warp for 128x128) while strips of small regions still give
+// 256-512 B contiguous segments.  Each CTA owns a contiguous range of regions and
+// writes its failure count for the ordered compaction.
 // MODE 0 = compare with array table, 1 = compare with a quad hash table (lookup
 // by global rid), 2 = write records (no compare), 3 = compare with a cuckoo table.
-template <uint32_t MASK, int MODE, int W>
-__global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
+template <uint32_t MASK, int MODE>
+__global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
                                                                 int64_t Q, int64_t R, int RM, int row_bytes,
-                                                                int cpr_log2, const uint32_t* __restrict__ ck,
+                                                                int cpr_log2, int g_log2,
+                                                                const uint32_t* __restrict__ ck,
                                                                 int64_t rid_offset, uint8_t* __restrict__ flags,
                                                                 uint32_t* __restrict__ records, int64_t rpc,
                                                                 uint32_t* __restrict__ cta_counts) {
   constexpr int S = selem_of(MASK);
-  constexpr int GROUPS = (kValThreads / 32) / W;
-  __shared__ CkRecord slots[2][GROUPS][W];
   __shared__ uint32_t s_fail;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const int g = warp / W, wi = warp - g * W;
-  const int cpr_mask = (1 << cpr_log2) - 1;
-  const int chunks = RM << cpr_log2;
-  const int my_chunks = chunks / W, c_begin = wi * my_chunks;
+  const int lg_log2 = 5 - g_log2;                       // lanes per region (log2)
+  const int G = 1 << g_log2;
+  const int gi = lane >> lg_log2, li = lane & ((1 << lg_log2) - 1);
+  const int chunks = RM << cpr_log2;                    // 16-byte chunks per region
+  const int cmask = (1 << cpr_log2) - 1;
   const uint64_t nbytes = (uint64_t)RM * (uint64_t)row_bytes;
+  // let the compaction grid (programmatic dependent launch) be scheduled early; it
+  // waits in griddepcontrol.wait until this whole grid has completed and flushed
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   if (threadIdx.x == 0) s_fail = 0;
   __syncthreads();
   const int64_t r0 = (int64_t)blockIdx.x * rpc;
   const int64_t r1 = r0 + rpc < R ? r0 + rpc : R;
-  int parity = 0;
-  for (int64_t r = r0 + g; r < r1; r += GROUPS) {
+  for (int64_t t0 = r0 + (int64_t)warp * G; t0 < r1; t0 += (int64_t)kValWarps * G) {
+    const int64_t r = t0 + gi;
+    const bool live = r < r1;
     const int64_t p = r / Q, q = r - p * Q;
     const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
     CkPartial<MASK> part;
-    for (int c0 = c_begin; c0 < c_begin + my_chunks; c0 += 32 * kValUnroll) {
+    for (int c0 = li; c0 < chunks; c0 += kValUnroll << lg_log2) {
       uint4 v[kValUnroll];
 #pragma unroll
       for (int u = 0; u < kValUnroll; ++u) {
-        const int c = c0 + u * 32 + lane;
-        if (c < c_begin + my_chunks)
-          v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cpr_mask) << 4));
+        const int c = c0 + (u << lg_log2);
+        if (live && c < chunks) v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cmask) << 4));
       }
 #pragma unroll
       for (int u = 0; u < kValUnroll; ++u) {
-        const int c = c0 + u * 32 + lane;
-        if (c < c_begin + my_chunks) {
-          const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cpr_mask) << 4) + 1);
+        const int c = c0 + (u << lg_log2);
+        if (live && c < chunks) {
+          const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cmask) << 4) + 1);
           part.add(v[u].x, pos);
           part.add(v[u].y, pos + 4);
           part.add(v[u].z, pos + 8);
@@ -73,20 +104,8 @@ __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __
         }
       }
     }
-    CkRecord rec = warp_reduce<MASK>(part);
-    bool finisher = true;
-    if constexpr (W > 1) {
-      if (lane == 0) slots[parity][g][wi] = rec;
-      asm volatile("bar.sync %0, %1;" ::"r"(1 + g), "r"(W * 32) : "memory");
-      finisher = (wi == 0);
-      if (finisher) {
-        rec = slots[parity][g][0];
-#pragma unroll
-        for (int w = 1; w < W; ++w) rec = combine(rec, slots[parity][g][w]);
-      }
-      parity ^= 1;
-    }
-    if (finisher && lane == 0) {
+    const CkRecord rec = segment_reduce<MASK>(part, lg_log2);
+    if (live && li == 0) {
       uint32_t w[3];
       record_words<MASK>(rec, nbytes, w);
       if constexpr (MODE == 2) {
@@ -117,48 +136,24 @@ __global__ void __launch_bounds__(kValThreads) validate_kernel(const uint8_t* __
 
 struct ValLaunch {
   dim3 grid;
-  int W;
   int64_t rpc;
+  int g_log2;
 };
-
-template <uint32_t MASK, int W>
-cudaError_t validate_dispatch_w(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out, int64_t ldc_bytes,
-                                int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2, const uint32_t* ck,
-                                int64_t rid_offset, uint8_t* flags, uint32_t* records, uint32_t* counts) {
-  if (mode == 0)
-    validate_kernel<MASK, 0, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                                rid_offset, flags, records, L.rpc, counts);
-  else if (mode == 1)
-    validate_kernel<MASK, 1, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                                rid_offset, flags, records, L.rpc, counts);
-  else if (mode == 3)
-    validate_kernel<MASK, 3, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                                rid_offset, flags, records, L.rpc, counts);
-  else
-    validate_kernel<MASK, 2, W><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck,
-                                                                rid_offset, flags, records, L.rpc, counts);
-  return cudaGetLastError();
-}
 
 template <uint32_t MASK>
 cudaError_t validate_dispatch_mode(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
                                    int64_t ldc_bytes, int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2,
                                    const uint32_t* ck, int64_t rid_offset, uint8_t* flags, uint32_t* records,
                                    uint32_t* counts) {
-  switch (L.W) {
-    case 8:
-      return validate_dispatch_w<MASK, 8>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
-                                          flags, records, counts);
-    case 4:
-      return validate_dispatch_w<MASK, 4>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
-                                          flags, records, counts);
-    case 2:
-      return validate_dispatch_w<MASK, 2>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
-                                          flags, records, counts);
-    default:
-      return validate_dispatch_w<MASK, 1>(mode, L, st, out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2, ck, rid_offset,
-                                          flags, records, counts);
-  }
+#define LP_VLAUNCH(MD)                                                                                    \
+  validate_kernel<MASK, MD><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2,     \
+                                                            L.g_log2, ck, rid_offset, flags, records, L.rpc, counts)
+  if (mode == 0) LP_VLAUNCH(0);
+  else if (mode == 1) LP_VLAUNCH(1);
+  else if (mode == 3) LP_VLAUNCH(3);
+  else LP_VLAUNCH(2);
+#undef LP_VLAUNCH
+  return cudaGetLastError();
 }
 
 // ---------------------------------------------------------------------------
@@ -243,6 +238,8 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
   __shared__ int warp_s[kCompactThreads / 32];
   __shared__ long long red[2][kCompactThreads / 32];
   __shared__ long long s_base;
+  // launched as a programmatic dependent of the validate grid: wait for its counts/flags
+  asm volatile("griddepcontrol.wait;" ::: "memory");
   const int first = (int)blockIdx.x * per_block;
   long long mine = 0, all = 0;
   for (int b = threadIdx.x; b < nblocks; b += kCompactThreads) {
@@ -399,25 +396,32 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
   return e;
 }
 
+// Strip width: G regions per warp.  G = 32 / cpr makes one warp load instruction
+// cover one row of the whole strip (512 B contiguous); it is halved while that
+// would leave fewer than kValMinWarps warp tasks (too few bytes in flight: 128x128
+// bf16 regions at G = 2 leave 2048 warps / 8 MiB in flight and measure 28.7 us
+// for 128 MiB vs 22.5 us at G = 1).  LP_VALIDATE_G=<log2> overrides (A/B runs).
+constexpr int64_t kValMinWarps = 4096;
+
 static ValLaunch plan_validate(const RegionGeom& g, int sm_count) {
   ValLaunch L;
-  const int chunks = g.RM * ((g.RN * g.es) / 16);
-  const int64_t resident_warps = (int64_t)sm_count * 32;  // ~4 CTAs of 8 warps per SM
-  // enough warps per region that each warp streams only a few 4-KiB batches when regions are few
-  // Splitting a region over W > 1 warps was measured slower (validate of 128 MiB /
-  // 4096 regions: 45 us at W = 4 vs 25 us at W = 1): one warp streams one region.
-  int W = 1;
-  (void)resident_warps;
-  (void)chunks;
-  L.W = W;
-  const int groups = 8 / W;
+  const int cpr = (g.RN * g.es) / 16;
+  int gl = 0;
+  while ((2 << gl) * cpr <= 32) ++gl;                  // G * cpr <= 32
+  while (gl > 0 && (g.R >> gl) < kValMinWarps) --gl;
+  if (const char* e = getenv("LP_VALIDATE_G")) {
+    const int v = atoi(e);
+    if (v >= 0 && v <= 5) gl = v;
+  }
+  L.g_log2 = gl;
+  const int64_t unit = (int64_t)kValWarps << gl;
   int64_t max_ctas = (int64_t)sm_count * 16;
   if (max_ctas > kMaxValCtas) max_ctas = kMaxValCtas;  // per-CTA counts live in the caller's workspace
-  int64_t ctas = (g.R + groups - 1) / groups;
+  int64_t ctas = (g.R + unit - 1) / unit;
   if (ctas > max_ctas) ctas = max_ctas;
   if (ctas < 1) ctas = 1;
   int64_t rpc = (g.R + ctas - 1) / ctas;
-  rpc = (rpc + groups - 1) / groups * groups;
+  rpc = (rpc + unit - 1) / unit * unit;
   ctas = (g.R + rpc - 1) / rpc;
   L.rpc = rpc;
   L.grid = dim3((unsigned)(ctas < 1 ? 1 : ctas));
@@ -436,8 +440,8 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   const int cpr = row_bytes / 16;
   int cpr_log2 = 0;
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
-  const ValLaunch L = plan_validate(g, sm_count);
   const int mode = records ? 2 : (hi.store == 0 ? 0 : (hi.store <= 2 ? 1 : 3));
+  const ValLaunch L = plan_validate(g, sm_count);
   const uint8_t* o = (const uint8_t*)out;
   const int64_t ldcb = g.ldc * g.es;
   cudaError_t e;
@@ -462,9 +466,20 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   // ordered compaction: one pass, offsets from the validate kernel's per-CTA counts
   int sg, per;
   scatter_grid(L.grid.x, sg, per);
-  compact_scatter_kernel<<<sg, kCompactThreads, 0, st>>>(flags, g.R, counts, (int)L.grid.x, L.rpc, per, g.rid_offset,
-                                                         list, d_n);
-  return cudaGetLastError();
+  // programmatic dependent launch: the scatter grid's launch overlaps the validate grid
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)sg);
+  cfg.blockDim = dim3(kCompactThreads);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, compact_scatter_kernel, (const uint8_t*)flags, (int64_t)g.R,
+                            (const uint32_t*)counts, (int)L.grid.x, (int64_t)L.rpc, per, (int64_t)g.rid_offset,
+                            list, d_n);
 }
 
 size_t compact_scratch_bytes(int64_t R) {

@@ -1,0 +1,100 @@
+"""GPU parity of the validate kernel over every warp-task geometry.
+
+The validate kernel maps a strip of G = 32 / LR horizontally adjacent regions onto one warp
+(LR = min(32, 16-byte chunks per region row) lanes per region, xor-butterfly or redux.sync
+reduction, 2^k chunks per lane per row when a region row is wider than 512 B).  These cases
+cover LR = 1 .. 32, 1/2/4 chunks per lane per row, strips that wrap a region row
+(Q % G != 0), odd region heights and CTA ranges with a ragged tail, for every checksum
+set -- records (lp_region_checksums) and failed lists (lp_validate) against the oracle.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from paper_conf_iiswc_yudhakzs20_b200 import lp
+from tests.gpu_util import dev_to_host, host_to_dev, oracle_validate
+
+pytestmark = pytest.mark.gpu
+
+# (M, N, RM, RN, dtype): row bytes RN*es -> chunks per row 1 .. 128
+GEOMS = [
+    (24, 4 * 37, 3, 4, "f32"),        # LR=1, G=32, Q=37 (wraps)
+    (14, 8 * 40, 7, 8, "f32"),        # LR=2, G=16
+    (64, 16 * 24, 1, 16, "f32"),      # LR=4, single-row regions
+    (96, 32 * 21, 32, 32, "f32"),     # LR=8, G=4, Q=21
+    (130, 64 * 10, 13, 64, "f32"),    # LR=16, G=2, Q odd... 10 (even)
+    (256, 128 * 5, 128, 128, "f32"),  # LR=32, G=1
+    (64, 256 * 3, 16, 256, "f32"),    # 2 chunks per lane per row
+    (32, 512 * 2, 8, 512, "f32"),     # 4 chunks per lane per row
+    (64, 32 * 33, 32, 32, "bf16"),    # LR=4, G=8, Q=33
+    (384, 128 * 7, 128, 128, "bf16"),  # LR=16, G=2, Q=7 (wraps)
+    (40, 256 * 3, 5, 256, "bf16"),    # LR=32
+    (16, 1024 * 2, 4, 1024, "bf16"),  # 4 chunks per lane per row
+    (2048, 32 * 64, 32, 32, "bf16"),  # many regions: several CTAs, ragged last CTA
+    (300 * 7, 128 * 3, 300, 128, "bf16"),  # RM > 256: strip kernel only
+    (1536, 128 * 12, 128, 128, "f32"),     # 64-KiB TMA units, 144 units: one per CTA
+    (4096, 32 * 96, 32, 32, "f32"),        # G = 8 units (GC = 64), 1536 units over the SMs
+]
+
+
+def _random_out(rng, M, N, dt):
+    if dt == "f32":
+        return rng.integers(0, 2**32, size=(M, N), dtype=np.uint64).astype(np.uint32).view(np.float32)
+    return rng.integers(0, 2**16, size=(M, N), dtype=np.uint64).astype(np.uint16)
+
+
+@pytest.fixture(params=["tma", "strip"])
+def kernel_path(request, monkeypatch):
+    """validate runs the TMA-staged kernel where the geometry fits a TMA box, else the strip kernel;
+    LP_VALIDATE_STRIP=1 forces the strip kernel so both paths are checked on every geometry."""
+    if request.param == "strip":
+        monkeypatch.setenv("LP_VALIDATE_STRIP", "1")
+    else:
+        monkeypatch.delenv("LP_VALIDATE_STRIP", raising=False)
+    return request.param
+
+
+@pytest.mark.parametrize("geom", GEOMS, ids=[f"{g[0]}x{g[1]}_{g[2]}x{g[3]}_{g[4]}" for g in GEOMS])
+@pytest.mark.parametrize("mask", ["mod|xor", "mod|xor|adler", "adler"])
+def test_validate_geometries(geom, mask, kernel_path):
+    M, N, RM, RN, dt = geom
+    rng = np.random.default_rng(M * 7919 + N + RM)
+    out_h = _random_out(rng, M, N, dt)
+    h = lp.LP(RM, RN, cksum=mask)
+    wl = lp.Workload.tmm(None, None, out_dtype=dt, m=M, n=N, k=16)
+    out = host_to_dev(out_h, dt)
+    _, ck, failed, d_n, ws = h.alloc(wl)
+    R = h.num_regions(wl)
+    sel = oracle.selem(h.mask)
+    # records of the current contents == the oracle's (lp_region_checksums = validate MODE 2)
+    h.region_checksums(wl, out, ck)
+    torch.cuda.synchronize()
+    table = dev_to_host(ck)[:R * sel].reshape(R, sel)
+    assert np.array_equal(table, oracle.records(out_h, RM, RN, h.mask))
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+    # corrupt ~15% of the regions (one random word each, every second one also a stale record)
+    bad = rng.choice(R, max(1, R * 15 // 100), replace=False)
+    Q = N // RN
+    words = out_h.view(np.uint32) if dt == "f32" else out_h.view(np.uint16)
+    ck_h = dev_to_host(ck).copy()
+    for j, r in enumerate(sorted(bad.tolist())):
+        p, q = divmod(r, Q)
+        i = int(rng.integers(RM))
+        c = int(rng.integers(RN))
+        words[p * RM + i, q * RN + c] ^= 1 << int(rng.integers(16))
+        if j % 2:
+            ck_h[r * sel] ^= 0x10
+    out.copy_(host_to_dev(out_h, dt))
+    ck.copy_(torch.from_numpy(ck_h.view(np.int32)).cuda())
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    n = int(d_n.item())
+    got = failed[:n].cpu().numpy()
+    exp = oracle_validate(out_h, ck_h, "array", RM, RN, h.mask)
+    assert np.array_equal(got, exp)
+    assert set(exp.tolist()) == set(bad.tolist())   # a single bit flip always changes MOD, XOR and Adler
