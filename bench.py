@@ -106,6 +106,8 @@ def parse():
     ap.add_argument("--store", default=None, help="override the workload's checksum store (design-space runs)")
     ap.add_argument("--cksum", default=None, help="override the workload's checksum set")
     ap.add_argument("--no-shuffle", action="store_true", help="SIMT body: sequential reduction ablation (L343)")
+    ap.add_argument("--no-pairing", action="store_true",
+                    help="tcgen05 recovery: one 128x128 tile per failed tile (no same-row pairing) -- A/B switch")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch the step eagerly instead of replaying captured CUDA graphs")
     return ap.parse_args()
@@ -241,7 +243,7 @@ def run_ours(args):
         wl = lp.Workload.stencil(a)
         body_flops = 0.0
     h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
-              shuffle=not args.no_shuffle)
+              shuffle=not args.no_shuffle, pairing=not args.no_pairing)
     h0 = lp.LP(RM, RN, cksum=0, device=local, body=W.get("body", "auto"))   # unprotected twin (overhead denominator)
     out, ck, failed, d_n, ws = h.alloc(wl)
     out_twin = torch.empty_like(out)
@@ -523,6 +525,7 @@ def run_ours(args):
             "config": {"workload": args.workload, "M_global": gM, "N": N, "K": K, "region": [RM, RN],
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
+                       "recovery": "one 128x128 tile per failed tile" if args.no_pairing else "same-row failed tiles paired into 128x256 tasks (when > #SM)",
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write, then 2x L2 read of another buffer: clean lines) before every recovery phase and every isolated kernel rep",
                        "launch": "CUDA graph replay per step segment" if args.graph else "eager"},

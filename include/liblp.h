@@ -123,8 +123,10 @@ typedef struct {
 /* lp_config_t.flags */
 typedef enum {
   LP_FLAG_TC_1CTA = 1u,    /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
-  LP_FLAG_NO_SHUFFLE = 2u  /* SIMT body, MOD|XOR: sequential shared-memory reduction instead of warp reduction
+  LP_FLAG_NO_SHUFFLE = 2u, /* SIMT body, MOD|XOR: sequential shared-memory reduction instead of warp reduction
                               (the paper's "without parallel reduction" ablation, L343, Table IV) */
+  LP_FLAG_NO_PAIRING = 4u  /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
+                              failed tiles of the same row band into 128x256 tasks (A/B switch) */
 } lp_config_flags;
 
 typedef struct {
@@ -184,7 +186,10 @@ LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* o
  * `workspace` (optional, lp_workspace_bytes bytes, may be NULL) lets liblp
  * de-duplicate failed regions that share one tensor-core tile (32x32 regions:
  * 16 per 128x128 tile) so each tile is recomputed once; with NULL every listed
- * region recomputes its tile (same final state, more work). */
+ * region recomputes its tile (same final state, more work).  With a workspace and
+ * the bf16 tcgen05 body, failed 128x128 tiles of the same 128-row band are also
+ * paired into one 128x256 task (A row panel read once for both) when more tiles
+ * failed than there are SMs; results are bit-identical either way. */
 LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
                             const int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 

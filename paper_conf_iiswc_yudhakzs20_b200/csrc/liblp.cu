@@ -161,7 +161,7 @@ int64_t dedupe_tiles(const lp::RegionGeom& g, int E) { return (g.M % E || g.N % 
 int64_t dedupe_capacity(const lp::RegionGeom& g) { return dedupe_tiles(g, 128); }
 
 struct WsLayout {
-  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, total;
+  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, d_ntasks, total;
 };
 
 WsLayout ws_layout(const lp::RegionGeom& g) {
@@ -176,7 +176,9 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   w.tile_counts = w.tile_flags + al((size_t)T);
   w.tile_list = w.tile_counts + al(lp::compact_scratch_bytes(T));
   w.d_ntiles = w.tile_list + al((size_t)T * 8);
-  w.total = w.d_ntiles + 256;
+  w.tasks = w.d_ntiles + 256;                       // paired recovery tasks: int32[max(R, T)]
+  w.d_ntasks = w.tasks + al((size_t)(g.R > T ? g.R : T) * 4);
+  w.total = w.d_ntasks + 256;
   return w;
 }
 
@@ -234,6 +236,8 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   a.list = list;
   a.d_n = d_n;
   a.list_is_tiles = 0;
+  a.tasks = nullptr;
+  a.d_ntasks = nullptr;
   a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
   a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
   a.sm_count = h->sm_count;
@@ -261,6 +265,18 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
       a.list = (const int64_t*)(ws + w.tile_list);
       a.d_n = (const int64_t*)(ws + w.d_ntiles);
       a.list_is_tiles = 1;
+    }
+    if (list && workspace && tc_ok && (a.list_is_tiles || g.RM == 128) && !(h->cfg.flags & LP_FLAG_NO_PAIRING)) {
+      // pair failed 128x128 tiles of the same row band into 128x256 re-execution tasks
+      const WsLayout w = ws_layout(g);
+      uint8_t* ws = (uint8_t*)workspace;
+      const int64_t off = a.list_is_tiles ? 0 : g.rid_offset;
+      const int64_t div = a.list_is_tiles ? g.N / 128 : g.Q;
+      cudaError_t e0 = lp::launch_pair_tasks(a.list, a.d_n, off, div, h->sm_count, (int32_t*)(ws + w.tasks),
+                                             (int64_t*)(ws + w.d_ntasks), st);
+      if (e0 != cudaSuccess) return cuda_fail(e0, "recovery pairing");
+      a.tasks = (const int32_t*)(ws + w.tasks);
+      a.d_ntasks = (const int64_t*)(ws + w.d_ntasks);
     }
     const char* why = nullptr;
     cudaError_t e = tc_ok ? lp::launch_tmm_tc(a, st, &why) : lp::launch_tmm_tf32(a, st, &why);
@@ -293,7 +309,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
     return fail(LP_ERR_UNSUPPORTED, "hash stores (the ablation) are built for MOD and MOD|XOR records");
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
-  if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE))
+  if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body != LP_BODY_SIMT || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT body with MOD|XOR records");

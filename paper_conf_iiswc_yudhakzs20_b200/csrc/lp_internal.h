@@ -38,6 +38,10 @@ size_t compact_scratch_bytes(int64_t R);
 cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi, void* out, void* ck,
                           const void* stale, const int64_t* rids, int64_t n, uint32_t mode, uint64_t seed,
                           cudaStream_t st);
+// ascending list of 128x128 tiles/regions -> recovery tasks of 1-2 entries of the same row band
+// (row = (list[i] - off) / div); pairing only when *d_n > min_pair.  tasks[t] = (i << 1) | paired.
+cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
+                              int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
 // failed regions -> unique tile ids of an E x E tile grid (tile = (p*RM/E)*(N/E) + q*RN/E), ascending
 cudaError_t launch_tiles_of_failed(const RegionGeom& g, int E, const int64_t* list, const int64_t* d_n,
@@ -63,6 +67,8 @@ struct TmmArgs {
   const int64_t* list;  // list mode (recovery) when non-null
   const int64_t* d_n;
   int list_is_tiles;    // list holds 128x128 tile ids (de-duplicated recovery of 32x32 regions)
+  const int32_t* tasks;  // tcgen05 list mode: paired recovery tasks (launch_pair_tasks), or null
+  const int64_t* d_ntasks;
   int force_1cta;       // tcgen05: use the 1-CTA 128x256 kernel even where the CTA-pair kernel applies
   int no_shuffle;       // SIMT: sequential shared-memory reduction (the paper's "no shuffle" ablation)
   int sm_count;

@@ -301,6 +301,104 @@ __global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t
   }
 }
 
+// ---------------------------------------------------------------------------
+// Recovery pairing (a10): the ascending failed list (128x128 regions or
+// de-duplicated 128x128 tiles) is cut into tasks of one or two entries of the same
+// 128-row band, so one CTA re-executes both with ONE A row panel staged for a
+// 128x256 tcgen05 tile (B gathered from the two column panels): 6 MiB of operand
+// reads per two regions instead of 8 MiB, and half the CTAs.  Inside each run of
+// equal rows, entries at even offsets from the run start head a task; a head takes
+// its successor when it lies in the same row.  Pairing is used only when there are
+// more entries than SMs (otherwise one entry per CTA finishes sooner).
+// tasks[t] = (list index << 1) | paired.  One CTA of 1024 threads, chunked scans.
+constexpr int kPairThreads = 1024;
+
+__device__ __forceinline__ int64_t block_scan_max_i64(int64_t v, int64_t* s_warp, int64_t* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int64_t y = __shfl_up_sync(0xFFFFFFFFu, v, o);
+    if (lane >= o) v = v > y ? v : y;
+  }
+  if (lane == 31) s_warp[wid] = v;
+  __syncthreads();
+  if (wid == 0) {
+    int64_t x = s_warp[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int64_t y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+      if (lane >= o) x = x > y ? x : y;
+    }
+    s_warp[lane] = x;
+  }
+  __syncthreads();
+  if (wid > 0) {
+    const int64_t y = s_warp[wid - 1];
+    v = v > y ? v : y;
+  }
+  *total = s_warp[31];
+  __syncthreads();
+  return v;
+}
+
+__device__ __forceinline__ int block_scan_excl_sum(int v, int* s_warp, int* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_warp[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    int t = s_warp[lane];
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int y = __shfl_up_sync(0xFFFFFFFFu, t, o);
+      if (lane >= o) t += y;
+    }
+    s_warp[lane] = t;
+  }
+  __syncthreads();
+  const int r = (wid > 0 ? s_warp[wid - 1] : 0) + x - v;
+  *total = s_warp[31];
+  __syncthreads();
+  return r;
+}
+
+__global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t* __restrict__ list,
+                                                                  const int64_t* __restrict__ d_n, int64_t off,
+                                                                  int64_t div, int64_t min_pair,
+                                                                  int32_t* __restrict__ tasks,
+                                                                  int64_t* __restrict__ d_ntasks) {
+  __shared__ int64_t s_max[32];
+  __shared__ int s_sum[32];
+  const int64_t n = *d_n;
+  const bool pairing = n > min_pair;
+  int64_t carry_ls = -1;  // index of the last run start seen so far
+  int64_t carry_t = 0;    // tasks emitted so far
+  for (int64_t base = 0; base < n; base += kPairThreads) {
+    const int64_t i = base + threadIdx.x;
+    const bool valid = i < n;
+    const int64_t row = valid ? (list[i] - off) / div : -1;
+    const int64_t prev = (valid && i > 0) ? (list[i - 1] - off) / div : -2;
+    const bool run_head = valid && row != prev;
+    int64_t blk_max;
+    int64_t ls = block_scan_max_i64(run_head ? i : -1, s_max, &blk_max);
+    ls = ls > carry_ls ? ls : carry_ls;
+    const bool head = valid && (!pairing || ((i - ls) & 1) == 0);
+    bool paired = false;
+    if (head && pairing && i + 1 < n) paired = (list[i + 1] - off) / div == row;
+    int tot;
+    const int idx = block_scan_excl_sum(head ? 1 : 0, s_sum, &tot);
+    if (head) tasks[carry_t + idx] = (int32_t)((i << 1) | (paired ? 1 : 0));
+    carry_t += tot;
+    carry_ls = blk_max > carry_ls ? blk_max : carry_ls;
+  }
+  if (threadIdx.x == 0) *d_ntasks = carry_t;
+}
+
 __global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed) {
   HashHeader* h = reinterpret_cast<HashHeader*>(ck);
   h->cap = cap;
@@ -532,6 +630,12 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int E, const int64_t* li
   tg.R = T;
   tg.rid_offset = 0;
   return launch_compact(tg, tile_flags, block_counts, tile_list, d_ntiles, st);
+}
+
+cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
+                              int32_t* tasks, int64_t* d_ntasks, cudaStream_t st) {
+  pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, tasks, d_ntasks);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st) {

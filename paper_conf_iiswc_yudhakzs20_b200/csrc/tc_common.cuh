@@ -78,7 +78,49 @@ struct TileSrc {
   int64_t Qr;                 // regions per output row band
   int reg;                    // region edge (32 or 128)
   int list_is_tiles;          // list holds tile ids (already de-duplicated)
-  __device__ __forceinline__ int64_t count() const { return list ? *d_n : num_m * num_n; }
+  const int32_t* tasks;       // paired list mode: (list index << 1) | paired (launch_pair_tasks)
+  const int64_t* d_ntasks;
+  int64_t n128;               // 128-column tiles per row (tile-id decoding)
+  __device__ __forceinline__ int64_t count() const {
+    return tasks ? *d_ntasks : (list ? *d_n : num_m * num_n);
+  }
+  // a list entry (128x128 tile id, or global rid of a 128x128 region) -> 128-row block, 128-col block
+  __device__ __forceinline__ void entry128(int64_t e, int64_t& mb, int64_t& cb) const {
+    if (list_is_tiles) {
+      mb = e / n128;
+      cb = e - mb * n128;
+    } else {
+      const int64_t rid = e - rid_offset;
+      mb = rid / Qr;
+      cb = rid - mb * Qr;
+    }
+  }
+  // Columns of tile t as two 128-column halves: [n_lo, n_lo+128) and, if has_hi,
+  // [n_hi, n_hi+128).  Full runs with BN = 256: contiguous halves; paired list
+  // mode: two failed tiles of the same row band (B gathered from two panels).
+  template <int BN>
+  __device__ __forceinline__ void cols(int64_t t, int64_t& mb, int64_t& n_lo, int64_t& n_hi, bool& has_hi) const {
+    if (tasks) {
+      const int32_t w = tasks[t];
+      const int64_t i = w >> 1;
+      int64_t cb;
+      entry128(list[i], mb, cb);
+      n_lo = cb * 128;
+      has_hi = (w & 1) != 0;
+      n_hi = n_lo;
+      if (has_hi) {
+        int64_t mb1, cb1;
+        entry128(list[i + 1], mb1, cb1);
+        n_hi = cb1 * 128;
+      }
+      return;
+    }
+    int64_t nb;
+    coords<BN>(t, mb, nb);
+    n_lo = nb * BN;
+    n_hi = n_lo + 128;
+    has_hi = BN == 256;
+  }
   template <int BN>
   __device__ __forceinline__ void coords(int64_t t, int64_t& mb, int64_t& nb) const {
     if (!list) {
@@ -212,6 +254,27 @@ __device__ __forceinline__ void epi_finish_128(int warp, int lane, const CkRecor
 #pragma unroll
     for (int w = 1; w < 4; ++w) rr = combine(rr, srec_acc[j * 4 + w]);
     const int64_t rid = m128 * Qr + n0 / 128 + j;
+    uint32_t words[3];
+    record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
+    store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+  }
+}
+
+// Same for a tile stored as two 128-column halves at n_lo and (if has_hi) n_hi --
+// contiguous in full runs, two column panels in paired recovery: one barrier, lane
+// h of the first epilogue warp finishes half h.
+template <typename OutT, uint32_t MASK, int STORE>
+__device__ __forceinline__ void epi_finish_halves(int warp, int lane, const CkRecord* srec_acc,
+                                                  uint32_t* __restrict__ ck, int64_t m128, int64_t n_lo, int64_t n_hi,
+                                                  bool has_hi, int64_t Qr, int64_t rid_offset) {
+  constexpr int ES = (int)sizeof(OutT);
+  named_bar_epi();
+  if (warp == kEpiWarp0 && (lane == 0 || (lane == 1 && has_hi))) {
+    const int j = lane;
+    CkRecord rr = srec_acc[j * 4 + 0];
+#pragma unroll
+    for (int w = 1; w < 4; ++w) rr = combine(rr, srec_acc[j * 4 + w]);
+    const int64_t rid = m128 * Qr + (j ? n_hi : n_lo) / 128;
     uint32_t words[3];
     record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
     store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);

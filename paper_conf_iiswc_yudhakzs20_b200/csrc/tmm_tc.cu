@@ -118,16 +118,22 @@ __global__ void __launch_bounds__(kThreads, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        int64_t mb, nb;
-        src.coords<BN>(t, mb, nb);
-        const int m0 = (int)(mb * kBM), n0 = (int)(nb * BN);
+        int64_t mb, n_lo, n_hi;
+        bool has_hi;
+        src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
+        const int m0 = (int)(mb * kBM);
+        // B is staged as 64-column chunks: 0,1 from the low half's panel, 2,3 from the high half's
+        const uint32_t bytes = Cfg::kABytes + (has_hi ? 4 : 2) * (kBK * 128);
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
-          mbar_expect_tx(&full[stage], Cfg::kStageBytes);
+          mbar_expect_tx(&full[stage], bytes);
           tma_load_2d(&tmap_a, &full[stage], sA + stage * Cfg::kABytes, kb * kBK, m0);
 #pragma unroll
-          for (int c = 0; c < BN / 64; ++c)
-            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), n0 + c * 64, kb * kBK);
+          for (int c = 0; c < BN / 64; ++c) {
+            if (c >= 2 && !has_hi) break;
+            const int64_t col = (c < 2 ? n_lo : n_hi) + (c & 1) * 64;
+            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), (int)col, kb * kBK);
+          }
           if (++stage == S) {
             stage = 0;
             phase ^= 1;
@@ -138,12 +144,16 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else if (warp == 1) {
     // ===================== MMA issuer (one thread) =====================
     if (lane == 0) {
-      constexpr uint32_t idesc = instr_desc<BN>();
       int stage = 0;
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        int64_t mb, n_lo, n_hi;
+        bool has_hi;
+        src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
+        // N = 256 when both halves are live, else N = 128 into the low half
+        const uint32_t idesc = (BN == 256 && has_hi) ? instr_desc<256>() : instr_desc<128>();
         mbar_wait(&tempty[acc], acc_phase ^ 1);  // epilogue drained this accumulator
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -180,20 +190,25 @@ __global__ void __launch_bounds__(kThreads, 1)
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      int64_t mb, nb;
-      src.coords<BN>(t, mb, nb);
+      int64_t mb, n_lo, n_hi;
+      bool has_hi;
+      src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
       CkRecord* srec_acc = srec + acc * (BN / 128) * 4;
-      epi_store<OutT, MASK, REG, BN, STORE>(t_row, C, ldc, mb, nb * BN, wq, lane, srec_acc, ck, src.Qr,
-                                            src.rid_offset);
+      epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
+                                             src.rid_offset);
+      if (BN == 256 && has_hi)
+        epi_store<OutT, MASK, REG, 128, STORE>(t_row + 128, C, ldc, mb, n_hi, wq, lane, srec_acc + 4, ck, src.Qr,
+                                               src.rid_offset);
       // all TMEM reads of this accumulator are complete (wait::ld): release it
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&tempty[acc]);
       if constexpr (MASK != 0 && REG == 128)
-        epi_finish_128<OutT, MASK, BN, STORE>(warp, lane, srec_acc, ck, mb, nb * BN, src.Qr, src.rid_offset);
+        epi_finish_halves<OutT, MASK, STORE>(warp, lane, srec_acc, ck, mb, n_lo, n_hi, BN == 256 && has_hi, src.Qr,
+                                             src.rid_offset);
       if (++acc == 2) {
         acc = 0;
         acc_phase ^= 1;
@@ -400,6 +415,9 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   src.Qr = a.N / REG;
   src.reg = REG;
   src.list_is_tiles = a.list_is_tiles;
+  src.tasks = a.list ? a.tasks : nullptr;
+  src.d_ntasks = a.d_ntasks;
+  src.n128 = a.N / 128;
   const int64_t R = (a.M / REG) * (a.N / REG);
   int64_t grid = a.list ? (R < a.sm_count ? R : a.sm_count) : src.num_m * src.num_n;
   if (grid > a.sm_count) grid = a.sm_count;
@@ -484,8 +502,9 @@ template <typename OutT, int REG>
 cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
   if (!a.list && a.M % 256 == 0 && a.N % 256 == 0 && !a.force_1cta) return launch_pair<OutT, REG>(a, st, why);
   // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
-  // 16 32x32 regions of a de-duplicated tile
-  const bool bn256 = (a.N % 256 == 0) && !a.list;
+  // 16 32x32 regions of a de-duplicated tile; paired tasks (two such tiles of one
+  // row band) run on the BN = 256 kernel with B gathered from two column panels
+  const bool bn256 = a.list ? (a.tasks != nullptr) : (a.N % 256 == 0);
   return bn256 ? launch_cfg<OutT, REG, 256>(a, st, why) : launch_cfg<OutT, REG, 128>(a, st, why);
 }
 

@@ -18,8 +18,8 @@ pytestmark = pytest.mark.gpu
 
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
-              store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True):
-    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle)
+              store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True, pairing=True):
+    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle, pairing=pairing)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -150,6 +150,23 @@ def test_tc_many_tiles_persistent(tc_pair):
     # more tiles than SMs: persistent scheduling + TMEM double buffering across tiles
     run_cycle(2048, 2048, 512, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", mode="stale_words",
               frac=0.05, check_values=True, tc_pair=tc_pair)
+
+
+@pytest.mark.parametrize("pairing", [True, False])
+@pytest.mark.parametrize("reg,N,frac", [(128, 2176, 0.7), (32, 2048, 0.1)])
+@pytest.mark.parametrize("out_dt", ["bf16", "f32"])
+def test_tc_paired_recovery(pairing, reg, N, frac, out_dt):
+    """More failed 128x128 tiles than SMs: failed tiles of one row band are re-executed in pairs on a 128x256
+    tcgen05 tile with B gathered from two column panels (odd runs leave single tiles; N = 2176 has 17 tile
+    columns).  Recovered bytes and records must equal the golden run either way."""
+    _, nf = run_cycle(2048, N, 256, reg, reg, "bf16", out_dt, "uniform", "mod|xor", "tcgen05", mode="stale_words",
+                      frac=frac, pairing=pairing)
+    assert nf > 148
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "cuckoo"])
+def test_tc_paired_recovery_hash_store(store):
+    run_cycle(2048, 2048, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, frac=0.75)
 
 
 @pytest.mark.parametrize("store", ["quad_cas", "quad_lock", "cuckoo", "cuckoo_lock"])
