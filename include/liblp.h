@@ -94,8 +94,12 @@ typedef enum { LP_F32 = 0, LP_BF16 = 1, LP_I32 = 2 } lp_dtype;
 
 /* Region bodies.  TMM = tiled matrix multiply (Listing 2, Listing 6
  * L546-554), C = A*B, idempotent.  STENCIL5 = 5-point stencil, out-of-place
- * (stand-in for the paper's bandwidth-bound class, Table I; Reading R19). */
-typedef enum { LP_WL_TMM = 0, LP_WL_STENCIL5 = 1 } lp_wl_kind;
+ * (stand-in for the paper's bandwidth-bound class, Table I; Reading R19).
+ * SPMV = CSR sparse matrix x dense vector, y = A*x (the paper's SPMV benchmark,
+ * Table I, bandwidth-bound; NEXT row N4): regions are region_n
+ * consecutive rows of y (region_m must be 1), i.e. y is viewed as the matrix
+ * [m / region_n][region_n] and region p = rows [p*region_n, (p+1)*region_n). */
+typedef enum { LP_WL_TMM = 0, LP_WL_STENCIL5 = 1, LP_WL_SPMV = 2 } lp_wl_kind;
 
 /* TMM body implementation: AUTO picks tcgen05 when the shape allows it. */
 typedef enum { LP_BODY_AUTO = 0, LP_BODY_SIMT = 1, LP_BODY_TCGEN05 = 2 } lp_body;
@@ -123,7 +127,7 @@ typedef struct {
 /* lp_config_t.flags */
 typedef enum {
   LP_FLAG_TC_1CTA = 1u,    /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
-  LP_FLAG_NO_SHUFFLE = 2u, /* SIMT body, MOD|XOR: sequential shared-memory reduction instead of warp reduction
+  LP_FLAG_NO_SHUFFLE = 2u, /* SIMT TMM and SPMV bodies: sequential shared-memory reduction instead of warp reduction
                               (the paper's "without parallel reduction" ablation, L343, Table IV) */
   LP_FLAG_NO_PAIRING = 4u  /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
                               failed tiles of the same row band into 128x256 tasks (A/B switch) */
@@ -142,6 +146,13 @@ typedef struct {
   int64_t ldc;       /* out row pitch in elements */
   int64_t row_offset, global_m; /* shard: rows [row_offset, row_offset+m) of global_m.
                                    STENCIL5 requires row_offset = 0, global_m = m. */
+  /* SPMV only (ignored otherwise): m = rows of A (= length of y = out), n = columns
+   * (= length of x = b), a = values (f32 [nnz]), b = x (f32 [n]), row_ptr (int64
+   * [m + 1], absolute offsets into a / col_idx for this shard's rows), col_idx
+   * (int32 [nnz], in [0, n)); ldc, lda, ldb, k are ignored.  Device pointers. */
+  const int64_t* row_ptr;
+  const int32_t* col_idx;
+  int64_t nnz;
 } lp_workload_t;
 
 typedef struct lp_ctx* lp_handle;

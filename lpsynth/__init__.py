@@ -10,6 +10,7 @@ import ctypes
 import os
 
 from .gen import DTYPES, KINDS, generate, raw, splitmix64, values_f32, f32_to_bf16_bits  # noqa: F401
+from . import csr  # noqa: F401
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 _LIB = None
@@ -26,6 +27,9 @@ def lib():
         L.synth_fill.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
                                  ctypes.c_int64, ctypes.c_int64, ctypes.c_uint64, ctypes.c_int,
                                  ctypes.c_int, ctypes.c_void_p]
+        L.synth_csr_cols.restype = ctypes.c_int
+        L.synth_csr_cols.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64,
+                                     ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p]
         _LIB = L
     return _LIB
 
@@ -42,3 +46,23 @@ def device_fill(tensor, seed: int, kind: str, dtype: str, row0: int = 0, ncols_g
                           cols if ncols_global is None else ncols_global, seed, KINDS[kind], DTYPES[dtype], s)
     if rc != 0:
         raise RuntimeError(f"synth_fill failed rc={rc}")
+
+
+def device_csr(seed_len: int, seed_col: int, seed_val: int, rows: int, ncols: int, kind: str = "uniform",
+               device="cuda", stream=None):
+    """The synthetic CSR matrix of csr.py on the device: (row_ptr int64 [rows+1], col_idx int32 [nnz],
+    values f32 [nnz]).  Row lengths / row_ptr are computed on the host (rows int64s); columns and
+    values are generated in HBM by the device twins."""
+    import torch
+
+    rp_h = csr.row_ptr(seed_len, rows)
+    nnz = int(rp_h[-1])
+    rp = torch.from_numpy(rp_h).to(device)
+    cols = torch.empty(nnz, dtype=torch.int32, device=device)
+    vals = torch.empty((1, nnz), dtype=torch.float32, device=device)
+    s = (stream or torch.cuda.current_stream()).cuda_stream
+    rc = lib().synth_csr_cols(rp.data_ptr(), rows, 0, ncols, seed_col, cols.data_ptr(), s)
+    if rc != 0:
+        raise RuntimeError(f"synth_csr_cols failed rc={rc}")
+    device_fill(vals, seed_val, kind, "f32", stream=stream)
+    return rp, cols, vals.view(-1)

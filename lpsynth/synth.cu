@@ -60,3 +60,35 @@ extern "C" int synth_fill(void* dst, int64_t rows, int64_t cols, int64_t ld, int
                                                                          seed, kind, dtype);
   return cudaGetLastError() == cudaSuccess ? 0 : 2;
 }
+
+// ---- SpMV structure (twin of lpsynth/csr.py columns()): one warp per row.
+namespace {
+constexpr int64_t kBandStride = 8;
+
+__global__ void synth_csr_cols_kernel(const int64_t* __restrict__ rp, int64_t rows, int64_t row0, int64_t ncols,
+                                      uint64_t seed, int32_t* __restrict__ cols) {
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5; i < rows; i += warps) {
+    const int64_t b = rp[i], e = rp[i + 1], len = e - b, r = row0 + i;
+    const int64_t base = r - (len * kBandStride) / 2;
+    for (int64_t k = lane; k < len; k += 32) {
+      const uint64_t h = splitmix64(seed * kGolden + (uint64_t)(b + k));
+      int64_t c = (base + k * kBandStride + (int64_t)(h % (uint64_t)kBandStride)) % ncols;
+      if (c < 0) c += ncols;
+      cols[b - rp[0] + k] = (int32_t)c;
+    }
+  }
+}
+}  // namespace
+
+// cols[0 .. rp[rows]-rp[0]) for rows [row0, row0+rows) given their device row_ptr slice rp[0..rows].
+extern "C" int synth_csr_cols(const int64_t* rp, int64_t rows, int64_t row0, int64_t ncols, uint64_t seed,
+                              int32_t* cols, void* stream) {
+  if (!rp || !cols || rows < 0 || ncols <= 0) return 1;
+  if (rows == 0) return 0;
+  int64_t blocks = (rows + 7) / 8;
+  if (blocks > 148 * 32) blocks = 148 * 32;
+  synth_csr_cols_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(rp, rows, row0, ncols, seed, cols);
+  return cudaGetLastError() == cudaSuccess ? 0 : 2;
+}

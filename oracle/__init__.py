@@ -85,6 +85,8 @@ def lib():
         L.lpo_round_bf16.argtypes = [_p, _i64, _p]
         L.lpo_stencil5_block.restype = None
         L.lpo_stencil5_block.argtypes = [_p, _i64, _i64, _i64, _i64, _i64, _i64, _i64, _p]
+        L.lpo_spmv_rows.restype = None
+        L.lpo_spmv_rows.argtypes = [_p, _p, _p, _p, _i64, _i64, _p]
         _LIB = L
     return _LIB
 
@@ -241,6 +243,20 @@ def stencil5_block(inp: np.ndarray, row0: int, col0: int, rows: int, cols: int) 
 def stencil5(inp: np.ndarray) -> np.ndarray:
     H, W = inp.shape
     return stencil5_block(inp, 0, 0, H, W)
+
+
+def spmv_rows(row_ptr: np.ndarray, col: np.ndarray, val: np.ndarray, x: np.ndarray, row0: int = 0,
+              rows: int | None = None) -> np.ndarray:
+    """fp64 y[row0:row0+rows] of the CSR product A @ x (lpo_spmv_rows; row_ptr absolute offsets)."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    val = np.ascontiguousarray(val, dtype=np.float32)
+    x = np.ascontiguousarray(x, dtype=np.float32)
+    if rows is None:
+        rows = len(row_ptr) - 1 - row0
+    y = np.zeros(rows, dtype=np.float64)
+    lib().lpo_spmv_rows(_ptr(row_ptr), _ptr(col), _ptr(val), _ptr(x), row0, rows, _ptr(y))
+    return y
 
 
 def rel_err(got: np.ndarray, ref: np.ndarray) -> float:

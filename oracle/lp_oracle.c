@@ -330,3 +330,19 @@ void lpo_stencil5_block(const float* in, int64_t H, int64_t W, int64_t ld, int64
       out[(i - row0) * cols + (j - col0)] = c + t;
     }
 }
+
+/* ------------------------------------------------------------------------ */
+/* Region body 3: sparse matrix - dense vector product, CSR (the paper's SPMV */
+/* benchmark, Table I, bandwidth-bound; NEXT row N4).  Definition:   */
+/*   y[i] = sum_{k = row_ptr[i]}^{row_ptr[i+1]-1} val[k] * x[col[k]]          */
+/* summed in fp64 in CSR order (exact for integer-valued inputs; the GPU's    */
+/* fp32 result is compared within the stated tolerance otherwise).            */
+/* Rows [row0, row0+rows) of the matrix; row_ptr holds absolute offsets.      */
+void lpo_spmv_rows(const int64_t* row_ptr, const int32_t* col, const float* val, const float* x, int64_t row0,
+                   int64_t rows, double* y /* rows */) {
+  for (int64_t i = 0; i < rows; ++i) {
+    double s = 0.0;
+    for (int64_t k = row_ptr[row0 + i]; k < row_ptr[row0 + i + 1]; ++k) s += (double)val[k] * (double)x[col[k]];
+    y[i] = s;
+  }
+}

@@ -74,7 +74,32 @@ bool aligned16(const void* p) { return (((uintptr_t)p) & 15u) == 0; }
 lp_status check_wl(const lp_ctx* h, const lp_workload_t* wl, lp::RegionGeom* g) {
   if (!h) return fail(LP_ERR_INVALID_ARG, "null handle");
   if (!wl) return fail(LP_ERR_INVALID_ARG, "null workload");
-  if (wl->kind != LP_WL_TMM && wl->kind != LP_WL_STENCIL5) return fail(LP_ERR_INVALID_ARG, "unknown workload kind %d", wl->kind);
+  if (wl->kind != LP_WL_TMM && wl->kind != LP_WL_STENCIL5 && wl->kind != LP_WL_SPMV)
+    return fail(LP_ERR_INVALID_ARG, "unknown workload kind %d", wl->kind);
+  if (wl->kind == LP_WL_SPMV) {
+    // regions = region_n consecutive rows of y, i.e. y viewed as [m / region_n][region_n]
+    const int RM = h->cfg.region_m, RN = h->cfg.region_n;
+    if (RM != 1) return fail(LP_ERR_INVALID_ARG, "SPMV regions are 1 x region_n row blocks (region_m must be 1)");
+    if (wl->in_dtype != LP_F32 || wl->out_dtype != LP_F32) return fail(LP_ERR_UNSUPPORTED, "SPMV is fp32 -> fp32");
+    if (wl->m <= 0 || wl->n <= 0) return fail(LP_ERR_INVALID_ARG, "m and n must be positive");
+    if (wl->m % RN) return fail(LP_ERR_INVALID_ARG, "m=%lld not divisible by region_n=%d (Reading R17)", (long long)wl->m, RN);
+    if (RN < 4 || (RN & (RN - 1))) return fail(LP_ERR_UNSUPPORTED, "SPMV region_n must be a power of two >= 4");
+    if (wl->row_offset < 0 || wl->global_m < wl->row_offset + wl->m || wl->row_offset % RN)
+      return fail(LP_ERR_INVALID_ARG, "shard rows [row_offset, row_offset+m) invalid for region_n");
+    g->M = wl->m / RN;
+    g->N = RN;
+    g->ldc = RN;
+    g->es = 4;
+    g->RM = 1;
+    g->RN = RN;
+    g->P = g->M;
+    g->Q = 1;
+    g->R = g->P;
+    g->rid_offset = wl->row_offset / RN;
+    if (g->rid_offset + g->R > (int64_t)0xFFFFFFFEll && h->cfg.store != LP_STORE_ARRAY)
+      return fail(LP_ERR_UNSUPPORTED, "hash stores key on 32-bit rids");
+    return LP_OK;
+  }
   if (wl->in_dtype < LP_F32 || wl->in_dtype > LP_I32 || wl->out_dtype < LP_F32 || wl->out_dtype > LP_I32)
     return fail(LP_ERR_INVALID_ARG, "unknown dtype");
   if ((wl->in_dtype == LP_I32) != (wl->out_dtype == LP_I32))
@@ -188,6 +213,8 @@ size_t workspace_bytes(const lp::RegionGeom& g) { return ws_layout(g).total; }
 lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
                    const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr) {
   const lp::HashInfo hi = hash_info(h, g);
+  if ((h->cfg.flags & LP_FLAG_NO_SHUFFLE) && wl->kind == LP_WL_STENCIL5)
+    return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is not built for the stencil body");
   if (wl->kind == LP_WL_STENCIL5) {
     if (!lp::stencil_supported(g.RM, g.RN)) return fail(LP_ERR_UNSUPPORTED, "stencil supports 128x128 regions");
     if (!wl->a) return fail(LP_ERR_INVALID_ARG, "null stencil input");
@@ -211,6 +238,29 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.sm_count = h->sm_count;
     cudaError_t e = lp::launch_stencil(a, st);
     return e == cudaSuccess ? ok() : cuda_fail(e, "stencil launch");
+  }
+  if (wl->kind == LP_WL_SPMV) {
+    if (!wl->a || !wl->b || !wl->row_ptr || !wl->col_idx) return fail(LP_ERR_INVALID_ARG, "null SPMV operand");
+    if (!aligned16(out)) return fail(LP_ERR_INVALID_ARG, "y must be 16-B aligned");
+    lp::SpmvArgs a;
+    a.row_ptr = wl->row_ptr;
+    a.col = wl->col_idx;
+    a.val = (const float*)wl->a;
+    a.x = (const float*)wl->b;
+    a.y = (float*)out;
+    a.m = wl->m;
+    a.RN = g.RN;
+    a.lpr = lp::spmv_lanes_per_row(wl->nnz, wl->m);
+    a.mask = h->mask;
+    a.hash = hi;
+    a.ck = (uint32_t*)ck;
+    a.rid_offset = g.rid_offset;
+    a.list = list;
+    a.d_n = d_n;
+    a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
+    a.sm_count = h->sm_count;
+    cudaError_t e = lp::launch_spmv(a, st);
+    return e == cudaSuccess ? ok() : cuda_fail(e, "SPMV launch");
   }
   if (!wl->a || !wl->b) return fail(LP_ERR_INVALID_ARG, "null A or B");
   if (wl->lda < wl->k || wl->ldb < wl->n) return fail(LP_ERR_INVALID_ARG, "lda < k or ldb < n");
@@ -246,7 +296,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   const bool tf_ok = !a.i32 && lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, a.out_bf16,
                                                        wl->lda, wl->ldb, wl->ldc, wl->a, wl->b, out);
   int body = h->cfg.body;
-  if (body == LP_BODY_AUTO) body = (tc_ok || tf_ok) ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
+  if (body == LP_BODY_AUTO) body = (tc_ok || tf_ok) && !a.no_shuffle ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
   if (body == LP_BODY_TCGEN05) {
     if (!tc_ok && !tf_ok)
       return fail(LP_ERR_UNSUPPORTED,
@@ -311,8 +361,8 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
-  if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body != LP_BODY_SIMT || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
-    return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT body with MOD|XOR records");
+  if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
+    return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");
   if ((int64_t)cfg->region_m * cfg->region_n * 4 > (16ll << 20))
     return fail(LP_ERR_UNSUPPORTED, "regions larger than 16 MiB are not supported");
   lp_ctx* h = new lp_ctx();

@@ -108,6 +108,28 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st);
 // mismatch, re-executes in place; *d_recovered (zeroed here) counts re-executed regions.
 cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recovered, cudaStream_t st);
 
+// ---- spmv.cu : CSR sparse matrix x dense vector region body (N4), regions of RN consecutive rows
+struct SpmvArgs {
+  const int64_t* row_ptr;  // [m + 1], absolute offsets into col / val
+  const int32_t* col;
+  const float* val;
+  const float* x;
+  float* y;                // [m]
+  int64_t m;
+  int RN;
+  int lpr;                 // lanes per row (spmv_lanes_per_row)
+  uint32_t mask;
+  HashInfo hash;
+  uint32_t* ck;
+  int64_t rid_offset;
+  const int64_t* list;
+  const int64_t* d_n;
+  int no_shuffle;
+  int sm_count;
+};
+int spmv_lanes_per_row(int64_t nnz, int64_t m);
+cudaError_t launch_spmv(const SpmvArgs& a, cudaStream_t st);
+
 // ---- fn_study.cu : false-negative study (N3)
 cudaError_t launch_fn_study(uint64_t seed, int64_t trials, int64_t nwords, int mode, int kmax,
                             unsigned long long* counts, uint32_t* dump, int64_t dump_trials, int sm_count,

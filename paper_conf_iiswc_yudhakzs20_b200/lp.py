@@ -24,7 +24,7 @@ LP_OK, LP_ERR_INVALID_ARG, LP_ERR_UNSUPPORTED, LP_ERR_CUDA, LP_ERR_CAPACITY, LP_
 CK_NONE, CK_MOD, CK_XOR, CK_ADLER32 = 0, 1, 2, 4
 STORE_ARRAY, STORE_QUAD_CAS, STORE_QUAD_LOCK, STORE_CUCKOO, STORE_CUCKOO_LOCK = 0, 1, 2, 3, 4
 F32, BF16, I32 = 0, 1, 2
-WL_TMM, WL_STENCIL5 = 0, 1
+WL_TMM, WL_STENCIL5, WL_SPMV = 0, 1, 2
 BODY_AUTO, BODY_SIMT, BODY_TCGEN05 = 0, 1, 2
 FLAG_TC_1CTA = 1
 FLAG_NO_SHUFFLE = 2
@@ -71,7 +71,8 @@ class CWorkload(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("in_dtype", ctypes.c_int32), ("out_dtype", ctypes.c_int32),
                 ("reserved", ctypes.c_int32), ("m", ctypes.c_int64), ("n", ctypes.c_int64), ("k", ctypes.c_int64),
                 ("a", ctypes.c_void_p), ("lda", ctypes.c_int64), ("b", ctypes.c_void_p), ("ldb", ctypes.c_int64),
-                ("ldc", ctypes.c_int64), ("row_offset", ctypes.c_int64), ("global_m", ctypes.c_int64)]
+                ("ldc", ctypes.c_int64), ("row_offset", ctypes.c_int64), ("global_m", ctypes.c_int64),
+                ("row_ptr", ctypes.c_void_p), ("col_idx", ctypes.c_void_p), ("nnz", ctypes.c_int64)]
 
 
 _LIB = None
@@ -166,6 +167,9 @@ class Workload:
     ldc: int = 0
     row_offset: int = 0
     global_m: int = 0
+    row_ptr: object = None
+    col_idx: object = None
+    nnz: int = 0
 
     @staticmethod
     def tmm(a, b, out_dtype="bf16", m=None, n=None, k=None, row_offset=0, global_m=None, ldc=None) -> "Workload":
@@ -189,9 +193,24 @@ class Workload:
             lda = W
         return Workload(WL_STENCIL5, H, W, 0, inp, None, F32, F32, lda, 0, W, 0, H)
 
+    @staticmethod
+    def spmv(values, x, row_ptr, col_idx, m=None, row_offset=0, global_m=None) -> "Workload":
+        """y[m] = A x for the CSR matrix (row_ptr int64 [m+1], col_idx int32 [nnz], values f32 [nnz]) and
+        x f32 [n] (the paper's SPMV, Table I; N4).  Regions = region_n consecutive rows of y (region_m = 1);
+        out is allocated as [m / region_n, region_n] by LP.alloc.  Tensors None -> sizing only (give m, n=len(x))."""
+        if row_ptr is not None:
+            m = row_ptr.numel() - 1
+        n = x.numel() if x is not None else 1
+        nnz = values.numel() if values is not None else 0
+        w = Workload(WL_SPMV, m, n, 0, values, x, F32, F32, 0, 0, 0, row_offset,
+                     global_m if global_m is not None else row_offset + m)
+        w.row_ptr, w.col_idx, w.nnz = row_ptr, col_idx, nnz
+        return w
+
     def c(self) -> CWorkload:
         return CWorkload(self.kind, self.in_dtype, self.out_dtype, 0, self.m, self.n, self.k, _ptr(self.a), self.lda,
-                         _ptr(self.b), self.ldb, self.ldc, self.row_offset, self.global_m or self.row_offset + self.m)
+                         _ptr(self.b), self.ldb, self.ldc, self.row_offset, self.global_m or self.row_offset + self.m,
+                         _ptr(self.row_ptr), _ptr(self.col_idx), self.nnz)
 
 
 class LP:
@@ -286,7 +305,10 @@ class LP:
         dev = torch.device("cuda", self.device if device is None else device)
         dt = {BF16: torch.bfloat16, F32: torch.float32, I32: torch.int32}[wl.out_dtype]
         R = self.num_regions(wl)
-        out = torch.empty((wl.m, wl.ldc), dtype=dt, device=dev)[:, :wl.n]
+        if wl.kind == WL_SPMV:   # y viewed as [m / region_n][region_n]
+            out = torch.empty((wl.m // self.region[1], self.region[1]), dtype=dt, device=dev)
+        else:
+            out = torch.empty((wl.m, wl.ldc), dtype=dt, device=dev)[:, :wl.n]
         ckb = max(self.cksum_bytes(wl), 16)
         ck = torch.empty((ckb + 3) // 4, dtype=torch.int32, device=dev)
         failed = torch.empty(max(R, 1), dtype=torch.int64, device=dev)
