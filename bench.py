@@ -85,12 +85,26 @@ WORKLOADS = {
     # the paper's own TMM (Table I/III/V: int TMM 4096^2, 32x32 thread-block regions, MOD+XOR; V100: 6.2%)
     "tmm4096_i32_paper": dict(kind="tmm", M=4096, N=4096, K=4096, in_dt="i32", out_dt="i32", region=32,
                               cksum="mod|xor", frac=0.05, store="array", weak=True, body="simt"),
+    # NEXT row N4: the paper's SPMV class (Table I, bandwidth-bound): CSR y = A x, 4 Mi rows, ~24 nnz/row
+    # (banded, heavy-tailed row lengths), regions of 1024 rows of y, 10% of the regions corrupted
+    "spmv4m": dict(kind="spmv", M=4194304, N=4194304, K=0, in_dt="f32", out_dt="f32", region=1024,
+                   cksum="mod|xor", frac=0.10, store="array", weak=False),
     # BASELINE configs[4]: 65536^3 bf16 region-sharded across ranks (strong scaling)
     "tmm65536_bf16": dict(kind="tmm", M=65536, N=65536, K=65536, in_dt="bf16", out_dt="bf16", region=128,
                           cksum="mod|xor", frac=0.05, store="array", weak=False),
 }
 
-KERNELS_PER_CALL = {"run_protected": 1, "inject": 1, "validate": 3, "recover": 1}
+def kernels_per_step(W, store):
+    """Our kernels launched by one step (init memset is not a kernel): protected body (+ hash header),
+    inject, 2 x (validate + ordered-compaction scatter), recovery (+ tile de-dup / pairing kernels)."""
+    body = 1 + (1 if store != "array" else 0)
+    if W["kind"] == "tmm" and W["in_dt"] == "bf16" and W.get("body") != "simt":
+        rec = 2 if W["region"] == 128 else 5          # pair builder + tcgen05; r32: mark, count, scatter too
+    elif W["kind"] == "tmm" and W["in_dt"] == "f32" and W.get("body") != "simt":
+        rec = 4                                        # tile mark, count, scatter, 3xTF32 list mode
+    else:
+        rec = 1
+    return body + 1 + 2 * 2 + rec
 
 
 def parse():
@@ -219,6 +233,9 @@ def run_ours(args):
     if args.cksum:
         W["cksum"] = args.cksum
     RM = RN = W["region"]
+    if W["kind"] == "spmv":
+        RM = 1
+    rp_host = None
     if W["kind"] == "tmm":
         gM = W["M"] * (world if W["weak"] else 1)
         sh = shard.plan(gM, W["N"], RM, RN, world, rank)
@@ -231,6 +248,20 @@ def run_ours(args):
         lpsynth.device_fill(b, 2, ikind, W["in_dt"])
         wl = lp.Workload.tmm(a, b, out_dtype=W["out_dt"], row_offset=sh.row_offset, global_m=gM)
         body_flops = 2.0 * M * N * K
+    elif W["kind"] == "spmv":
+        from lpsynth import csr
+        gM = W["M"]
+        if world > 1:
+            raise SystemExit("spmv workload is single-GPU in this round")
+        sh = shard.plan(gM // RN, RN, 1, RN, 1, 0)   # y viewed as [M / RN][RN]
+        M, N, K = W["M"], W["N"], 0
+        rp_d, cols_d, vals_d = lpsynth.device_csr(31, 32, 33, M, N, "uniform")
+        x_d = torch.empty((1, N), dtype=torch.float32, device=dev)
+        lpsynth.device_fill(x_d, 34, "uniform", "f32")
+        rp_host = csr.row_ptr(31, M)
+        a, b = vals_d, x_d.view(-1)
+        wl = lp.Workload.spmv(vals_d, x_d.view(-1), rp_d, cols_d)
+        body_flops = 2.0 * float(rp_host[-1])
     else:
         gM = W["M"]
         if world > 1:
@@ -268,7 +299,7 @@ def run_ours(args):
         flush_rd.max()
     st = torch.cuda.current_stream()
 
-    out_bytes = M * N * es_out
+    out_bytes = out.numel() * es_out
     ck_bytes = h.cksum_bytes(wl)
     es_in = 2 if W["in_dt"] == "bf16" else 4
     Qr = N // RN
@@ -280,6 +311,10 @@ def run_ours(args):
             ps = {int(r) // Qr for r in rids_local}
             qs = {int(r) % Qr for r in rids_local}
             return (len(ps) * RM * K + len(qs) * K * RN) * es_in + len(rids_local) * RM * RN * es_out
+        if W["kind"] == "spmv":
+            # per region: its nnz (value + column index), row_ptr slice, y rows written, x band read once
+            return sum(int(rp_host[(r + 1) * RN] - rp_host[r * RN]) * 8 + (RN + 1) * 8 + RN * 4 + RN * 4
+                       for r in rids_local)
         return len(rids_local) * ((RM + 2) * (RN + 2) * 4 + RM * RN * 4)
 
     def ev():
@@ -460,9 +495,18 @@ def run_ours(args):
 
     line = None
     if rank == 0:
-        launches = args.steps * (KERNELS_PER_CALL["run_protected"] + KERNELS_PER_CALL["inject"] +
-                                 2 * KERNELS_PER_CALL["validate"] + KERNELS_PER_CALL["recover"])
-        if W["kind"] == "tmm":
+        launches = args.steps * kernels_per_step(W, W["store"])
+        if W["kind"] == "spmv":
+            nnz = float(rp_host[-1])
+            sb = nnz * 8 + (M + 1) * 8 + N * 4 + M * 4
+            achieved = sb / (t_prot * 1e-3) / 1e9
+            roof = {"bound": "hbm", "kernel": f"spmv_kernel (protected, {W['cksum']})", "achieved": round(achieved, 1),
+                    "peak": hbm, "unit": "GB/s", "frac": round(achieved / hbm, 4),
+                    "peak_source": f"{peak_src} HBM copy",
+                    "algorithmic_per_launch": f"nnz*(4 B value + 4 B column) + (m+1)*8 B row_ptr + n*4 B x + "
+                                              f"m*4 B y = {sb:.4g} B",
+                    "traffic": ncu_traffic("spmv_kernel", args.workload)}
+        elif W["kind"] == "tmm":
             if W.get("body") == "simt":
                 kname = "tmm_simt_kernel"
                 # FP32 FFMA peak: 148 SMs x 128 FMA/clk x 2 flop x max SM clock (guide unit counts);
@@ -557,7 +601,7 @@ def run_ours(args):
         }
     if world > 1:
         dist.barrier()
-    if rank == 0 and world == 1 and not args.no_cpu_baseline and W["kind"] in ("tmm", "stencil"):
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(W, args.cpu_seconds, out, ck, a, b, R, RM, RN, wl_kind=W["kind"])
     if rank == 0:
         print(json.dumps(line), flush=True)
@@ -594,6 +638,21 @@ def _oracle_sample_gbs(W, seconds, out_np, ck_np, A_np, B_np, RM, RN, R, mask):
             oracle.gemm_block_f64(A_np, B_np, 0, RN * recovered, RM, RN)
             n_bytes += (RM * W["K"] + W["K"] * RN) * A_np.dtype.itemsize + RM * RN * es
             recovered += 1
+    elif W["kind"] == "spmv":
+        # A_np = the host CSR recipe (row_ptr, x); each re-executed region regenerates its rows' columns and
+        # values from the seeds (same recipe as the device twin) and runs the fp64 oracle product
+        from lpsynth import csr, gen
+        rp, x = A_np
+        RNs = RN
+        while time.perf_counter() - t1 < seconds * 0.5 or recovered == 0:
+            r0 = RNs * (recovered % (len(rp) // RNs))
+            sl = rp[r0:r0 + RNs + 1]
+            cnt = int(sl[-1] - sl[0])
+            cols = csr.columns(32, sl, len(x), row0=r0)
+            vals = gen.values_f32(33, 1, cnt, "uniform", col0=int(sl[0]), ncols_global=int(rp[-1]))[0]
+            oracle.spmv_rows(sl - sl[0], cols, vals, x, 0, RNs)
+            n_bytes += cnt * 8 + (RNs + 1) * 8 + RNs * 8
+            recovered += 1
     else:
         while time.perf_counter() - t1 < seconds * 0.5 or recovered == 0:
             oracle.stencil5_block(A_np, RM * recovered, 0, RM, RN)
@@ -614,6 +673,10 @@ def cpu_baseline(W, seconds, out, ck, a, b, R, RM, RN, wl_kind):
     if wl_kind == "tmm":
         A_np = dev_to_host(a[:RM].contiguous())
         B_np = dev_to_host(b)
+    elif wl_kind == "spmv":
+        from lpsynth import csr
+        A_np = (csr.row_ptr(31, W["M"]), dev_to_host(b))
+        B_np = None
     else:
         A_np = dev_to_host(a[:RM * 64].contiguous())
         B_np = None
@@ -641,7 +704,17 @@ def run_reference(args):
     sel = oracle.selem(mask)
     # a bounded slab of the same workload: RM rows of A, a 16-region-wide slab of B/out
     cols = RN * 16
-    if W["kind"] == "tmm":
+    if W["kind"] == "spmv":
+        # the first 16 regions (16 x RN rows) of the same synthetic matrix and the full x
+        from lpsynth import csr
+        RM = 1
+        rp = csr.row_ptr(31, RN * 16)
+        x = gen.values_f32(34, 1, W["N"], "uniform")[0]
+        c = csr.columns(32, rp, W["N"])
+        v = gen.values_f32(33, 1, int(rp[-1]), "uniform")[0]
+        out = oracle.spmv_rows(rp, c, v, x).astype(np.float32).reshape(16, RN)
+        A, B = (rp, x), None
+    elif W["kind"] == "tmm":
         A = gen.generate(1, RM, W["K"], "uniform", W["in_dt"])
         B = gen.generate(2, W["K"], cols, "uniform", W["in_dt"])
         out = oracle.round_bf16(oracle.gemm_block_f64(A, B, 0, 0, RM, cols)) if W["out_dt"] == "bf16" else \

@@ -83,7 +83,7 @@ lp_status check_wl(const lp_ctx* h, const lp_workload_t* wl, lp::RegionGeom* g) 
     if (wl->in_dtype != LP_F32 || wl->out_dtype != LP_F32) return fail(LP_ERR_UNSUPPORTED, "SPMV is fp32 -> fp32");
     if (wl->m <= 0 || wl->n <= 0) return fail(LP_ERR_INVALID_ARG, "m and n must be positive");
     if (wl->m % RN) return fail(LP_ERR_INVALID_ARG, "m=%lld not divisible by region_n=%d (Reading R17)", (long long)wl->m, RN);
-    if (RN < 4 || (RN & (RN - 1))) return fail(LP_ERR_UNSUPPORTED, "SPMV region_n must be a power of two >= 4");
+    if (!lp::spmv_supported(RN)) return fail(LP_ERR_UNSUPPORTED, "SPMV region_n must be a power of two in [4, 16384]");
     if (wl->row_offset < 0 || wl->global_m < wl->row_offset + wl->m || wl->row_offset % RN)
       return fail(LP_ERR_INVALID_ARG, "shard rows [row_offset, row_offset+m) invalid for region_n");
     g->M = wl->m / RN;
@@ -241,7 +241,9 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   }
   if (wl->kind == LP_WL_SPMV) {
     if (!wl->a || !wl->b || !wl->row_ptr || !wl->col_idx) return fail(LP_ERR_INVALID_ARG, "null SPMV operand");
-    if (!aligned16(out)) return fail(LP_ERR_INVALID_ARG, "y must be 16-B aligned");
+    if (!aligned16(out) || !aligned16(wl->a) || !aligned16(wl->col_idx))
+      return fail(LP_ERR_INVALID_ARG, "y, values and col_idx must be 16-B aligned");
+    if (wl->nnz < 0) return fail(LP_ERR_INVALID_ARG, "negative nnz");
     lp::SpmvArgs a;
     a.row_ptr = wl->row_ptr;
     a.col = wl->col_idx;
@@ -249,8 +251,9 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.x = (const float*)wl->b;
     a.y = (float*)out;
     a.m = wl->m;
+    a.n = wl->n;
+    a.nnz = wl->nnz;
     a.RN = g.RN;
-    a.lpr = lp::spmv_lanes_per_row(wl->nnz, wl->m);
     a.mask = h->mask;
     a.hash = hi;
     a.ck = (uint32_t*)ck;

@@ -110,14 +110,13 @@ cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recove
 
 // ---- spmv.cu : CSR sparse matrix x dense vector region body (N4), regions of RN consecutive rows
 struct SpmvArgs {
-  const int64_t* row_ptr;  // [m + 1], absolute offsets into col / val
+  const int64_t* row_ptr;  // [m + 1], absolute offsets into col / val (16-B aligned arrays)
   const int32_t* col;
   const float* val;
   const float* x;
   float* y;                // [m]
-  int64_t m;
+  int64_t m, n, nnz;       // rows, columns (length of x), stored elements (val / col length)
   int RN;
-  int lpr;                 // lanes per row (spmv_lanes_per_row)
   uint32_t mask;
   HashInfo hash;
   uint32_t* ck;
@@ -127,7 +126,7 @@ struct SpmvArgs {
   int no_shuffle;
   int sm_count;
 };
-int spmv_lanes_per_row(int64_t nnz, int64_t m);
+bool spmv_supported(int RN);
 cudaError_t launch_spmv(const SpmvArgs& a, cudaStream_t st);
 
 // ---- fn_study.cu : false-negative study (N3)

@@ -99,17 +99,33 @@ def test_spmv_region_sizes(RN):
     run_spmv_cycle(synth(max(RN * 24, 4 * 4096), 30000, "int5"), RN, "int5", frac=0.25)
 
 
-@pytest.mark.parametrize("length", [3, 40, 120])
-def test_spmv_lanes_per_row_variants(length):
-    """Mean row length picks 4 / 16 / 32 lanes per row (the recipe's ~24 picks 8 or 16)."""
-    rows = 8192
-    lens = 1 + (np.arange(rows) * 7919) % (2 * length - 1)
+@pytest.mark.parametrize("length", [2, 40, 1500])
+def test_spmv_row_length_mixes(length):
+    """Short rows with empty ones (a 2048-element chunk spans > 256 rows), long rows, and rows longer than a
+    chunk (each row is still summed in CSR order across chunk boundaries)."""
+    rows = 8192 if length < 1000 else 1024
+    lens = (np.arange(rows) * 7919) % (2 * length + 1)
     rp = np.zeros(rows + 1, dtype=np.int64)
     np.cumsum(lens, out=rp[1:])
-    cols = csr.columns(2, rp, 9000)
+    ncols = max(9000, 2 * length * csr.BAND_STRIDE)
+    cols = csr.columns(2, rp, ncols)
     vals = gen.values_f32(3, 1, int(rp[-1]), "int5")[0]
-    x = gen.values_f32(4, 1, 9000, "int5")[0]
-    run_spmv_cycle((rp, cols, vals, x), 512, "int5", mode="stale_region", frac=0.3)
+    x = gen.values_f32(4, 1, ncols, "int5")[0]
+    run_spmv_cycle((rp, cols, vals, x), 512 if length < 1000 else 64, "int5", mode="stale_region", frac=0.3)
+
+
+def test_spmv_nnz_not_multiple_of_4_and_unaligned_regions():
+    """Region nnz ranges start at arbitrary offsets and the array ends in a partial 16-byte vector."""
+    rows = 4096
+    lens = 1 + (np.arange(rows) * 31) % 7
+    rp = np.zeros(rows + 1, dtype=np.int64)
+    np.cumsum(lens, out=rp[1:])
+    if rp[-1] % 4 == 0:
+        rp[-1] += 1
+    cols = csr.columns(5, rp, 5000)
+    vals = gen.values_f32(6, 1, int(rp[-1]), "uniform")[0]
+    x = gen.values_f32(7, 1, 5000, "uniform")[0]
+    run_spmv_cycle((rp, cols, vals, x), 256, "uniform", frac=0.3)
 
 
 @pytest.mark.parametrize("store", ["quad_cas", "quad_lock", "cuckoo"])
