@@ -113,6 +113,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="process-group backend for N>1 (gloo + --same-device: test the N>1 path on one GPU)")
+    ap.add_argument("--same-device", action="store_true", help="test hook: put every rank on cuda:0")
     ap.add_argument("--workload", default="tmm8192_bf16", choices=sorted(WORKLOADS))
     ap.add_argument("--overhead-reps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -223,9 +226,14 @@ def run_ours(args):
     from paper_conf_iiswc_yudhakzs20_b200 import lp, report, shard
 
     world, rank, local = dist_env()
+    if args.same_device:       # test hook: every rank on cuda:0 (exercise the N>1 path on a 1-GPU box)
+        local = 0
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(args.dist_backend)
     dev = torch.device("cuda", local)
     W = dict(WORKLOADS[args.workload])
     if args.store:
@@ -284,8 +292,8 @@ def run_ours(args):
     lpsynth.device_fill(stale.view(torch.int32) if es_out == 4 else stale.view(torch.int16).view(torch.bfloat16),
                         3, "bits", "bf16" if es_out == 2 else "u32", row0=sh.row_offset, ncols_global=N)
     out.copy_(stale)
-    inj_host = lp.choose_regions(R, W["frac"], 1000 + rank)
-    inj = torch.from_numpy(inj_host).to(dev)
+    inj_host = lp.choose_regions(R, W["frac"], 1000 + rank)          # local region indices of this shard
+    inj = torch.from_numpy(inj_host + sh.rid_offset).to(dev)           # lp_inject takes GLOBAL rids
     k_inj = len(inj_host)
     counts = torch.zeros(3, dtype=torch.int64, device=dev)
     l2 = torch.cuda.get_device_properties(dev).L2_cache_size

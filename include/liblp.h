@@ -219,7 +219,8 @@ LP_API lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const
                               lp_stream_t stream);
 
 /* Crash injection (harness only): corrupt the n regions whose GLOBAL rids are
- * in device array rids[0..n) according to `mode` (lp_inject_mode), using the
+ * in device array rids[0..n) (ids outside this shard's range are skipped)
+ * according to `mode` (lp_inject_mode), using the
  * stale image `stale` (same shape/pitch as out; may be NULL for BITFLIP and
  * STALE_RECORD) and counter-based choices seeded by `seed`. */
 LP_API lp_status lp_inject(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const void* stale,

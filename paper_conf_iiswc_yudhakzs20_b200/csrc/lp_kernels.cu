@@ -423,9 +423,10 @@ __global__ void stats_kernel(const uint32_t* ck, int has_hash, int64_t* d_stats)
 template <int S>
 __global__ void inject_kernel(uint8_t* out, int64_t ldc_bytes, int64_t Q, int RM, int row_bytes,
                               const uint8_t* stale, uint32_t* ck, int store, const int64_t* rids, int64_t rid_offset,
-                              uint32_t mode, uint64_t seed) {
+                              int64_t R, uint32_t mode, uint64_t seed) {
   const int64_t grid = rids[blockIdx.x];
   const int64_t r = grid - rid_offset;
+  if (r < 0 || r >= R) return;  // not a region of this shard (rids are global): nothing to corrupt
   const int64_t p = r / Q, q = r - p * Q;
   const int64_t base = p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
   const int wpr = row_bytes / 4;
@@ -608,7 +609,7 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
 #define LP_ICASE(SV)                                                                                           \
   inject_kernel<SV><<<(unsigned)n, 256, 0, st>>>((uint8_t*)out, g.ldc * g.es, g.Q, g.RM, row_bytes,           \
                                                  (const uint8_t*)stale, (uint32_t*)ck, hi.store, rids,        \
-                                                 g.rid_offset, mode, seed)
+                                                 g.rid_offset, g.R, mode, seed)
   if (S == 1) LP_ICASE(1);
   else if (S == 2) LP_ICASE(2);
   else LP_ICASE(3);

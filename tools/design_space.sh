@@ -1,19 +1,22 @@
 #!/bin/bash
 # The paper's design space (Fig. 5 / Tables III-IV / V) on its own TMM (int32 4096^2, 32x32 thread-block
-# regions, MOD+XOR), B200: store x lock x reduction.  -> gpurun_out/design/*.json
-mkdir -p gpurun_out/design
+# regions, MOD+XOR), B200: store x lock x reduction.  -> gpurun_out/design_<workload>/*.json
+# Usage: bash tools/design_space.sh [workload]   (default tmm4096_i32_paper; spmv4m = the paper's SPMV class)
+WL=${1:-tmm4096_i32_paper}
+D=gpurun_out/design_$WL
+mkdir -p $D
 for st in array quad_cas quad_lock cuckoo cuckoo_lock; do
   for sh in "" "--no-shuffle"; do
     tag=${st}${sh:+_noshfl}
-    timeout 900 python bench.py --workload tmm4096_i32_paper --store $st $sh --steps 3 --warmup 3 --overhead-reps 10 \
-      --no-cpu-baseline > gpurun_out/design/$tag.json 2> gpurun_out/design/$tag.err || tail -2 gpurun_out/design/$tag.err
+    timeout 900 python bench.py --workload $WL --store $st $sh --steps 3 --warmup 3 --overhead-reps 10 \
+      --no-cpu-baseline > $D/$tag.json 2> $D/$tag.err || tail -2 $D/$tag.err
   done
 done
-python - <<'PY'
+D=$D python - <<'PY'
 import glob, json, os
 print("| store | reduction | t_prot ms | t_unprot ms | LP overhead | slowdown (x) | hash collisions |")
 print("|---|---|---|---|---|---|---|")
-for f in sorted(glob.glob("gpurun_out/design/*.json")):
+for f in sorted(glob.glob(os.environ["D"] + "/*.json")):
     try:
         d = json.loads(open(f).read().strip().splitlines()[-1])
     except Exception:
