@@ -171,7 +171,11 @@ LP_API lp_status lp_num_regions(lp_handle h, const lp_workload_t* wl, int64_t* r
  * (total load <= 50%, L270). */
 LP_API lp_status lp_cksum_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
 
-/* Bytes of the scratch `workspace` lp_validate needs (flags + scan counters). */
+/* Bytes of the scratch `workspace` lp_validate / lp_recover use (flags, scan counters,
+ * recovery tile lists, the fused-compaction ticket).  The caller zero-fills it ONCE
+ * before its first use (cudaMemset); every call leaves the ticket back at zero, so the
+ * workspace can be reused (and replayed in CUDA graphs) without re-initialisation.
+ * One workspace per in-flight call (calls sharing a workspace must be stream-ordered). */
 LP_API lp_status lp_workspace_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
 
 /* Fill the table with the sentinel 0xFFFFFFFF (Reading R8; hash: all keys empty,
@@ -187,7 +191,8 @@ LP_API lp_status lp_run_protected(lp_handle h, const lp_workload_t* wl, void* ou
  * (hash stores: lookup; an absent key counts as failed), write the failed
  * GLOBAL rids in ascending order to failed_list[0 .. *d_n_failed) and the count
  * to *d_n_failed (device int64).  failed_cap must be >= R.  workspace must hold
- * lp_workspace_bytes bytes. */
+ * lp_workspace_bytes bytes (zero-filled before first use).  R <= 16384: one launch
+ * (the last CTA compacts); larger R: validate + a dependent compaction launch. */
 LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, const void* cksum, int64_t* failed_list,
                       int64_t failed_cap, int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 

@@ -186,7 +186,7 @@ int64_t dedupe_tiles(const lp::RegionGeom& g, int E) { return (g.M % E || g.N % 
 int64_t dedupe_capacity(const lp::RegionGeom& g) { return dedupe_tiles(g, 128); }
 
 struct WsLayout {
-  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, d_ntasks, total;
+  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, d_ntasks, ticket, total;
 };
 
 WsLayout ws_layout(const lp::RegionGeom& g) {
@@ -203,7 +203,8 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   w.d_ntiles = w.tile_list + al((size_t)T * 8);
   w.tasks = w.d_ntiles + 256;                       // paired recovery tasks: int32[max(R, T)]
   w.d_ntasks = w.tasks + al((size_t)(g.R > T ? g.R : T) * 4);
-  w.total = w.d_ntasks + 256;
+  w.ticket = w.d_ntasks + 256;                      // fused-compaction ticket (u32; zero-initialised, kept at 0)
+  w.total = w.ticket + 256;
   return w;
 }
 
@@ -462,8 +463,9 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
   uint8_t* flags = (uint8_t*)workspace + w.flags;
   uint32_t* counts = (uint32_t*)((uint8_t*)workspace + w.counts);
   cudaStream_t st = (cudaStream_t)stream;
+  uint32_t* ticket = (uint32_t*)((uint8_t*)workspace + w.ticket);
   cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st, counts,
-                                      failed_list, d_n_failed);
+                                      failed_list, d_n_failed, ticket);
   return e == cudaSuccess ? ok() : cuda_fail(e, "validate launch");
 }
 

@@ -25,12 +25,15 @@ struct HashInfo {
 
 // ---- lp_kernels.cu
 cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaStream_t st);
-// Validation + ordered compaction (2 launches): flags[R], per-CTA failure counts,
-// ascending failed list + device count.  records != null => records mode (no compare,
-// no compaction).
+// Validation + ordered compaction: flags[R], per-CTA failure counts, ascending failed
+// list + device count.  With a ticket (a zero-initialised u32 the kernel leaves at 0)
+// and R <= kFusedCompactMaxR, the last validate CTA to finish compacts the flags
+// itself (1 launch); otherwise a PDL scatter launch follows (2 launches).
+// records != null => records mode (no compare, no compaction).
+constexpr int64_t kFusedCompactMaxR = 16384;
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
                             uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
-                            int64_t* list, int64_t* d_n);
+                            int64_t* list, int64_t* d_n, uint32_t* ticket = nullptr);
 size_t validate_counts_bytes(const RegionGeom& g, int sm_count);
 cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* block_counts, int64_t* list,
                            int64_t* d_n, cudaStream_t st);

@@ -43,6 +43,59 @@ __device__ __forceinline__ CkRecord segment_reduce(const CkPartial<MASK>& p, int
   return r;
 }
 
+
+// Fused ordered compaction (a9) for small tables: every validate CTA bumps a ticket after
+// its flags and count are written; the last one to arrive (it sees ticket == grid - 1)
+// turns flags[0, R) into the ascending list of failed global rids + the device count, and
+// resets the ticket for the next call.  Ordering: bar.sync, then a gpu-scope fence and the
+// ticket RMW by thread 0 (cumulative: the CTA's flag stores are visible before the
+// ticket moves); the last CTA fences again before reading the flags (L2: ld.global.cg).
+__device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int64_t R, int64_t rid_offset,
+                                                      uint32_t* ticket, int64_t* list, int64_t* d_n) {
+  __shared__ int s_last;
+  __shared__ int s_warp[kValWarps];
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(ticket, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  const int per = (int)((R + kValThreads - 1) / kValThreads);   // <= 64 flags per thread
+  const int64_t i0 = (int64_t)threadIdx.x * per;
+  const int64_t i1 = i0 + per < R ? i0 + per : R;
+  int c = 0;
+  for (int64_t i = i0; i < i1; ++i) c += __ldcg(flags + i) ? 1 : 0;
+  // block exclusive scan of c
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  int x = c;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const int y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) s_warp[wid] = x;
+  __syncthreads();
+  int woff = 0, total = 0;
+#pragma unroll
+  for (int w = 0; w < kValWarps; ++w) {
+    const int v = s_warp[w];
+    if (w < wid) woff += v;
+    total += v;
+  }
+  int64_t pos = woff + x - c;
+  for (int64_t i = i0; i < i1 && c > 0; ++i) {
+    if (__ldcg(flags + i)) {
+      list[pos++] = rid_offset + i;
+      --c;
+    }
+  }
+  if (threadIdx.x == 0) {
+    *d_n = total;
+    *ticket = 0u;
+  }
+}
+
 // Validate (a8): a warp task is a strip of G = 2^g_log2 horizontally adjacent
 // regions (consecutive rids), LG = 32 / G lanes per region.  Lane li of a group
 // reads the 16-byte chunks li, li + LG, ... of its region in row-major order, so
@@ -62,7 +115,9 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
                                                                 const uint32_t* __restrict__ ck,
                                                                 int64_t rid_offset, uint8_t* __restrict__ flags,
                                                                 uint32_t* __restrict__ records, int64_t rpc,
-                                                                uint32_t* __restrict__ cta_counts) {
+                                                                uint32_t* __restrict__ cta_counts,
+                                                                uint32_t* __restrict__ ticket,
+                                                                int64_t* __restrict__ list, int64_t* __restrict__ d_n) {
   constexpr int S = selem_of(MASK);
   __shared__ uint32_t s_fail;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -131,6 +186,7 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
   if constexpr (MODE != 2) {
     __syncthreads();
     if (threadIdx.x == 0) cta_counts[blockIdx.x] = s_fail;
+    if (ticket) fused_compact_if_last(flags, R, rid_offset, ticket, list, d_n);
   }
 }
 
@@ -144,10 +200,11 @@ template <uint32_t MASK>
 cudaError_t validate_dispatch_mode(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
                                    int64_t ldc_bytes, int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2,
                                    const uint32_t* ck, int64_t rid_offset, uint8_t* flags, uint32_t* records,
-                                   uint32_t* counts) {
+                                   uint32_t* counts, uint32_t* ticket, int64_t* list, int64_t* d_n) {
 #define LP_VLAUNCH(MD)                                                                                    \
   validate_kernel<MASK, MD><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2,     \
-                                                            L.g_log2, ck, rid_offset, flags, records, L.rpc, counts)
+                                                            L.g_log2, ck, rid_offset, flags, records, L.rpc, counts, \
+                                                            ticket, list, d_n)
   if (mode == 0) LP_VLAUNCH(0);
   else if (mode == 1) LP_VLAUNCH(1);
   else if (mode == 3) LP_VLAUNCH(3);
@@ -534,13 +591,15 @@ size_t validate_counts_bytes(const RegionGeom& g, int sm_count) {
 
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
                             uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
-                            int64_t* list, int64_t* d_n) {
+                            int64_t* list, int64_t* d_n, uint32_t* ticket) {
   const int row_bytes = g.RN * g.es;
   const int cpr = row_bytes / 16;
   int cpr_log2 = 0;
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
   const int mode = records ? 2 : (hi.store == 0 ? 0 : (hi.store <= 2 ? 1 : 3));
   const ValLaunch L = plan_validate(g, sm_count);
+  const bool fuse = !records && ticket && g.R <= kFusedCompactMaxR && !getenv("LP_VALIDATE_NO_FUSE");
+  uint32_t* tk = fuse ? ticket : nullptr;
   const uint8_t* o = (const uint8_t*)out;
   const int64_t ldcb = g.ldc * g.es;
   cudaError_t e;
@@ -548,7 +607,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
 #define LP_VCASE(M)                                                                                          \
   case M:                                                                                                    \
     e = validate_dispatch_mode<M>(mode, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                \
-                                  (const uint32_t*)ck, g.rid_offset, flags, records, counts);               \
+                                  (const uint32_t*)ck, g.rid_offset, flags, records, counts, tk, list, d_n);\
     break;
     LP_VCASE(1)
     LP_VCASE(2)
@@ -561,7 +620,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
     default:
       return cudaErrorInvalidValue;
   }
-  if (e != cudaSuccess || records) return e;
+  if (e != cudaSuccess || records || fuse) return e;
   // ordered compaction: one pass, offsets from the validate kernel's per-CTA counts
   int sg, per;
   scatter_grid(L.grid.x, sg, per);

@@ -313,7 +313,7 @@ class LP:
         ck = torch.empty((ckb + 3) // 4, dtype=torch.int32, device=dev)
         failed = torch.empty(max(R, 1), dtype=torch.int64, device=dev)
         d_n = torch.zeros(1, dtype=torch.int64, device=dev)
-        ws = torch.empty(self.workspace_bytes(wl), dtype=torch.uint8, device=dev)
+        ws = torch.zeros(self.workspace_bytes(wl), dtype=torch.uint8, device=dev)   # zero-filled once (ABI contract)
         return out, ck, failed, d_n, ws
 
 

@@ -46,14 +46,15 @@ def _random_out(rng, M, N, dt):
     return rng.integers(0, 2**16, size=(M, N), dtype=np.uint64).astype(np.uint16)
 
 
-@pytest.fixture(params=["tma", "strip"])
+@pytest.fixture(params=["fused", "two_launch"])
 def kernel_path(request, monkeypatch):
-    """validate runs the TMA-staged kernel where the geometry fits a TMA box, else the strip kernel;
-    LP_VALIDATE_STRIP=1 forces the strip kernel so both paths are checked on every geometry."""
-    if request.param == "strip":
-        monkeypatch.setenv("LP_VALIDATE_STRIP", "1")
+    """Tables of R <= 16384 regions are compacted by the last validate CTA (one launch); larger ones by
+    a dependent scatter launch.  LP_VALIDATE_NO_FUSE=1 forces the two-launch form so both compaction
+    paths are checked on every geometry."""
+    if request.param == "two_launch":
+        monkeypatch.setenv("LP_VALIDATE_NO_FUSE", "1")
     else:
-        monkeypatch.delenv("LP_VALIDATE_STRIP", raising=False)
+        monkeypatch.delenv("LP_VALIDATE_NO_FUSE", raising=False)
     return request.param
 
 
@@ -91,10 +92,46 @@ def test_validate_geometries(geom, mask, kernel_path):
             ck_h[r * sel] ^= 0x10
     out.copy_(host_to_dev(out_h, dt))
     ck.copy_(torch.from_numpy(ck_h.view(np.int32)).cuda())
-    h.validate(wl, out, ck, failed, d_n, ws)
-    torch.cuda.synchronize()
-    n = int(d_n.item())
-    got = failed[:n].cpu().numpy()
-    exp = oracle_validate(out_h, ck_h, "array", RM, RN, h.mask)
-    assert np.array_equal(got, exp)
+    for _ in range(2):                              # the fused path's ticket is back at zero after each call
+        failed.fill_(-1)
+        h.validate(wl, out, ck, failed, d_n, ws)
+        torch.cuda.synchronize()
+        n = int(d_n.item())
+        got = failed[:n].cpu().numpy()
+        exp = oracle_validate(out_h, ck_h, "array", RM, RN, h.mask)
+        assert np.array_equal(got, exp)
     assert set(exp.tolist()) == set(bad.tolist())   # a single bit flip always changes MOD, XOR and Adler
+
+
+def test_validate_graph_replay_and_large_table():
+    """lp_validate captured in a CUDA graph and replayed (the fused ticket resets itself), and a table
+    above the fused limit (R = 65536: two-launch path) -- both against the oracle."""
+    for M, N, reg in [(2048, 2048, 32), (8192, 8192, 32)]:
+        rng = np.random.default_rng(M + reg)
+        out_h = _random_out(rng, M, N, "bf16")
+        h = lp.LP(reg, reg, cksum="mod|xor")
+        wl = lp.Workload.tmm(None, None, out_dtype="bf16", m=M, n=N, k=16)
+        out = host_to_dev(out_h, "bf16")
+        _, ck, failed, d_n, ws = h.alloc(wl)
+        R = h.num_regions(wl)
+        h.region_checksums(wl, out, ck)
+        ck_h = dev_to_host(ck).copy()
+        bad = np.sort(rng.choice(R, 37, replace=False))
+        ck_h[bad * 2 + 1] ^= 0x1
+        ck.copy_(torch.from_numpy(ck_h.view(np.int32)).cuda())
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream()
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s):
+            h.validate(wl, out, ck, failed, d_n, ws)          # warm-up outside capture
+        torch.cuda.current_stream().wait_stream(s)
+        with torch.cuda.graph(g):
+            h.validate(wl, out, ck, failed, d_n, ws)
+        for _ in range(3):
+            failed.fill_(-1)
+            d_n.fill_(-1)
+            g.replay()
+            torch.cuda.synchronize()
+            n = int(d_n.item())
+            assert n == 37 and np.array_equal(failed[:n].cpu().numpy(), bad), (M, reg)
