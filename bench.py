@@ -94,17 +94,19 @@ WORKLOADS = {
                           cksum="mod|xor", frac=0.05, store="array", weak=False),
 }
 
-def kernels_per_step(W, store):
+def kernels_per_step(W, store, R):
     """Our kernels launched by one step (init memset is not a kernel): protected body (+ hash header),
-    inject, 2 x (validate + ordered-compaction scatter), recovery (+ tile de-dup / pairing kernels)."""
+    inject, 2 x validate (+ the ordered-compaction scatter when R > 16384; smaller tables are compacted
+    by the last validate CTA), recovery (+ tile de-dup / pairing kernels)."""
     body = 1 + (1 if store != "array" else 0)
+    val = 1 if R <= 16384 else 2
     if W["kind"] == "tmm" and W["in_dt"] == "bf16" and W.get("body") != "simt":
         rec = 2 if W["region"] == 128 else 5          # pair builder + tcgen05; r32: mark, count, scatter too
     elif W["kind"] == "tmm" and W["in_dt"] == "f32" and W.get("body") != "simt":
         rec = 4                                        # tile mark, count, scatter, 3xTF32 list mode
     else:
         rec = 1
-    return body + 1 + 2 * 2 + rec
+    return body + 1 + 2 * val + rec
 
 
 def parse():
@@ -531,7 +533,7 @@ def run_ours(args):
 
     line = None
     if rank == 0:
-        launches = args.steps * kernels_per_step(W, W["store"])
+        launches = args.steps * kernels_per_step(W, W["store"], R)
         if W["kind"] == "spmv":
             nnz = float(rp_host[-1])
             sb = nnz * 8 + (M + 1) * 8 + N * 4 + M * 4
