@@ -61,11 +61,28 @@ __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int6
   __syncthreads();
   if (!s_last) return;
   __threadfence();
-  const int per = (int)((R + kValThreads - 1) / kValThreads);   // <= 64 flags per thread
-  const int64_t i0 = (int64_t)threadIdx.x * per;
-  const int64_t i1 = i0 + per < R ? i0 + per : R;
+  // thread t owns the 16-byte-aligned flag range [t * per, (t + 1) * per), per = 16 * nv <= 64:
+  // nv independent 16-B loads (flags are 0/1 bytes, so popc of a word counts its set flags)
+  constexpr int kMaxV = (int)(kFusedCompactMaxR / kValThreads / 16);
+  const int nv = (int)((R + kValThreads * 16 - 1) / (kValThreads * 16));
+  const int64_t i0 = (int64_t)threadIdx.x * nv * 16;
+  uint4 fv[kMaxV];
   int c = 0;
-  for (int64_t i = i0; i < i1; ++i) c += __ldcg(flags + i) ? 1 : 0;
+#pragma unroll
+  for (int u = 0; u < kMaxV; ++u) {
+    fv[u] = make_uint4(0u, 0u, 0u, 0u);
+    const int64_t b = i0 + u * 16;
+    if (u < nv && b < R) {
+      if (b + 16 <= R) {
+        fv[u] = __ldcg(reinterpret_cast<const uint4*>(flags + b));
+      } else {  // the table's ragged end
+        uint32_t w[4] = {0u, 0u, 0u, 0u};
+        for (int k = 0; k < (int)(R - b); ++k) w[k >> 2] |= (uint32_t)__ldcg(flags + b + k) << (8 * (k & 3));
+        fv[u] = make_uint4(w[0], w[1], w[2], w[3]);
+      }
+    }
+    c += __popc(fv[u].x) + __popc(fv[u].y) + __popc(fv[u].z) + __popc(fv[u].w);
+  }
   // block exclusive scan of c
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   int x = c;
@@ -84,10 +101,19 @@ __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int6
     total += v;
   }
   int64_t pos = woff + x - c;
-  for (int64_t i = i0; i < i1 && c > 0; ++i) {
-    if (__ldcg(flags + i)) {
-      list[pos++] = rid_offset + i;
-      --c;
+  if (c > 0) {
+#pragma unroll
+    for (int u = 0; u < kMaxV; ++u) {
+      const uint32_t w4[4] = {fv[u].x, fv[u].y, fv[u].z, fv[u].w};
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint32_t m = w4[q];
+        while (m) {  // set bytes in ascending order
+          const int bit = __ffs(m) - 1;
+          list[pos++] = rid_offset + i0 + u * 16 + q * 4 + (bit >> 3);
+          m &= m - 1;
+        }
+      }
     }
   }
   if (threadIdx.x == 0) {
