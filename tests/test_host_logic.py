@@ -125,3 +125,58 @@ def test_choose_regions_is_seeded_and_rounded():
     assert np.array_equal(a, lp.choose_regions(64, 0.05, 7))
     assert len(lp.choose_regions(65536, 0.01, 1)) == 655 and len(lp.choose_regions(65536, 0.10, 1)) == 6554
     assert len(lp.choose_regions(65536, 0.50, 1)) == 32768
+
+
+class _Fake:
+    """A fake device buffer: an address (aligned or not) and an element count -- argument checks run
+    before any device access, so these never reach a kernel."""
+
+    def __init__(self, addr, n=1 << 20):
+        self.addr, self.n = addr, n
+
+    def data_ptr(self):
+        return self.addr
+
+    def numel(self):
+        return self.n
+
+
+def _status(fn):
+    with pytest.raises(lp.LPError) as e:
+        fn()
+    return e.value.status
+
+
+def test_validate_recover_inject_argument_errors():
+    """The boundary's synchronous argument errors (liblp.h conventions): every one is refused before a
+    launch, on a machine with or without a GPU."""
+    h = lp.LP(32, 32, cksum="mod|xor")
+    wl = lp.Workload.tmm(None, None, out_dtype="f32", m=64, n=64, k=64)      # R = 4
+    A = _Fake(1 << 20)
+    assert _status(lambda: h.validate(wl, A, A, _Fake(1 << 20, 3), A, A, stream=0)) == lp.LP_ERR_INVALID_ARG   # cap < R
+    assert _status(lambda: h.validate(wl, None, A, A, A, A, stream=0)) == lp.LP_ERR_INVALID_ARG               # null out
+    assert _status(lambda: h.validate(wl, _Fake((1 << 20) + 4), A, A, A, A, stream=0)) == lp.LP_ERR_INVALID_ARG  # misaligned
+    assert _status(lambda: h.validate(wl, A, A, A, A, None, stream=0)) == lp.LP_ERR_INVALID_ARG               # no workspace
+    h0 = lp.LP(32, 32, cksum=0)
+    assert _status(lambda: h0.validate(wl, A, A, A, A, A, stream=0)) == lp.LP_ERR_STATE                       # unprotected
+    assert _status(lambda: h.recover(wl, A, A, None, A, stream=0)) == lp.LP_ERR_INVALID_ARG                   # no list
+    assert _status(lambda: h.inject(wl, A, A, A, _Fake(1 << 20, 5), stream=0)) == lp.LP_ERR_INVALID_ARG       # n > R
+    assert _status(lambda: h.inject(wl, A, A, None, _Fake(1 << 20, 2), mode="stale_region", stream=0)) == lp.LP_ERR_INVALID_ARG
+    assert _status(lambda: h.inject(wl, A, A, A, _Fake(1 << 20, 2), mode=9, stream=0)) == lp.LP_ERR_INVALID_ARG
+    empty = lp.Workload.tmm(None, None, out_dtype="f32", m=0, n=64, k=64)
+    assert _status(lambda: h.num_regions(empty)) == lp.LP_ERR_INVALID_ARG                          # m = 0
+    bad_ld = lp.Workload.tmm(None, None, out_dtype="f32", m=64, n=64, k=64)
+    bad_ld.ldc = 32
+    assert _status(lambda: h.num_regions(bad_ld)) == lp.LP_ERR_INVALID_ARG                         # ldc < n
+    assert "ldc" in lp.lib().lp_last_error().decode()
+
+
+def test_spmv_and_stencil_shape_errors():
+    hs = lp.LP(1, 1000, cksum="mod")                                        # not a power of two
+    wl = lp.Workload.spmv(None, None, None, None, m=4000)
+    assert _status(lambda: hs.num_regions(wl)) == lp.LP_ERR_UNSUPPORTED
+    h2 = lp.LP(2, 1024, cksum="mod")                                        # SPMV regions are 1 x region_n
+    assert _status(lambda: h2.num_regions(lp.Workload.spmv(None, None, None, None, m=4096))) == lp.LP_ERR_INVALID_ARG
+    h3 = lp.LP(1, 1024, cksum="mod")
+    assert _status(lambda: h3.num_regions(lp.Workload.spmv(None, None, None, None, m=1000))) == lp.LP_ERR_INVALID_ARG
+    assert h3.num_regions(lp.Workload.spmv(None, None, None, None, m=4096)) == 4
