@@ -50,6 +50,22 @@ struct CkPartial {
       w += (uint64_t)pos * bs + ws;
     }
   }
+  // four consecutive words (byte positions pos, pos + 4, pos + 8, pos + 12): the same sums as four
+  // add() calls, with Adler's position weights folded per 16 bytes -- sum_k (pos + 4k) * bs_k + ws_k
+  // = pos * sum_k bs_k + sum_k dp4a(word_k, {4k, 4k+1, 4k+2, 4k+3}) -- so one 64-bit multiply-add
+  // per vector instead of four.
+  __device__ __forceinline__ void add4(uint32_t x, uint32_t y, uint32_t z, uint32_t v, uint32_t pos) {
+    if constexpr ((MASK & kMod) != 0) mod += (x + y) + (z + v);
+    if constexpr ((MASK & kXor) != 0) xr ^= x ^ y ^ z ^ v;
+    if constexpr ((MASK & kAdler) != 0) {
+      const uint32_t bs = (uint32_t)__dp4a(x, 0x01010101u, __dp4a(y, 0x01010101u,
+                                           __dp4a(z, 0x01010101u, __dp4a(v, 0x01010101u, 0u))));
+      const uint32_t ws = (uint32_t)__dp4a(x, 0x03020100u, __dp4a(y, 0x07060504u,
+                                           __dp4a(z, 0x0B0A0908u, __dp4a(v, 0x0F0E0D0Cu, 0u))));
+      s += bs;
+      w += (uint64_t)pos * bs + ws;
+    }
+  }
   __device__ __forceinline__ void merge(const CkPartial& o) {
     mod += o.mod;
     xr ^= o.xr;

@@ -178,10 +178,7 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
         const int c = c0 + (u << lg_log2);
         if (live && c < chunks) {
           const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cmask) << 4) + 1);
-          part.add(v[u].x, pos);
-          part.add(v[u].y, pos + 4);
-          part.add(v[u].z, pos + 8);
-          part.add(v[u].w, pos + 12);
+          part.add4(v[u].x, v[u].y, v[u].z, v[u].w, pos);
         }
       }
     }

@@ -81,10 +81,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       for (int r = 0; r < kRowsW; ++r) {
         const uint4 w4 = ld_stream_u4(out + (int64_t)(i0 + r) * ldo + j);
         const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
-        vp.add(w4.x, pos);
-        vp.add(w4.y, pos + 4);
-        vp.add(w4.z, pos + 8);
-        vp.add(w4.w, pos + 12);
+        vp.add4(w4.x, w4.y, w4.z, w4.w, pos);
       }
       const CkRecord vr = warp_reduce<MASK>(vp);
       if (lane == 0) warp_rec[wid] = vr;
@@ -139,10 +136,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       __stcs(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
       if constexpr (MASK != 0) {
         const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
-        part.add(__float_as_uint(o.x), pos);
-        part.add(__float_as_uint(o.y), pos + 4);
-        part.add(__float_as_uint(o.z), pos + 8);
-        part.add(__float_as_uint(o.w), pos + 12);
+        part.add4(__float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w), pos);
       }
     }
     if constexpr (MASK != 0 && COMBINE == 1) {

@@ -186,7 +186,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
         const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
                                          : (uint32_t)(lane * 32 * ES + 1);
 #pragma unroll
-        for (int i = 0; i < 16; ++i) part.add(w[i], pos0 + 4 * i);
+        for (int i = 0; i < 4; ++i) part.add4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3], pos0 + 16 * i);
       }
     } else {
       uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
@@ -216,7 +216,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
         const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
                                          : (uint32_t)(lane * 32 * ES + 1);
 #pragma unroll
-        for (int i = 0; i < 32; ++i) part.add(r[i], pos0 + 4 * i);
+        for (int i = 0; i < 8; ++i) part.add4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3], pos0 + 16 * i);
       }
     }
     if constexpr (MASK != 0) {
