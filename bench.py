@@ -559,8 +559,9 @@ def run_ours(args):
             elif W["in_dt"] == "bf16":
                 kname = "tmm_tc2_kernel" if (M % 256 == 0 and N % 256 == 0) else "tmm_tc_kernel"
                 achieved = body_flops / (t_prot * 1e-3) / 1e12
-                # kernels of several ms run back to back under the 1 kW cap: sustained peak
-                long_kernel = t_prot > 2.0 and bf16_s is not None
+                # kernels of several ms run back to back under the 1 kW cap: sustained peak -- unless this
+                # run was not throttled (achieved above the sustained figure): then the burst peak
+                long_kernel = t_prot > 2.0 and bf16_s is not None and achieved <= bf16_s
                 pk = bf16_s if long_kernel else bf16
                 roof = {"bound": "tensor", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 1),
                         "peak": pk, "unit": "TFLOP/s", "frac": round(achieved / pk, 4),
@@ -570,9 +571,9 @@ def run_ours(args):
                         "traffic": ncu_traffic(kname, args.workload)}
             else:
                 kname = "tmm_tf32x3_kernel"
-                base = bf16_s if (t_prot > 2.0 and bf16_s is not None) else bf16
-                tf32_peak = base * (1.125 / 2.25)   # measured bf16 x nominal tf32/bf16 dense ratio (guide table)
                 achieved = 3.0 * body_flops / (t_prot * 1e-3) / 1e12   # 3 tf32 MMAs per fp32 MAC
+                base = bf16_s if (t_prot > 2.0 and bf16_s is not None and achieved <= 0.5 * bf16_s) else bf16
+                tf32_peak = base * (1.125 / 2.25)   # measured bf16 x nominal tf32/bf16 dense ratio (guide table)
                 roof = {"bound": "tensor", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 1),
                         "peak": round(tf32_peak, 1), "unit": "TFLOP/s (tf32 tensor work)",
                         "frac": round(achieved / tf32_peak, 4),
