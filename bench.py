@@ -525,6 +525,15 @@ def run_ours(args):
     if world > 1:
         dist.all_reduce(agg, op=dist.ReduceOp.MAX)
         dist.all_reduce(tot, op=dist.ReduceOp.SUM)
+    # per-rank spread (recovery imbalance follows each rank's injected count)
+    spread = None
+    if world > 1:
+        loc = torch.tensor([sum_vr / args.steps, t_prot, t_validate, float(k_local)], dtype=torch.float64, device=dev)
+        lo, hi = loc.clone(), loc.clone()
+        dist.all_reduce(lo, op=dist.ReduceOp.MIN)
+        dist.all_reduce(hi, op=dist.ReduceOp.MAX)
+        names = ["t_recovery_phase_ms", "t_protected_ms", "t_validate_ms", "n_failed"]
+        spread = {n: {"min": round(a, 4), "max": round(b, 4)} for n, a, b in zip(names, lo.tolist(), hi.tolist())}
     sum_vr, sum_step, t_e2e, t_prot_max, t_unprot_max = agg.tolist()
     bytes_vr_total = tot.item()
     value = bytes_vr_total * args.steps / (sum_vr * 1e-3) / 1e9
@@ -626,6 +635,7 @@ def run_ours(args):
             "t_recovery_phase_ms": round(sum_vr / args.steps, 4),
             "n_failed_per_step": n_failed,
             "n_failed_after_recover": n_after,
+            "per_rank": spread,
             "hash_collisions": hash_stats[0] if W["store"] != "array" else None,
             "hash_error": hash_stats[1] if W["store"] != "array" else None,
             "bytes_recovery_phase": int(bytes_vr_total),

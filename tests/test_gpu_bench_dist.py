@@ -29,6 +29,7 @@ def test_two_rank_bench_same_device():
     assert d["config"]["regions_per_rank"] * 2 == (d["config"]["M_global"] // 128) * (d["config"]["N"] // 128)
     assert d["n_failed_per_step"] == 2 * round(0.05 * d["config"]["regions_per_rank"])
     assert d["value"] > 0 and d["roofline"]["achieved"] > 0
+    assert d["per_rank"]["n_failed"]["min"] == d["per_rank"]["n_failed"]["max"] == round(0.05 * d["config"]["regions_per_rank"])
 
 
 def test_inject_skips_rids_of_other_shards():
