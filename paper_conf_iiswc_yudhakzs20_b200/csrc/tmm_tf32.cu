@@ -45,8 +45,10 @@ constexpr int kFTile = 16384;                     // one 128 x 32 fp32 operand t
 constexpr int kFRawBytes = 2 * kFTile;            // raw stage: [A (K-major)][B (MN-major, 4 x 32-col chunks)]
 constexpr int kFCvBytes = 4 * kFTile;             // converted stage: [A_hi][A_lo][B_hi][B_lo], all K-major SW128
 constexpr int kFSmemBytes = kFRawStages * kFRawBytes + kFCvStages * kFCvBytes + 512 + 1024;
-// K is accumulated in chunks of kFChunkKB x 32 = 512 in alternating TMEM accumulators;
-// the epilogue warps sum the chunk results into C with IEEE fp32 adds.  The tcgen05
+// K is accumulated in chunks of kFChunkKB x 32 = 512 in one TMEM accumulator (columns
+// 0..255); after each chunk the epilogue warps fold it into a TMEM-resident running
+// sum (columns 256..511) with IEEE fp32 adds and release the accumulator; C and the
+// LP record are stored from the running sum after the last chunk.  The tcgen05
 // fp32 accumulator is markedly less accurate than round-to-nearest (measured: error
 // std 2.0e-4 vs 8.6e-6 for exact products at K = 4096, growing ~K^1.5), so long K
 // runs are cut into short, freshly-zeroed chunks.  Measured at 8192^3 (normwise
@@ -249,14 +251,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
                                  ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
       int stage = 0;
       uint32_t phase = 0;
-      int acc = 0;
       uint32_t acc_phase = 0;
       for (int64_t t = pair; t < ntiles; t += npairs) {
         for (int kb0 = 0; kb0 < nkb; kb0 += chunk_kb) {
           const int kb1 = kb0 + chunk_kb < nkb ? kb0 + chunk_kb : nkb;
-          mbar_wait(&tempty[acc], acc_phase ^ 1);
+          mbar_wait(&tempty[0], acc_phase ^ 1);   // the epilogue has folded the previous chunk out of ACC
           tc_fence_after();
-          const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
+          const uint32_t d_tmem = tmem_base;       // ACC = TMEM columns [0, 256); SUM = [256, 512)
           for (int kb = kb0; kb < kb1; ++kb) {
             mbar_wait(&cv_full[stage], phase);
             tc_fence_after();
@@ -277,49 +278,61 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
               phase ^= 1;
             }
           }
-          tc_commit_pair(&tfull[acc]);  // this chunk's partial sum is ready
-          if (++acc == 2) {
-            acc = 0;
-            acc_phase ^= 1;
-          }
+          tc_commit_pair(&tfull[0]);  // this chunk's partial sum is ready
+          acc_phase ^= 1;
         }
       }
     }
   } else {
     // ===================== epilogue (warps 2..5) =====================
     const int wq = warp & 3;
-    int acc = 0;
     uint32_t acc_phase = 0;
-    for (int64_t t = pair; t < ntiles; t += npairs) {
+    int tile_iter = 0;
+    for (int64_t t = pair; t < ntiles; t += npairs, ++tile_iter) {
       int64_t mb, nb;
       tiles.coords(t, mb, nb);
       const int64_t m128 = mb * 2 + rank;
+      CkRecord* srec_acc = srec + (tile_iter & 1) * 2 * 4;   // per-tile double buffer of the warp partials
+      const uint32_t t_acc = tmem_base + ((uint32_t)(wq * 32) << 16);
+      const uint32_t t_sum = t_acc + (uint32_t)BN;
       for (int kb0 = 0; kb0 < nkb; kb0 += chunk_kb) {
         const bool first = kb0 == 0, last = kb0 + chunk_kb >= nkb;
-        mbar_wait(&tfull[acc], acc_phase);
+        mbar_wait(&tfull[0], acc_phase);
         tc_fence_after();
-        const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
-        CkRecord* srec_acc = srec + acc * 2 * 4;
-        // C (+)= chunk; the LP checksum is folded over the final words on the last chunk only
-        epi_store<float, MASK, REG, BN, STORE>(t_row, C, ldc, m128, nb * BN, wq, lane, srec_acc, ck, tiles.Qr,
-                                               tiles.rid_offset, !first, last);
+        // SUM (+)= ACC in TMEM: IEEE fp32 adds in chunk order (Reading R22), then ACC goes back to the MMA
+#pragma unroll 1
+        for (int g = 0; g < BN / 32; ++g) {
+          uint32_t r[32];
+          LP_TMEM_LD32(t_acc + g * 32, r);
+          if (!first) {
+            uint32_t q[32];
+            LP_TMEM_LD32(t_sum + g * 32, q);
+            tc_wait_ld();
+#pragma unroll
+            for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__fadd_rn(__uint_as_float(q[i]), __uint_as_float(r[i])));
+          } else {
+            tc_wait_ld();
+          }
+          LP_TMEM_ST32(t_sum + g * 32, r);
+        }
+        tc_wait_st();
         tc_fence_before();
         __syncwarp();
         if (lane == 0) {
           if (rank == 0)
-            mbar_arrive(&tempty[acc]);
+            mbar_arrive(&tempty[0]);
           else
-            mbar_arrive_remote(mapa_rank0(&tempty[acc]));
+            mbar_arrive_remote(mapa_rank0(&tempty[0]));
         }
-        if constexpr (MASK != 0 && REG == 128) {
-          if (last)
+        if (last) {
+          // C = SUM; the LP checksum is folded over exactly the stored words
+          epi_store<float, MASK, REG, BN, STORE>(t_sum, C, ldc, m128, nb * BN, wq, lane, srec_acc, ck, tiles.Qr,
+                                                 tiles.rid_offset, false, true);
+          if constexpr (MASK != 0 && REG == 128)
             epi_finish_128<float, MASK, BN, STORE>(warp, lane, srec_acc, ck, m128, nb * BN, tiles.Qr,
                                                    tiles.rid_offset);
         }
-        if (++acc == 2) {
-          acc = 0;
-          acc_phase ^= 1;
-        }
+        acc_phase ^= 1;
       }
     }
   }
