@@ -19,7 +19,8 @@
 //            measured), fence.proxy.async, then arrive on the leader's barrier
 //   warp 1   (leader) MMA issuer: 3 x tcgen05.mma.cta_group::2.kind::tf32 per
 //            8-wide K step from a 2-deep converted ring, commits multicast
-//   warps 2-5 epilogue: identical LP epilogue to the bf16 kernels (fp32 words).
+//   warps 2-5 epilogue: per K chunk SUM += ACC in TMEM (tcgen05.ld / fadd / tcgen05.st),
+//            then on the last chunk the LP epilogue of the bf16 kernels from SUM (fp32 words).
 // Recovery re-runs this same kernel on a de-duplicated list of 256x256 tiles, so
 // the recomputed bits equal the golden ones (same instruction sequence).
 #include <cuda.h>
