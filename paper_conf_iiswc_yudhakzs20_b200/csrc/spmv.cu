@@ -46,7 +46,7 @@ constexpr int kSpWarps = kSpThreads / 32;
 #define LP_SPMV_PT 8
 #endif
 #ifndef LP_SPMV_MINB
-#define LP_SPMV_MINB 4
+#define LP_SPMV_MINB 5
 #endif
 constexpr int kPerThread = LP_SPMV_PT;               // nnz per thread per chunk (kPerThread / 4 uint4)
 constexpr int kVec = kPerThread / 4;
