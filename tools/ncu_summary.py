@@ -17,7 +17,7 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__warps_active.avg.pct_of_peak_sustained_active", "launch__grid_size", "sm__cycles_elapsed.avg.per_second",
         "sm__pipe_alu_cycles_active.avg.pct_of_peak_sustained_active"]
 SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "us": 1e-6, "ms": 1e-3, "ns": 1e-9, "s": 1}
-WL = {"tmm": "tmm8192_bf16", "stencil": "stencil32768", "spmv": "spmv4m"}
+WL = {"tmm": "tmm8192_bf16", "stencil": "stencil32768", "spmv": "spmv4m", "tf32": "tmm8192_f32"}
 
 
 def raw(path):
@@ -57,7 +57,7 @@ def main(rdir):
         rd, wr = num(d["dram__bytes_read.sum"]), num(d["dram__bytes_write.sum"])
         out.append(f"| dram read+write per launch | {rd + wr:.4g} B |")
         out.append("")
-        wl = WL["stencil" if "stencil" in tag else ("spmv" if "spmv" in tag else "tmm")]
+        wl = WL["stencil" if "stencil" in tag else ("spmv" if "spmv" in tag else ("tf32" if "tf32" in tag else "tmm"))]
         kern = name.split("<")[0].split("::")[-1].replace("void ", "").strip()
         if "recover" in tag:
             kern += "_list_mode"
