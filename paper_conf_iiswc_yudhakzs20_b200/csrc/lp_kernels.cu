@@ -351,12 +351,29 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
   const int64_t lo = (int64_t)first * chunk;
   int64_t hi = (int64_t)(first + per_block) * chunk;
   if (hi > R) hi = R;
-  for (int64_t i0 = lo; i0 < hi; i0 += kCompactThreads) {
-    const int64_t i = i0 + threadIdx.x;
-    const int f = (i < hi && flags[i]) ? 1 : 0;
+  // 16 flags per thread per pass (two 8-byte loads: lo is a multiple of 8 because every validate
+  // CTA owns a multiple of 8 regions), one block scan per 4096 flags, emitted from registers
+  for (int64_t i0 = lo; i0 < hi; i0 += (int64_t)kCompactThreads * 16) {
+    const int64_t st = i0 + (int64_t)threadIdx.x * 16;
+    uint32_t w[4] = {0u, 0u, 0u, 0u};
+    if (st + 16 <= hi) {
+      const uint2 a = *reinterpret_cast<const uint2*>(flags + st);
+      const uint2 b = *reinterpret_cast<const uint2*>(flags + st + 8);
+      w[0] = a.x; w[1] = a.y; w[2] = b.x; w[3] = b.y;
+    } else {
+      for (int k = 0; k < 16 && st + k < hi; ++k) w[k >> 2] |= (uint32_t)flags[st + k] << (8 * (k & 3));
+    }
+    const int c = __popc(w[0]) + __popc(w[1]) + __popc(w[2]) + __popc(w[3]);   // flags are 0/1 bytes
     int total;
-    const int off = block_exclusive_scan(f, warp_s, &total);
-    if (f) list[base + off] = rid_offset + i;
+    long long pos = base + block_exclusive_scan(c, warp_s, &total);
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      uint32_t m = w[q];
+      while (m) {  // set bytes in ascending order
+        list[pos++] = rid_offset + st + q * 4 + ((__ffs(m) - 1) >> 3);
+        m &= m - 1;
+      }
+    }
     base += total;
     __syncthreads();  // warp_s reuse
   }
