@@ -51,6 +51,35 @@ def stencil(store="array"):
     print("ok stencil", store, flush=True)
 
 
+def spmv():
+    from lpsynth import csr, gen
+    rows, RN = 8192, 1024
+    rp = csr.row_ptr(5, rows)
+    cols = csr.columns(6, rp, rows)
+    vals = gen.values_f32(7, 1, int(rp[-1]), "int5")[0]
+    x = gen.values_f32(8, 1, rows, "int5")[0]
+    h = lp.LP(1, RN, cksum="mod|xor")
+    wl = lp.Workload.spmv(torch.from_numpy(vals).cuda(), torch.from_numpy(x).cuda(), torch.from_numpy(rp).cuda(),
+                          torch.from_numpy(cols).cuda())
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    cycle(h, wl, out, ck, failed, d_n, ws, torch.zeros_like(out))
+    print("ok spmv", flush=True)
+
+
+def validate_large_table():
+    """R = 65536 > 16384: validate + the separate ordered-compaction launch."""
+    out = torch.randn(2048, 4096, device="cuda").to(torch.bfloat16)
+    h = lp.LP(32, 32, cksum="mod|xor")
+    wl = lp.Workload.tmm(None, None, out_dtype="bf16", m=2048, n=4096, k=16)
+    _, ck, failed, d_n, ws = h.alloc(wl)
+    h.region_checksums(wl, out, ck)
+    ck[1::97] ^= 1
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) > 0
+    print("ok validate R =", h.num_regions(wl), flush=True)
+
+
 tmm(256, 256, 128, 32, "f32", "f32", "simt")
 tmm(256, 256, 128, 32, "i32", "i32", "simt", store="cuckoo", shuffle=False)
 tmm(256, 512, 128, 128, "bf16", "bf16", "tcgen05")
@@ -58,3 +87,6 @@ tmm(256, 512, 128, 32, "bf16", "f32", "tcgen05", store="quad_cas")
 tmm(256, 512, 64, 128, "f32", "f32", "tcgen05", store="cuckoo")
 stencil()
 stencil("quad_cas")
+tmm(256, 512, 1024, 128, "f32", "f32", "tcgen05")     # 3xTF32: two 512-K chunks through the TMEM running sum
+spmv()
+validate_large_table()
