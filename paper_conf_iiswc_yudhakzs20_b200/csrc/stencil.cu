@@ -18,11 +18,13 @@
 //
 // LP epilogue: each lane folds the exact stored words into its checksum
 // partials (L192) and the warp reduces them with redux.sync (Listing 4).  The
-// 8 warps' partials are combined WITHOUT a CTA barrier: lane 0 of each warp
-// folds its partial into shared accumulators with shared-memory atomics and
-// the last warp to arrive finalises and stores the record at table[rid]
-// (L349).  (A Listing-3 style barrier combine, kept for list-mode recovery where
-// a CTA handles several regions, costs 29% here: measured.)
+// 8 warps' partials are combined behind a SPLIT barrier: every warp parks its
+// partial in shared memory and arrives (bar.arrive) on a named barrier; only
+// warp 0 waits (bar.sync), combines (Listing 3) and stores the record at
+// table[rid] (L349).  The unprotected twin keeps the same barrier (it also
+// speeds the plain kernel up), so the LP overhead compares like with like.
+// (List-mode recovery, where a CTA handles several regions, uses the barrier
+// combine; measured A/Bs in DESIGN.md.)
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -33,6 +35,9 @@ namespace lp {
 namespace {
 
 constexpr int kRM = 128, kRN = 128;
+#ifndef LP_STENCIL_TWIN_BAR
+#define LP_STENCIL_TWIN_BAR 1
+#endif
 
 __device__ __forceinline__ float st5(float c, float u, float d, float l, float r) {
   const float s = __fadd_rn(__fadd_rn(__fadd_rn(u, d), l), r);
@@ -60,12 +65,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
                                                               const int64_t* __restrict__ d_n) {
   constexpr int kRowsW = 16;
   __shared__ CkRecord warp_rec[8];
-  __shared__ uint32_t s_acc[5];  // COMBINE == 1: mod, xor, adler s, adler w, arrivals
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  if constexpr (COMBINE == 1) {
-    if (threadIdx.x < 5) s_acc[threadIdx.x] = 0u;
-    __syncthreads();
-  }
   __shared__ int s_bad;
   const int64_t ntiles = (list && COMBINE != 2) ? *d_n : R;
   for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
@@ -140,27 +140,29 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       }
     }
     if constexpr (MASK != 0 && COMBINE == 1) {
-      // barrier-free combine (one region per CTA): warp partials fold into the
-      // shared accumulators with shared-memory atomics; the last warp to arrive
-      // finalises and stores the record.
+      // split-barrier combine (one region per CTA): every warp parks its partial in shared memory and
+      // ARRIVES on named barrier 2 without waiting; only warp 0 waits (bar.sync) and then combines the
+      // 8 partials (Listing 3) and stores the record.  No shared state needs initialising, and 7 of the
+      // 8 warps retire as soon as their stores are issued.
       const CkRecord wr = warp_reduce<MASK>(part);
-      if (lane == 0) {
-        if constexpr ((MASK & kMod) != 0) atomicAdd(&s_acc[0], wr.mod);
-        if constexpr ((MASK & kXor) != 0) atomicXor(&s_acc[1], wr.xr);
-        if constexpr ((MASK & kAdler) != 0) {
-          atomicAdd(&s_acc[2], wr.s);
-          atomicAdd(&s_acc[3], wr.wmod);
-        }
-        __threadfence_block();
-        if (atomicAdd(&s_acc[4], 1u) == 7u) {
-          __threadfence_block();
-          const CkRecord rr{atomicAdd(&s_acc[0], 0u), atomicAdd(&s_acc[1], 0u), atomicAdd(&s_acc[2], 0u),
-                            atomicAdd(&s_acc[3], 0u)};
+      if (lane == 0) warp_rec[wid] = wr;
+      if (wid != 0) {
+        asm volatile("bar.arrive 2, 256;" ::: "memory");
+      } else {
+        asm volatile("bar.sync 2, 256;" ::: "memory");
+        if (lane == 0) {
+          CkRecord rr = warp_rec[0];
+#pragma unroll
+          for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
           uint32_t words[3];
           record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
           store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
         }
       }
+    } else if constexpr (MASK == 0 && COMBINE == 1 && LP_STENCIL_TWIN_BAR) {
+      // the unprotected twin keeps the same split barrier, so the LP overhead compares like with like
+      if (wid != 0) asm volatile("bar.arrive 2, 256;" ::: "memory");
+      else asm volatile("bar.sync 2, 256;" ::: "memory");
     } else if constexpr (MASK != 0) {
       const CkRecord wr = warp_reduce<MASK>(part);
       __syncthreads();  // warp_rec may still be read by the check phase (COMBINE == 2)
