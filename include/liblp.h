@@ -129,6 +129,8 @@ typedef enum {
   LP_FLAG_TC_1CTA = 1u,    /* tcgen05 body: use the 1-SM 128x256 kernel even where the 2-SM CTA-pair kernel applies */
   LP_FLAG_NO_SHUFFLE = 2u, /* SIMT TMM and SPMV bodies: sequential shared-memory reduction instead of warp reduction
                               (the paper's "without parallel reduction" ablation, L343, Table IV) */
+  LP_FLAG_NO_FUSED_COMPACT = 8u, /* lp_validate: always compact the failed flags in a separate (PDL) launch instead
+                                    of in the last validate CTA for tables of <= 16384 regions (A/B switch) */
   LP_FLAG_NO_PAIRING = 4u  /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
                               failed tiles of the same row band into 128x256 tasks (A/B switch) */
 } lp_config_flags;

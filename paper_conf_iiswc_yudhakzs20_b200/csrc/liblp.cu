@@ -363,7 +363,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
     return fail(LP_ERR_UNSUPPORTED, "hash stores (the ablation) are built for MOD and MOD|XOR records");
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
-  if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING))
+  if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING | LP_FLAG_NO_FUSED_COMPACT))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");
@@ -463,7 +463,7 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
   uint8_t* flags = (uint8_t*)workspace + w.flags;
   uint32_t* counts = (uint32_t*)((uint8_t*)workspace + w.counts);
   cudaStream_t st = (cudaStream_t)stream;
-  uint32_t* ticket = (uint32_t*)((uint8_t*)workspace + w.ticket);
+  uint32_t* ticket = (h->cfg.flags & LP_FLAG_NO_FUSED_COMPACT) ? nullptr : (uint32_t*)((uint8_t*)workspace + w.ticket);
   cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st, counts,
                                       failed_list, d_n_failed, ticket);
   return e == cudaSuccess ? ok() : cuda_fail(e, "validate launch");

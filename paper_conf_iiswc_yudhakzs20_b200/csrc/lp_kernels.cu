@@ -605,10 +605,12 @@ static ValLaunch plan_validate(const RegionGeom& g, int sm_count) {
   int gl = 0;
   while ((2 << gl) * cpr <= 32) ++gl;                  // G * cpr <= 32
   while (gl > 0 && (g.R >> gl) < kValMinWarps) --gl;
-  if (const char* e = getenv("LP_VALIDATE_G")) {
-    const int v = atoi(e);
-    if (v >= 0 && v <= 5) gl = v;
-  }
+  static const int g_override = [] {  // LP_VALIDATE_G=<log2>: A/B override, read once per process
+    const char* e = getenv("LP_VALIDATE_G");
+    const int v = e ? atoi(e) : -1;
+    return (v >= 0 && v <= 5) ? v : -1;
+  }();
+  if (g_override >= 0) gl = g_override;
   L.g_log2 = gl;
   const int64_t unit = (int64_t)kValWarps << gl;
   int64_t max_ctas = (int64_t)sm_count * 16;
@@ -638,7 +640,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
   const int mode = records ? 2 : (hi.store == 0 ? 0 : (hi.store <= 2 ? 1 : 3));
   const ValLaunch L = plan_validate(g, sm_count);
-  const bool fuse = !records && ticket && g.R <= kFusedCompactMaxR && !getenv("LP_VALIDATE_NO_FUSE");
+  const bool fuse = !records && ticket && g.R <= kFusedCompactMaxR;
   uint32_t* tk = fuse ? ticket : nullptr;
   const uint8_t* o = (const uint8_t*)out;
   const int64_t ldcb = g.ldc * g.es;

@@ -47,14 +47,10 @@ def _random_out(rng, M, N, dt):
 
 
 @pytest.fixture(params=["fused", "two_launch"])
-def kernel_path(request, monkeypatch):
+def kernel_path(request):
     """Tables of R <= 16384 regions are compacted by the last validate CTA (one launch); larger ones by
-    a dependent scatter launch.  LP_VALIDATE_NO_FUSE=1 forces the two-launch form so both compaction
-    paths are checked on every geometry."""
-    if request.param == "two_launch":
-        monkeypatch.setenv("LP_VALIDATE_NO_FUSE", "1")
-    else:
-        monkeypatch.delenv("LP_VALIDATE_NO_FUSE", raising=False)
+    a dependent scatter launch.  LP(fused_compact=False) (LP_FLAG_NO_FUSED_COMPACT) forces the two-launch
+    form so both compaction paths are checked on every geometry."""
     return request.param
 
 
@@ -64,7 +60,7 @@ def test_validate_geometries(geom, mask, kernel_path):
     M, N, RM, RN, dt = geom
     rng = np.random.default_rng(M * 7919 + N + RM)
     out_h = _random_out(rng, M, N, dt)
-    h = lp.LP(RM, RN, cksum=mask)
+    h = lp.LP(RM, RN, cksum=mask, fused_compact=(kernel_path == "fused"))
     wl = lp.Workload.tmm(None, None, out_dtype=dt, m=M, n=N, k=16)
     out = host_to_dev(out_h, dt)
     _, ck, failed, d_n, ws = h.alloc(wl)
