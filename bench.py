@@ -127,6 +127,8 @@ def parse():
     ap.add_argument("--no-shuffle", action="store_true", help="SIMT body: sequential reduction ablation (L343)")
     ap.add_argument("--no-pairing", action="store_true",
                     help="tcgen05 recovery: one 128x128 tile per failed tile (no same-row pairing) -- A/B switch")
+    ap.add_argument("--recover-tile128", action="store_true",
+                    help="tcgen05 recovery of 32x32 regions: 128x128 tiles instead of 128x64 slices -- A/B switch")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch the step eagerly instead of replaying captured CUDA graphs")
     return ap.parse_args()
@@ -284,7 +286,7 @@ def run_ours(args):
         wl = lp.Workload.stencil(a)
         body_flops = 0.0
     h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
-              shuffle=not args.no_shuffle, pairing=not args.no_pairing)
+              shuffle=not args.no_shuffle, pairing=not args.no_pairing, recover_slices=not args.recover_tile128)
     h0 = lp.LP(RM, RN, cksum=0, device=local, body=W.get("body", "auto"))   # unprotected twin (overhead denominator)
     out, ck, failed, d_n, ws = h.alloc(wl)
     out_twin = torch.empty_like(out)
@@ -617,7 +619,7 @@ def run_ours(args):
             "config": {"workload": args.workload, "M_global": gM, "N": N, "K": K, "region": [RM, RN],
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
-                       "recovery": "one 128x128 tile per failed tile" if args.no_pairing else "same-row failed tiles paired into 128x256 tasks (when > #SM)",
+                       "recovery": recovery_desc(args, RM),
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write, then 2x L2 read of another buffer: clean lines) before every recovery phase and every isolated kernel rep",
                        "launch": "CUDA graph replay per step segment" if args.graph else "eager"},
@@ -820,6 +822,14 @@ def run_reference(args):
                                        f"of regions"},
             "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
+
+
+def recovery_desc(args, RM):
+    if args.no_pairing:
+        return "one 128x128 tile per failed tile"
+    if RM == 32 and not args.recover_tile128:
+        return "failed 32x32 regions de-duplicated into 128x64 slices, same-row slices paired into 128x128 tasks (when > #SM)"
+    return "same-row failed tiles paired into 128x256 tasks (when > #SM)"
 
 
 def main():

@@ -131,8 +131,11 @@ typedef enum {
                               (the paper's "without parallel reduction" ablation, L343, Table IV) */
   LP_FLAG_NO_FUSED_COMPACT = 8u, /* lp_validate: always compact the failed flags in a separate (PDL) launch instead
                                     of in the last validate CTA for tables of <= 16384 regions (A/B switch) */
-  LP_FLAG_NO_PAIRING = 4u  /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
+  LP_FLAG_NO_PAIRING = 4u, /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
                               failed tiles of the same row band into 128x256 tasks (A/B switch) */
+  LP_FLAG_RECOVER_TILE128 = 16u /* tcgen05 bf16 recovery of 32x32 regions: de-duplicate failed regions into 128x128
+                                   tiles (paired into 128x256 tasks) instead of 128x64 slices paired into 128x128
+                                   tasks (A/B switch; both re-execute every failed region, L51-57) */
 } lp_config_flags;
 
 typedef struct {

@@ -388,13 +388,13 @@ static void scatter_grid(int64_t nblocks, int& grid, int& per_block) {
 
 // ---------------------------------------------------------------------------
 __global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t* __restrict__ d_n,
-                                 int64_t rid_offset, int64_t Q, int64_t tiles_per_row, int per,
+                                 int64_t rid_offset, int64_t Q, int64_t tiles_per_row, int per_m, int per_n,
                                  uint8_t* __restrict__ tile_flags) {
   const int64_t n = *d_n;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t rid = list[i] - rid_offset;
     const int64_t p = rid / Q, q = rid - p * Q;
-    tile_flags[(p / per) * tiles_per_row + q / per] = 1;  // idempotent plain store
+    tile_flags[(p / per_m) * tiles_per_row + q / per_n] = 1;  // idempotent plain store
   }
 }
 
@@ -718,14 +718,13 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
   return cudaGetLastError();
 }
 
-cudaError_t launch_tiles_of_failed(const RegionGeom& g, int E, const int64_t* list, const int64_t* d_n,
+cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const int64_t* list, const int64_t* d_n,
                                    uint8_t* tile_flags, int64_t T, uint32_t* block_counts, int64_t* tile_list,
                                    int64_t* d_ntiles, cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(tile_flags, 0, (size_t)T, st);
   if (e != cudaSuccess) return e;
-  const int per = E / g.RM;
   tile_mark_kernel<<<(unsigned)(g.R < 148 * 4 * 256 ? (g.R + 255) / 256 : 148 * 4), 256, 0, st>>>(
-      list, d_n, g.rid_offset, g.Q, g.N / E, per, tile_flags);
+      list, d_n, g.rid_offset, g.Q, g.N / EN, EM / g.RM, EN / g.RN, tile_flags);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   RegionGeom tg = g;

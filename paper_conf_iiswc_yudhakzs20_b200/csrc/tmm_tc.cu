@@ -123,16 +123,24 @@ __global__ void __launch_bounds__(kThreads, 1)
         src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
         const int m0 = (int)(mb * kBM);
         // B is staged as 64-column chunks: 0,1 from the low half's panel, 2,3 from the high half's
-        const uint32_t bytes = Cfg::kABytes + (has_hi ? 4 : 2) * (kBK * 128);
+        // (128x64 slice tasks: chunk 0 = the low slice, chunk 1 = the high slice if paired)
+        const bool sl = BN == 128 && src.slice64;
+        const uint32_t bytes = Cfg::kABytes + (sl ? (has_hi ? 2 : 1) : (has_hi ? 4 : 2)) * (kBK * 128);
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], bytes);
           tma_load_2d(&tmap_a, &full[stage], sA + stage * Cfg::kABytes, kb * kBK, m0);
+          if (sl) {
+            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes, (int)n_lo, kb * kBK);
+            if (has_hi)
+              tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + kBK * 128, (int)n_hi, kb * kBK);
+          } else {
 #pragma unroll
-          for (int c = 0; c < BN / 64; ++c) {
-            if (c >= 2 && !has_hi) break;
-            const int64_t col = (c < 2 ? n_lo : n_hi) + (c & 1) * 64;
-            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), (int)col, kb * kBK);
+            for (int c = 0; c < BN / 64; ++c) {
+              if (c >= 2 && !has_hi) break;
+              const int64_t col = (c < 2 ? n_lo : n_hi) + (c & 1) * 64;
+              tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), (int)col, kb * kBK);
+            }
           }
           if (++stage == S) {
             stage = 0;
@@ -152,8 +160,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         int64_t mb, n_lo, n_hi;
         bool has_hi;
         src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
-        // N = 256 when both halves are live, else N = 128 into the low half
-        const uint32_t idesc = (BN == 256 && has_hi) ? instr_desc<256>() : instr_desc<128>();
+        // N = 256 when both halves are live, else N = 128 into the low half;
+        // slice tasks: N = 128 for a pair, N = 64 for a lone slice
+        const uint32_t idesc = (BN == 256 && has_hi) ? instr_desc<256>()
+                               : (BN == 128 && src.slice64 && !has_hi) ? instr_desc<64>()
+                                                                       : instr_desc<128>();
         mbar_wait(&tempty[acc], acc_phase ^ 1);  // epilogue drained this accumulator
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -197,8 +208,21 @@ __global__ void __launch_bounds__(kThreads, 1)
       tc_fence_after();
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
       CkRecord* srec_acc = srec + acc * (BN / 128) * 4;
-      epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
-                                             src.rid_offset);
+      bool sliced = false;
+      if constexpr (REG == 32 && BN == 128) {
+        if (src.slice64) {
+          // accumulator columns [0,64) -> the low slice, [64,128) -> the high slice (32x32 records per chunk)
+          epi_store<OutT, MASK, REG, 64, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
+                                                src.rid_offset);
+          if (has_hi)
+            epi_store<OutT, MASK, REG, 64, STORE>(t_row + 64, C, ldc, mb, n_hi, wq, lane, srec_acc, ck, src.Qr,
+                                                  src.rid_offset);
+          sliced = true;
+        }
+      }
+      if (!sliced)
+        epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
+                                               src.rid_offset);
       if (BN == 256 && has_hi)
         epi_store<OutT, MASK, REG, 128, STORE>(t_row + 128, C, ldc, mb, n_hi, wq, lane, srec_acc + 4, ck, src.Qr,
                                                src.rid_offset);
@@ -418,6 +442,8 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   src.tasks = a.list ? a.tasks : nullptr;
   src.d_ntasks = a.d_ntasks;
   src.n128 = a.N / 128;
+  src.slice64 = a.slice64;
+  src.n64 = a.N / 64;
   const int64_t R = (a.M / REG) * (a.N / REG);
   int64_t grid = a.list ? (R < a.sm_count ? R : a.sm_count) : src.num_m * src.num_n;
   if (grid > a.sm_count) grid = a.sm_count;
@@ -504,7 +530,7 @@ cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
   // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
   // 16 32x32 regions of a de-duplicated tile; paired tasks (two such tiles of one
   // row band) run on the BN = 256 kernel with B gathered from two column panels
-  const bool bn256 = a.list ? (a.tasks != nullptr) : (a.N % 256 == 0);
+  const bool bn256 = a.list ? (a.tasks != nullptr && !a.slice64) : (a.N % 256 == 0);
   return bn256 ? launch_cfg<OutT, REG, 256>(a, st, why) : launch_cfg<OutT, REG, 128>(a, st, why);
 }
 

@@ -18,8 +18,10 @@ pytestmark = pytest.mark.gpu
 
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
-              store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True, pairing=True):
-    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle, pairing=pairing)
+              store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True, pairing=True,
+              recover_slices=True):
+    h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle, pairing=pairing,
+              recover_slices=recover_slices)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -162,6 +164,19 @@ def test_tc_paired_recovery(pairing, reg, N, frac, out_dt):
     _, nf = run_cycle(2048, N, 256, reg, reg, "bf16", out_dt, "uniform", "mod|xor", "tcgen05", mode="stale_words",
                       frac=frac, pairing=pairing)
     assert nf > 148
+
+
+@pytest.mark.parametrize("slices", [True, False])
+@pytest.mark.parametrize("N,frac", [(2048, 0.01), (2176, 0.1), (2048, 0.5), (1152, 1.0)])
+@pytest.mark.parametrize("out_dt", ["bf16", "f32"])
+def test_tc_slice_recovery(slices, N, frac, out_dt):
+    """32x32 regions recovered as de-duplicated 128x64 slices (two slices of a row band per N = 128 tcgen05
+    task, B gathered from two 64-column panels; a lone slice runs N = 64) vs the 128x128-tile path
+    (LP_FLAG_RECOVER_TILE128).  frac 0.01: fewer slices than SMs (no pairing); N = 2176: 34 slice columns
+    per row band, odd runs; frac 1.0: every region.  Recovered bytes and records must equal the golden run."""
+    _, nf = run_cycle(2048, N, 256, 32, 32, "bf16", out_dt, "uniform", "mod|xor", "tcgen05", mode="stale_words",
+                      frac=frac, recover_slices=slices)
+    assert nf > 0
 
 
 @pytest.mark.parametrize("store", ["quad_cas", "cuckoo"])
