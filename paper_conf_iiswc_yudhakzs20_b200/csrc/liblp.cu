@@ -316,8 +316,8 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     const int E = tc_ok ? 128 : 256;  // tile edge of the list-mode kernel
     const bool need_dedupe = tf_ok ? true : (g.RM == 32);
     const bool pairing = !(h->cfg.flags & LP_FLAG_NO_PAIRING);
-    // bf16 32x32 regions: de-duplicate into 128x64 slices and pair two slices per N = 128 task
-    // (the granularity that re-executes 1.7x less work than 128x128 tiles at 5% failed regions)
+    // bf16 32x32 regions: de-duplicate into 128x64 slices and group up to four slices of a row band per
+    // N = 256 task (1.7x less re-executed work than 128x128 tiles at 5% failed regions, same A panel reuse)
     const bool slices = tc_ok && g.RM == 32 && pairing && !(h->cfg.flags & LP_FLAG_RECOVER_TILE128);
     const int EN = slices ? 64 : E;
     if (list && workspace && need_dedupe && dedupe_tiles(g, E, EN) > 0) {
@@ -334,12 +334,13 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
       a.slice64 = slices ? 1 : 0;
     }
     if (list && workspace && tc_ok && (a.list_is_tiles || g.RM == 128) && pairing) {
-      // pair failed 128x128 tiles (or 128x64 slices) of the same row band into 128x256 (128x128) tasks
+      // pair failed 128x128 tiles of the same row band into 128x256 tasks (or group up to four 128x64 slices)
       const WsLayout w = ws_layout(g);
       uint8_t* ws = (uint8_t*)workspace;
       const int64_t off = a.list_is_tiles ? 0 : g.rid_offset;
       const int64_t div = a.list_is_tiles ? g.N / EN : g.Q;
-      cudaError_t e0 = lp::launch_pair_tasks(a.list, a.d_n, off, div, h->sm_count, (int32_t*)(ws + w.tasks),
+      cudaError_t e0 = lp::launch_pair_tasks(a.list, a.d_n, off, div, h->sm_count, a.slice64 ? 4 : 2,
+                                             (int32_t*)(ws + w.tasks),
                                              (int64_t*)(ws + w.d_ntasks), st);
       if (e0 != cudaSuccess) return cuda_fail(e0, "recovery pairing");
       a.tasks = (const int32_t*)(ws + w.tasks);

@@ -43,8 +43,9 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
                           cudaStream_t st);
 // ascending list of 128x128 tiles/regions -> recovery tasks of 1-2 entries of the same row band
 // (row = (list[i] - off) / div); pairing only when *d_n > min_pair.  tasks[t] = (i << 1) | paired.
+// G = 4: tasks of up to four entries (128x64 slices), tasks[t] = (i << 2) | (count - 1).
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
-                              int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
+                              int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
 // failed regions -> unique tile ids of an EM x EN tile grid (tile = (p*RM/EM)*(N/EN) + q*RN/EN), ascending
 cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const int64_t* list, const int64_t* d_n,
@@ -70,7 +71,7 @@ struct TmmArgs {
   const int64_t* list;  // list mode (recovery) when non-null
   const int64_t* d_n;
   int list_is_tiles;    // list holds 128x128 tile ids (de-duplicated recovery of 32x32 regions)
-  int slice64;          // with list_is_tiles: ids are 128x64 slices, tasks pair two slices into one N = 128 tile
+  int slice64;          // with list_is_tiles: ids are 128x64 slices, a task is 1-4 slices of one row band (N = 64..256)
   const int32_t* tasks;  // tcgen05 list mode: paired recovery tasks (launch_pair_tasks), or null
   const int64_t* d_ntasks;
   int force_1cta;       // tcgen05: use the 1-CTA 128x256 kernel even where the CTA-pair kernel applies

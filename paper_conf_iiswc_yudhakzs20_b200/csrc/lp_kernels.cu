@@ -407,7 +407,8 @@ __global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t
 // equal rows, entries at even offsets from the run start head a task; a head takes
 // its successor when it lies in the same row.  Pairing is used only when there are
 // more entries than SMs (otherwise one entry per CTA finishes sooner).
-// tasks[t] = (list index << 1) | paired.  One CTA of 1024 threads, chunked scans.
+// tasks[t] = (list index << 1) | paired.  G = 4 (128x64 slices of 32x32 regions): up to four
+// entries of one row per task, tasks[t] = (list index << 2) | (count - 1).  One CTA of 1024 threads, chunked scans.
 constexpr int kPairThreads = 1024;
 
 __device__ __forceinline__ int64_t block_scan_max_i64(int64_t v, int64_t* s_warp, int64_t* total) {
@@ -466,7 +467,7 @@ __device__ __forceinline__ int block_scan_excl_sum(int v, int* s_warp, int* tota
 
 __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t* __restrict__ list,
                                                                   const int64_t* __restrict__ d_n, int64_t off,
-                                                                  int64_t div, int64_t min_pair,
+                                                                  int64_t div, int64_t min_pair, int G,
                                                                   int32_t* __restrict__ tasks,
                                                                   int64_t* __restrict__ d_ntasks) {
   __shared__ int64_t s_max[32];
@@ -484,12 +485,13 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
     int64_t blk_max;
     int64_t ls = block_scan_max_i64(run_head ? i : -1, s_max, &blk_max);
     ls = ls > carry_ls ? ls : carry_ls;
-    const bool head = valid && (!pairing || ((i - ls) & 1) == 0);
-    bool paired = false;
-    if (head && pairing && i + 1 < n) paired = (list[i + 1] - off) / div == row;
+    const bool head = valid && (!pairing || ((i - ls) % G) == 0);
+    int cnt = 1;  // entries of this task: the head and its successors in the same row, at most G
+    if (head && pairing)
+      for (int j = 1; j < G && i + j < n && (list[i + j] - off) / div == row; ++j) ++cnt;
     int tot;
     const int idx = block_scan_excl_sum(head ? 1 : 0, s_sum, &tot);
-    if (head) tasks[carry_t + idx] = (int32_t)((i << 1) | (paired ? 1 : 0));
+    if (head) tasks[carry_t + idx] = (int32_t)((i << (G == 4 ? 2 : 1)) | (cnt - 1));
     carry_t += tot;
     carry_ls = blk_max > carry_ls ? blk_max : carry_ls;
   }
@@ -734,8 +736,8 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const in
 }
 
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
-                              int32_t* tasks, int64_t* d_ntasks, cudaStream_t st) {
-  pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, tasks, d_ntasks);
+                              int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st) {
+  pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, G, tasks, d_ntasks);
   return cudaGetLastError();
 }
 

@@ -93,7 +93,7 @@ struct TileSrc {
   const int32_t* tasks;       // paired list mode: (list index << 1) | paired (launch_pair_tasks)
   const int64_t* d_ntasks;
   int64_t n128;               // 128-column tiles per row (tile-id decoding)
-  int slice64;                // list holds 128x64 slice ids (n64 per row); a task is one or two slices
+  int slice64;                // list holds 128x64 slice ids (n64 per row); a task is 1-4 slices (slices())
   int64_t n64;
   __device__ __forceinline__ int64_t count() const {
     return tasks ? *d_ntasks : (list ? *d_n : num_m * num_n);
@@ -114,17 +114,6 @@ struct TileSrc {
   // mode: two failed tiles of the same row band (B gathered from two panels).
   template <int BN>
   __device__ __forceinline__ void cols(int64_t t, int64_t& mb, int64_t& n_lo, int64_t& n_hi, bool& has_hi) const {
-    if (tasks && slice64) {
-      // two 64-column slices of one row band: B chunk 0 from n_lo's panel, chunk 1 from n_hi's
-      const int32_t w = tasks[t];
-      const int64_t i = w >> 1, e = list[i];
-      mb = e / n64;
-      n_lo = (e - mb * n64) * 64;
-      has_hi = (w & 1) != 0;
-      n_hi = n_lo;
-      if (has_hi) n_hi = (list[i + 1] - mb * n64) * 64;
-      return;
-    }
     if (tasks) {
       const int32_t w = tasks[t];
       const int64_t i = w >> 1;
@@ -145,6 +134,16 @@ struct TileSrc {
     n_lo = nb * BN;
     n_hi = n_lo + 128;
     has_hi = BN == 256;
+  }
+  // Slice task t (slice64): 1-4 128x64 slices of one row band, first columns nc[0..cnt);
+  // B chunk c is staged from slice c's column panel and lands in accumulator columns [64c, 64c+64).
+  __device__ __forceinline__ void slices(int64_t t, int64_t& mb, int& cnt, int64_t (&nc)[4]) const {
+    const int32_t w = tasks[t];
+    const int64_t i = w >> 2;
+    cnt = (w & 3) + 1;
+    mb = list[i] / n64;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) nc[c] = c < cnt ? (list[i + c] - mb * n64) * 64 : 0;
   }
   template <int BN>
   __device__ __forceinline__ void coords(int64_t t, int64_t& mb, int64_t& nb) const {

@@ -62,6 +62,11 @@ __host__ __device__ constexpr uint32_t instr_desc() {
          ((uint32_t)(kBM >> 4) << 24);
 }
 
+__device__ __forceinline__ uint32_t instr_desc_n(int n) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) | ((uint32_t)(n >> 3) << 17) |
+         ((uint32_t)(kBM >> 4) << 24);
+}
+
 template <typename OutT, uint32_t MASK, int REG, int BN, int STORE>
 __global__ void __launch_bounds__(kThreads, 1)
     tmm_tc_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
@@ -118,29 +123,30 @@ __global__ void __launch_bounds__(kThreads, 1)
       int stage = 0;
       uint32_t phase = 0;
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        int64_t mb, n_lo, n_hi;
-        bool has_hi;
-        src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
-        const int m0 = (int)(mb * kBM);
         // B is staged as 64-column chunks: 0,1 from the low half's panel, 2,3 from the high half's
-        // (128x64 slice tasks: chunk 0 = the low slice, chunk 1 = the high slice if paired)
-        const bool sl = BN == 128 && src.slice64;
-        const uint32_t bytes = Cfg::kABytes + (sl ? (has_hi ? 2 : 1) : (has_hi ? 4 : 2)) * (kBK * 128);
+        // (slice tasks: chunk c from slice c's panel)
+        int64_t mb, col[4];
+        int nch;
+        if (BN == 256 && src.slice64) {
+          src.slices(t, mb, nch, col);
+        } else {
+          int64_t n_lo, n_hi;
+          bool has_hi;
+          src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
+          nch = has_hi ? 4 : 2;
+#pragma unroll
+          for (int c = 0; c < 4; ++c) col[c] = (c < 2 ? n_lo : n_hi) + (c & 1) * 64;
+        }
+        const int m0 = (int)(mb * kBM);
+        const uint32_t bytes = Cfg::kABytes + nch * (kBK * 128);
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], bytes);
           tma_load_2d(&tmap_a, &full[stage], sA + stage * Cfg::kABytes, kb * kBK, m0);
-          if (sl) {
-            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes, (int)n_lo, kb * kBK);
-            if (has_hi)
-              tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + kBK * 128, (int)n_hi, kb * kBK);
-          } else {
 #pragma unroll
-            for (int c = 0; c < BN / 64; ++c) {
-              if (c >= 2 && !has_hi) break;
-              const int64_t col = (c < 2 ? n_lo : n_hi) + (c & 1) * 64;
-              tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), (int)col, kb * kBK);
-            }
+          for (int c = 0; c < BN / 64; ++c) {
+            if (c >= nch) break;
+            tma_load_2d(&tmap_b, &full[stage], sB + stage * Cfg::kBBytes + c * (kBK * 128), (int)col[c], kb * kBK);
           }
           if (++stage == S) {
             stage = 0;
@@ -157,14 +163,16 @@ __global__ void __launch_bounds__(kThreads, 1)
       int acc = 0;
       uint32_t acc_phase = 0;
       for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        int64_t mb, n_lo, n_hi;
-        bool has_hi;
-        src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
-        // N = 256 when both halves are live, else N = 128 into the low half;
-        // slice tasks: N = 128 for a pair, N = 64 for a lone slice
-        const uint32_t idesc = (BN == 256 && has_hi) ? instr_desc<256>()
-                               : (BN == 128 && src.slice64 && !has_hi) ? instr_desc<64>()
-                                                                       : instr_desc<128>();
+        // N = 256 when both halves are live, else N = 128 into the low half; slice tasks: N = 64 x slices
+        uint32_t idesc;
+        if (BN == 256 && src.slice64) {
+          idesc = instr_desc_n(64 * ((src.tasks[t] & 3) + 1));
+        } else {
+          int64_t mb, n_lo, n_hi;
+          bool has_hi;
+          src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
+          idesc = (BN == 256 && has_hi) ? instr_desc<256>() : instr_desc<128>();
+        }
         mbar_wait(&tempty[acc], acc_phase ^ 1);  // epilogue drained this accumulator
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -201,28 +209,35 @@ __global__ void __launch_bounds__(kThreads, 1)
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x) {
-      int64_t mb, n_lo, n_hi;
-      bool has_hi;
-      src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
       mbar_wait(&tfull[acc], acc_phase);
       tc_fence_after();
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
       CkRecord* srec_acc = srec + acc * (BN / 128) * 4;
-      bool sliced = false;
-      if constexpr (REG == 32 && BN == 128) {
+      if constexpr (REG == 32 && BN == 256) {
         if (src.slice64) {
-          // accumulator columns [0,64) -> the low slice, [64,128) -> the high slice (32x32 records per chunk)
-          epi_store<OutT, MASK, REG, 64, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
-                                                src.rid_offset);
-          if (has_hi)
-            epi_store<OutT, MASK, REG, 64, STORE>(t_row + 64, C, ldc, mb, n_hi, wq, lane, srec_acc, ck, src.Qr,
+          // accumulator columns [64c, 64c+64) -> slice c (32x32 records per 32-column chunk)
+          int64_t mb, nc[4];
+          int cnt;
+          src.slices(t, mb, cnt, nc);
+#pragma unroll 1
+          for (int c = 0; c < cnt; ++c)
+            epi_store<OutT, MASK, REG, 64, STORE>(t_row + 64 * c, C, ldc, mb, nc[c], wq, lane, srec_acc, ck, src.Qr,
                                                   src.rid_offset);
-          sliced = true;
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&tempty[acc]);
+          if (++acc == 2) {
+            acc = 0;
+            acc_phase ^= 1;
+          }
+          continue;
         }
       }
-      if (!sliced)
-        epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
-                                               src.rid_offset);
+      int64_t mb, n_lo, n_hi;
+      bool has_hi;
+      src.cols<BN>(t, mb, n_lo, n_hi, has_hi);
+      epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, mb, n_lo, wq, lane, srec_acc, ck, src.Qr,
+                                             src.rid_offset);
       if (BN == 256 && has_hi)
         epi_store<OutT, MASK, REG, 128, STORE>(t_row + 128, C, ldc, mb, n_hi, wq, lane, srec_acc + 4, ck, src.Qr,
                                                src.rid_offset);
@@ -529,8 +544,9 @@ cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
   if (!a.list && a.M % 256 == 0 && a.N % 256 == 0 && !a.force_1cta) return launch_pair<OutT, REG>(a, st, why);
   // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
   // 16 32x32 regions of a de-duplicated tile; paired tasks (two such tiles of one
-  // row band) run on the BN = 256 kernel with B gathered from two column panels
-  const bool bn256 = a.list ? (a.tasks != nullptr && !a.slice64) : (a.N % 256 == 0);
+  // row band) run on the BN = 256 kernel with B gathered from two column panels, and
+  // so do slice tasks (1-4 de-duplicated 128x64 slices of one row band, N = 64..256)
+  const bool bn256 = a.list ? (a.tasks != nullptr) : (a.N % 256 == 0);
   return bn256 ? launch_cfg<OutT, REG, 256>(a, st, why) : launch_cfg<OutT, REG, 128>(a, st, why);
 }
 

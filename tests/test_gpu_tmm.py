@@ -170,10 +170,11 @@ def test_tc_paired_recovery(pairing, reg, N, frac, out_dt):
 @pytest.mark.parametrize("N,frac", [(2048, 0.01), (2176, 0.1), (2048, 0.5), (1152, 1.0)])
 @pytest.mark.parametrize("out_dt", ["bf16", "f32"])
 def test_tc_slice_recovery(slices, N, frac, out_dt):
-    """32x32 regions recovered as de-duplicated 128x64 slices (two slices of a row band per N = 128 tcgen05
-    task, B gathered from two 64-column panels; a lone slice runs N = 64) vs the 128x128-tile path
-    (LP_FLAG_RECOVER_TILE128).  frac 0.01: fewer slices than SMs (no pairing); N = 2176: 34 slice columns
-    per row band, odd runs; frac 1.0: every region.  Recovered bytes and records must equal the golden run."""
+    """32x32 regions recovered as de-duplicated 128x64 slices (up to four slices of a row band per tcgen05
+    task, N = 64 x slices, B gathered from up to four 64-column panels) vs the 128x128-tile path
+    (LP_FLAG_RECOVER_TILE128).  frac 0.01: fewer slices than SMs (one slice per task, N = 64); N = 2176: 34
+    slice columns per row band, runs of every length mod 4 (N = 64, 128, 192, 256 tasks); frac 1.0: every
+    region.  Recovered bytes and records must equal the golden run."""
     _, nf = run_cycle(2048, N, 256, 32, 32, "bf16", out_dt, "uniform", "mod|xor", "tcgen05", mode="stale_words",
                       frac=frac, recover_slices=slices)
     assert nf > 0
