@@ -465,6 +465,8 @@ __device__ __forceinline__ int block_scan_excl_sum(int v, int* s_warp, int* tota
   return r;
 }
 
+constexpr int kPairPer = 4;  // entries per thread per block pass (4096 per pass: fewer block scans)
+
 __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t* __restrict__ list,
                                                                   const int64_t* __restrict__ d_n, int64_t off,
                                                                   int64_t div, int64_t min_pair, int G,
@@ -472,26 +474,47 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
                                                                   int64_t* __restrict__ d_ntasks) {
   __shared__ int64_t s_max[32];
   __shared__ int s_sum[32];
+  __shared__ int64_t s_incl[kPairThreads];
   const int64_t n = *d_n;
   const bool pairing = n > min_pair;
+  const int sh = G == 4 ? 2 : 1;
   int64_t carry_ls = -1;  // index of the last run start seen so far
   int64_t carry_t = 0;    // tasks emitted so far
-  for (int64_t base = 0; base < n; base += kPairThreads) {
-    const int64_t i = base + threadIdx.x;
-    const bool valid = i < n;
-    const int64_t row = valid ? (list[i] - off) / div : -1;
-    const int64_t prev = (valid && i > 0) ? (list[i - 1] - off) / div : -2;
-    const bool run_head = valid && row != prev;
+  for (int64_t base = 0; base < n; base += (int64_t)kPairThreads * kPairPer) {
+    const int64_t i0 = base + (int64_t)threadIdx.x * kPairPer;
+    int64_t rows[kPairPer];
+    bool rh[kPairPer];
+    int64_t prev = (i0 > 0 && i0 - 1 < n) ? (list[i0 - 1] - off) / div : -2;
+    int64_t lmax = -1;  // last run start among this thread's entries
+#pragma unroll
+    for (int j = 0; j < kPairPer; ++j) {
+      const int64_t i = i0 + j;
+      rows[j] = i < n ? (list[i] - off) / div : -1;
+      rh[j] = i < n && rows[j] != prev;
+      if (rh[j]) lmax = i;
+      prev = rows[j];
+    }
     int64_t blk_max;
-    int64_t ls = block_scan_max_i64(run_head ? i : -1, s_max, &blk_max);
+    s_incl[threadIdx.x] = block_scan_max_i64(lmax, s_max, &blk_max);
+    __syncthreads();
+    int64_t ls = threadIdx.x ? s_incl[threadIdx.x - 1] : -1;  // last run start before this thread's entries
     ls = ls > carry_ls ? ls : carry_ls;
-    const bool head = valid && (!pairing || ((i - ls) % G) == 0);
-    int cnt = 1;  // entries of this task: the head and its successors in the same row, at most G
-    if (head && pairing)
-      for (int j = 1; j < G && i + j < n && (list[i + j] - off) / div == row; ++j) ++cnt;
+    int32_t w[kPairPer];
+    int nh = 0;
+#pragma unroll
+    for (int j = 0; j < kPairPer; ++j) {
+      const int64_t i = i0 + j;
+      if (rh[j]) ls = i;
+      if (i < n && (!pairing || ((i - ls) % G) == 0)) {
+        int cnt = 1;  // entries of this task: the head and its successors in the same row, at most G
+        if (pairing)
+          for (int k = 1; k < G && i + k < n && (list[i + k] - off) / div == rows[j]; ++k) ++cnt;
+        w[nh++] = (int32_t)((i << sh) | (cnt - 1));
+      }
+    }
     int tot;
-    const int idx = block_scan_excl_sum(head ? 1 : 0, s_sum, &tot);
-    if (head) tasks[carry_t + idx] = (int32_t)((i << (G == 4 ? 2 : 1)) | (cnt - 1));
+    const int idx = block_scan_excl_sum(nh, s_sum, &tot);
+    for (int k = 0; k < nh; ++k) tasks[carry_t + idx + k] = w[k];
     carry_t += tot;
     carry_ls = blk_max > carry_ls ? blk_max : carry_ls;
   }

@@ -123,6 +123,12 @@ def test_c3_tmm16384_r32_array_full():
     _tmm_full(16384, 16384, 16384, 32, "mod|xor", "array", "int5", "bf16", nsample=4, seed=9)
 
 
+def test_tmm8192_r32_half_failed_slice_grouping():
+    """8192^2 with 32x32 regions and half of them failed: ~8000 failed 128x64 slices, so the grouping kernel
+    takes several 4096-entry passes (run starts and task counts carried across passes)."""
+    _tmm_full(8192, 8192, 128, 32, "mod|xor", "array", "int5", "bf16", nsample=2, frac=0.5, seed=21)
+
+
 def test_c5_tmm65536_rank3_of_8_shard():
     """configs[4]: one rank's shard of the 65536^3 region-sharded TMM (rank 3 of 8), exactly as bench.py launches it."""
     s = shard.plan(65536, 65536, 128, 128, 8, 3)
