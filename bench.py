@@ -127,6 +127,8 @@ def parse():
     ap.add_argument("--no-shuffle", action="store_true", help="SIMT body: sequential reduction ablation (L343)")
     ap.add_argument("--no-pairing", action="store_true",
                     help="tcgen05 recovery: one 128x128 tile per failed tile (no same-row pairing) -- A/B switch")
+    ap.add_argument("--inject-frac", type=float, default=None,
+                    help="override the workload's injected fraction of regions (design-space runs)")
     ap.add_argument("--recover-tile128", action="store_true",
                     help="tcgen05 recovery of 32x32 regions: 128x128 tiles instead of 128x64 slices -- A/B switch")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
@@ -244,6 +246,8 @@ def run_ours(args):
         W["store"] = args.store
     if args.cksum:
         W["cksum"] = args.cksum
+    if args.inject_frac is not None:
+        W["frac"] = args.inject_frac
     RM = RN = W["region"]
     if W["kind"] == "spmv":
         RM = 1

@@ -407,8 +407,8 @@ __global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t
 // equal rows, entries at even offsets from the run start head a task; a head takes
 // its successor when it lies in the same row.  Pairing is used only when there are
 // more entries than SMs (otherwise one entry per CTA finishes sooner).
-// tasks[t] = (list index << 1) | paired.  G = 4 (128x64 slices of 32x32 regions): up to four
-// entries of one row per task, tasks[t] = (list index << 2) | (count - 1).  One CTA of 1024 threads, chunked scans.
+// tasks[t] = (list index << 1) | paired.  G = 4 (128x64 slices of 32x32 regions): up to
+// min(4, max(2, ceil(n / #SM))) entries of one row per task, tasks[t] = (list index << 2) | (count - 1).  One CTA of 1024 threads, chunked scans.
 constexpr int kPairThreads = 1024;
 
 __device__ __forceinline__ int64_t block_scan_max_i64(int64_t v, int64_t* s_warp, int64_t* total) {
@@ -478,6 +478,12 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
   const int64_t n = *d_n;
   const bool pairing = n > min_pair;
   const int sh = G == 4 ? 2 : 1;
+  // slice grouping (G = 4): as many entries per task as it takes to fill the SMs once, 2..4
+  // (300 failed slices on 148 SMs: tasks of 3 -> one wave of N = 192, not 75 tasks of N = 256)
+  if (G == 4 && pairing) {
+    const int64_t need = (n + min_pair - 1) / min_pair;
+    G = need < 2 ? 2 : (need > 4 ? 4 : (int)need);
+  }
   int64_t carry_ls = -1;  // index of the last run start seen so far
   int64_t carry_t = 0;    // tasks emitted so far
   for (int64_t base = 0; base < n; base += (int64_t)kPairThreads * kPairPer) {
