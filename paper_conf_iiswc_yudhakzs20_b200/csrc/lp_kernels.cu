@@ -475,6 +475,8 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
   __shared__ int64_t s_max[32];
   __shared__ int s_sum[32];
   __shared__ int64_t s_incl[kPairThreads];
+  // the re-execution grid that follows may start its prologue now (it waits for this grid to finish)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int64_t n = *d_n;
   const bool pairing = n > min_pair;
   const int sh = G == 4 ? 2 : 1;

@@ -113,6 +113,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_holder;
+  // list mode is launched programmatically dependent on the grouping kernel: the prologue above
+  // (barriers, TMEM allocation, tensor-map prefetch) overlaps its tail; the task list is read only
+  // after it has completed and flushed (a no-op for ordinary launches)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
 
   const int64_t ntiles = src.count();
   const int nkb = (int)(K / kBK);
@@ -436,6 +440,23 @@ bool make_map_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64_t oute
                     CU_TENSOR_MAP_SWIZZLE_128B);
 }
 
+// List-mode (recovery) launches carry the programmatic-stream-serialization attribute so the CTAs
+// can be scheduled while the grouping kernel (which triggers launch_dependents) is still running.
+template <typename Kern, typename... Args>
+cudaError_t launch_maybe_pdl(Kern kfn, unsigned grid, int smem, cudaStream_t st, bool pdl, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kfn, args...);
+}
+
 template <typename OutT, int REG, int BN>
 cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   using Cfg = TcCfg<BN>;
@@ -472,7 +493,9 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
     auto kfn = tmm_tc_kernel<OutT, M, REG, BN, S>;                                                         \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
     if (e != cudaSuccess) return e;                                                                         \
-    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, src, a.ck);                \
+    e = launch_maybe_pdl(kfn, (unsigned)grid, smem, st, a.list != nullptr, ma, mb, (OutT*)a.C, a.ldc, a.K, src, \
+                         a.ck);                                                                             \
+    if (e != cudaSuccess) return e;                                                                         \
     break;                                                                                                  \
   }
 #define LP_TC_CASE3(M) LP_TC_CASE(M, 0)
