@@ -133,9 +133,11 @@ typedef enum {
                                     of in the last validate CTA for tables of <= 16384 regions (A/B switch) */
   LP_FLAG_NO_PAIRING = 4u, /* tcgen05 bf16 recovery: one 128x128 tile per failed region/tile instead of pairing
                               failed tiles of the same row band into 128x256 tasks (A/B switch) */
-  LP_FLAG_RECOVER_TILE128 = 16u /* tcgen05 bf16 recovery of 32x32 regions: de-duplicate failed regions into 128x128
+  LP_FLAG_RECOVER_TILE128 = 16u, /* tcgen05 bf16 recovery of 32x32 regions: de-duplicate failed regions into 128x128
                                    tiles (paired into 128x256 tasks) instead of 128x64 slices paired into 128x128
                                    tasks (A/B switch; both re-execute every failed region, L51-57) */
+  LP_FLAG_CUCKOO_SHORT_CHAINS = 32u /* cuckoo stores, test hook: the body's inserts give up after 16 evictions
+                                       instead of 128, so entries reach the stash and the rehash (L270) runs */
 } lp_config_flags;
 
 typedef struct {
@@ -172,8 +174,11 @@ LP_API lp_status lp_num_regions(lp_handle h, const lp_workload_t* wl, int64_t* r
 /* Bytes of the checksum buffer.  ARRAY: R * 4 * selem (selem = popcount(cksum),
  * L528 "number of checksums in an element").  QUAD_*: 64-byte header + cap *
  * 4 * (1 + selem) with cap = smallest prime >= ceil(R / 0.7) (L267 load <= 70%).
- * CUCKOO*: 64-byte header + 2 tables * cap * 16 with cap = smallest prime >= R
- * (total load <= 50%, L270). */
+ * CUCKOO*: 64-byte header + (2 tables * cap + 256 stash entries) * 16 with
+ * cap = smallest prime >= ceil(1.15 R) (total load <= 43.5%, L270).
+ * Hash header (u32 words): cap, seed, lock, error, collisions (u64), stash_n,
+ * rehashes, max_evict, 7 reserved.  The seed changes when a cuckoo table is
+ * rehashed: lookups must read it from the header. */
 LP_API lp_status lp_cksum_bytes(lp_handle h, const lp_workload_t* wl, size_t* bytes);
 
 /* Bytes of the scratch `workspace` lp_validate / lp_recover use (flags, scan counters,
@@ -189,7 +194,12 @@ LP_API lp_status lp_cksum_init(lp_handle h, const lp_workload_t* wl, void* cksum
 
 /* The LP-protected region kernel: computes out = body(wl) and, in the same
  * kernel, stores one record per region into cksum (no second pass over out).
- * cfg.cksum == 0 runs the unprotected twin (cksum may be NULL). */
+ * cfg.cksum == 0 runs the unprotected twin (cksum may be NULL).
+ * Cuckoo stores: an insert whose eviction walk reaches the bound (a cycle, L270)
+ * parks its entry in the table's stash; a one-CTA rehash kernel enqueued after the
+ * body (and after lp_recover) then rebuilds T1/T2 in place under a new seed and
+ * re-inserts the stash, retrying with further seeds.  It returns at once when the
+ * stash is empty.  lp_stats reports error = 1 only if an entry could not be placed. */
 LP_API lp_status lp_run_protected(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, lp_stream_t stream);
 
 /* Validation: recompute every region's record from `out`, compare with `cksum`

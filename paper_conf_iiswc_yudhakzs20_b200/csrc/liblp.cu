@@ -60,9 +60,11 @@ bool is_prime(uint64_t n) {
   return true;
 }
 
-// quadratic probing: load <= 70% (L267); cuckoo: per-table capacity, total load <= 50% (L270)
+// quadratic probing: load <= 70% (L267); cuckoo: per-table capacity 1.15 R, total load <= 43.5%
+// (L270 bounds the load; 50% is the threshold of two-table cuckoo hashing, where eviction
+// cycles become common -- the rehash then has to run often)
 uint32_t hash_cap(int64_t R, int store) {
-  uint64_t c = store >= LP_STORE_CUCKOO ? (uint64_t)R : (uint64_t)std::ceil((double)R / 0.7);
+  uint64_t c = store >= LP_STORE_CUCKOO ? (uint64_t)std::ceil((double)R * 1.15) : (uint64_t)std::ceil((double)R / 0.7);
   if (c < 2) c = 2;
   while (!is_prime(c)) ++c;
   return (uint32_t)c;
@@ -171,12 +173,14 @@ lp::HashInfo hash_info(const lp_ctx* h, const lp::RegionGeom& g) {
   hi.store = h->cfg.store;
   hi.cap = h->cfg.store == LP_STORE_ARRAY ? 0u : hash_cap(g.R, h->cfg.store);
   hi.seed = h->cfg.hash_seed;
+  hi.max_evict = (h->cfg.flags & LP_FLAG_CUCKOO_SHORT_CHAINS) ? 16u : 0u;
   return hi;
 }
 
 size_t cksum_bytes(const lp_ctx* h, const lp::RegionGeom& g) {
   if (h->cfg.store == LP_STORE_ARRAY) return (size_t)g.R * 4u * (size_t)h->selem;
-  if (h->cfg.store >= LP_STORE_CUCKOO) return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R, h->cfg.store) * 2u * 16u;
+  if (h->cfg.store >= LP_STORE_CUCKOO)
+    return sizeof(lp::HashHeader) + ((size_t)hash_cap(g.R, h->cfg.store) * 2u + lp::kCuckooStash) * 16u;
   return sizeof(lp::HashHeader) + (size_t)hash_cap(g.R, h->cfg.store) * 4u * (size_t)(1 + h->selem);
 }
 
@@ -358,6 +362,14 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   return e == cudaSuccess ? ok() : cuda_fail(e, "SIMT TMM launch");
 }
 
+// Cuckoo stores: inserts that hit the eviction bound parked their entry in the stash;
+// rebuild the tables with a new seed on the device (a no-op launch while the stash is empty).
+lp_status cuckoo_rehash(const lp_ctx* h, void* cksum, cudaStream_t st) {
+  if (h->cfg.store < LP_STORE_CUCKOO || h->mask == 0) return ok();
+  cudaError_t e = lp::launch_cuckoo_rehash(cksum, st);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "cuckoo rehash launch");
+}
+
 }  // namespace
 
 extern "C" {
@@ -378,7 +390,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING | LP_FLAG_NO_FUSED_COMPACT |
-                                 LP_FLAG_RECOVER_TILE128))
+                                 LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");
@@ -455,7 +467,8 @@ lp_status lp_run_protected(lp_handle h, const lp_workload_t* wl, void* out, void
   if (h->mask && !aligned16(cksum)) return fail(LP_ERR_INVALID_ARG, "cksum must be 16-B aligned");
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
-  return run_body(h, wl, g, out, cksum, nullptr, nullptr, (cudaStream_t)stream);
+  if ((s = run_body(h, wl, g, out, cksum, nullptr, nullptr, (cudaStream_t)stream))) return s;
+  return cuckoo_rehash(h, cksum, (cudaStream_t)stream);
 }
 
 lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, const void* cksum, int64_t* failed_list,
@@ -494,7 +507,8 @@ lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksu
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
   if (workspace && !aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
-  return run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace);
+  if ((s = run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace))) return s;
+  return cuckoo_rehash(h, cksum, (cudaStream_t)stream);
 }
 
 lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, int64_t* d_n_recovered,

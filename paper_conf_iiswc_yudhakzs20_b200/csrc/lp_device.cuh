@@ -143,12 +143,17 @@ __device__ __forceinline__ void store_array(uint32_t* table, int64_t local_rid, 
 
 // Hash-store layout inside the caller's cksum buffer (Reading R14):
 //   [0]  u32 cap      [1] u32 seed     [2] u32 lock word   [3] u32 error flag
-//   [4..5] u64 collisions (sum of probes-1)       [6..15] reserved
-//   then cap entries of (1 + selem) u32: key (0xFFFFFFFF = empty), record.
+//   [4..5] u64 collisions (sum of probes-1)
+//   [6]  u32 stash_n (cuckoo: entries parked by chains that hit the eviction bound)
+//   [7]  u32 rehashes (cuckoo: completed rehash attempts)  [8] u32 max_evict (0 = kCuckooMaxEvict)
+//   [9..15] reserved
+//   then cap entries of (1 + selem) u32: key (0xFFFFFFFF = empty), record   (quadratic probing)
+//   or   T1[cap], T2[cap] 16-byte entries + a stash of kCuckooStash entries (cuckoo).
 struct HashHeader {
   uint32_t cap, seed, lock, error;
   unsigned long long collisions;
-  uint32_t reserved[10];
+  uint32_t stash_n, rehashes, max_evict;
+  uint32_t reserved[7];
 };
 static_assert(sizeof(HashHeader) == 64, "hash header is 64 bytes");
 
@@ -249,10 +254,16 @@ __device__ __forceinline__ bool quad_lookup(const uint32_t* ckbuf, uint32_t rid,
 // (atomicExch()) ... we will always insert the entry to a hash table entry no
 // matter whether it is occupied or empty".  An entry is 16 bytes {key, rec0,
 // rec1, rec2} exchanged with ONE 128-bit atom.exch so a record always travels with
-// its key.  Per-table capacity = smallest prime >= R: total load <= 50% (L270).
-// A chain longer than kCuckooMaxEvict sets the error flag (the paper rehashes
-// with new functions; Reading R24).  Layout: HashHeader, T1[cap], T2[cap].
+// its key.  Per-table capacity = smallest prime >= 1.15 R: total load <= 43.5%,
+// below the 50% threshold of two-table cuckoo hashing (L270 bounds the load).
+// L270: "When a cycle is detected, the cuckoo hash table performs hash tables
+// rehashing" (Reading R24): an entry still homeless after max_evict placements is
+// parked in a small stash behind T2, and the rehash kernel that follows every
+// protected / recovery run (cuckoo_rehash_kernel) rebuilds T1/T2 in place with a
+// new seed and re-inserts the stash.  Only a stash overflow loses an entry (error
+// flag).  Layout: HashHeader, T1[cap], T2[cap], stash[kCuckooStash].
 constexpr int kCuckooMaxEvict = 128;
+constexpr int kCuckooStash = 256;
 
 __host__ __device__ __forceinline__ uint32_t cuckoo_h(int t, uint32_t key, uint32_t seed, uint32_t cap) {
   return (t == 0 ? hash_fmix32(key, seed) : hash_fmix32(key, seed * 0x9E3779B9u + 0x7F4A7C15u)) % cap;
@@ -275,6 +286,31 @@ __device__ __forceinline__ uint4 cuckoo_entry(uint32_t rid, const uint32_t* w) {
   return make_uint4(rid, S > 0 ? w[0] : 0u, S > 1 ? w[1] : 0u, S > 2 ? w[2] : 0u);
 }
 
+// Placement walk of one entry (Fig. 4): exchange into T1[H1], carry the occupant to the
+// other table, ... .  Returns the number of placements, or 0 when the walk hit the
+// eviction bound and the homeless entry went to the stash (rehash pending).
+__device__ __forceinline__ uint32_t cuckoo_place(HashHeader* hdr, uint4* tab, uint32_t cap, uint32_t seed, uint4 e,
+                                                 int bound, bool count) {
+  int t = 0;
+  for (int i = 0; i < bound; ++i) {
+    const uint4 old = atom_exch_128(tab + (uint64_t)t * cap + cuckoo_h(t, e.x, seed, cap), e);
+    if (old.x == kEmptyKey || old.x == e.x) {  // empty slot, or the same key's stale entry (dropped)
+      if (i && count) atomicAdd(&hdr->collisions, (unsigned long long)i);
+      return (uint32_t)i + 1;
+    }
+    e = old;  // carry the evicted entry to its slot in the other table
+    t ^= 1;
+  }
+  const uint32_t k = atomicAdd(&hdr->stash_n, 1u);
+  if (k < (uint32_t)kCuckooStash) {
+    uint4* stash = tab + 2ull * cap;
+    stash[k] = e;
+  } else {
+    atomicExch(&hdr->error, 1u);  // stash full: this entry is lost
+  }
+  return 0;
+}
+
 template <uint32_t MASK>
 __device__ __forceinline__ uint32_t cuckoo_insert(uint32_t* ckbuf, uint32_t rid, const uint32_t* w) {
   HashHeader* hdr = reinterpret_cast<HashHeader*>(ckbuf);
@@ -294,18 +330,8 @@ __device__ __forceinline__ uint32_t cuckoo_insert(uint32_t* ckbuf, uint32_t rid,
       break;
     }
   }
-  int t = 0;
-  for (int i = 0; i < kCuckooMaxEvict; ++i) {
-    const uint4 old = atom_exch_128(tab + (uint64_t)t * cap + cuckoo_h(t, e.x, seed, cap), e);
-    if (old.x == kEmptyKey || old.x == e.x) {  // empty slot, or the same key's stale entry (dropped)
-      if (i) atomicAdd(&hdr->collisions, (unsigned long long)i);
-      return (uint32_t)i + 1;
-    }
-    e = old;  // carry the evicted entry to its slot in the other table
-    t ^= 1;
-  }
-  atomicExch(&hdr->error, 1u);
-  return 0;
+  const uint32_t me = hdr->max_evict;
+  return cuckoo_place(hdr, tab, cap, seed, e, me ? (int)me : kCuckooMaxEvict, true);
 }
 
 template <uint32_t MASK>

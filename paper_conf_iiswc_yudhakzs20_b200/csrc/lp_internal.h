@@ -18,9 +18,10 @@ struct RegionGeom {
 };
 
 struct HashInfo {
-  int store;      // 0 array, 1 quad CAS, 2 quad lock
-  uint32_t cap;   // hash capacity (0 for array)
+  int store;      // 0 array, 1 quad CAS, 2 quad lock, 3 cuckoo, 4 cuckoo + lock
+  uint32_t cap;   // hash capacity (0 for array; cuckoo: per table)
   uint32_t seed;
+  uint32_t max_evict = 0;  // cuckoo eviction bound of the body's inserts (0 = kCuckooMaxEvict)
 };
 
 // ---- lp_kernels.cu
@@ -46,6 +47,8 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
 // G = 4: tasks of up to four entries (128x64 slices), tasks[t] = (i << 2) | (count - 1).
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
                               int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
+// cuckoo stores: rebuild T1/T2 with a new seed if the stash is non-empty (no-op otherwise)
+cudaError_t launch_cuckoo_rehash(void* ck, cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
 // failed regions -> unique tile ids of an EM x EN tile grid (tile = (p*RM/EM)*(N/EN) + q*RN/EN), ascending
 cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const int64_t* list, const int64_t* d_n,

@@ -529,13 +529,75 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
   if (threadIdx.x == 0) *d_ntasks = carry_t;
 }
 
-__global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed) {
+__global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed, uint32_t max_evict) {
   HashHeader* h = reinterpret_cast<HashHeader*>(ck);
   h->cap = cap;
   h->seed = seed;
   h->lock = 0;
   h->error = 0;
   h->collisions = 0ull;
+  h->stash_n = 0;
+  h->rehashes = 0;
+  h->max_evict = max_evict;
+}
+
+// Cuckoo rehash (L270: "When a cycle is detected, the cuckoo hash table performs hash
+// tables rehashing"; Reading R24).  Runs after every protected / recovery run of a cuckoo
+// store and returns at once while the stash is empty.  Otherwise, per attempt: a new seed
+// (new H1, H2); the stash is copied to shared memory and emptied; every thread walks a
+// strided share of T1/T2 and takes out (one 128-bit exchange) each entry that is not at
+// its slot under the new seed, re-placing it with the ordinary eviction walk; then the old
+// stash entries are placed.  Walks place entries only at their new-seed slots, so after
+// the pass every entry sits at H1'/H2' -- or, if a walk hit the bound, in the stash again,
+// and the next attempt tries another seed.  Rehash walks use the default bound and do not
+// count as insertion collisions (Table II counts inserts).
+constexpr int kRehashAttempts = 16;
+__global__ void __launch_bounds__(1024) cuckoo_rehash_kernel(uint32_t* ck) {
+  HashHeader* hdr = reinterpret_cast<HashHeader*>(ck);
+  if (*reinterpret_cast<volatile uint32_t*>(&hdr->stash_n) == 0) return;
+  __shared__ uint4 s_stash[kCuckooStash];
+  __shared__ uint32_t s_n, s_seed;
+  __shared__ unsigned long long s_coll;
+  uint4* tab = reinterpret_cast<uint4*>(ck + sizeof(HashHeader) / 4);
+  const uint32_t cap = hdr->cap;
+  if (threadIdx.x == 0) s_coll = hdr->collisions;
+  for (int attempt = 0; attempt < kRehashAttempts; ++attempt) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      const uint32_t n = hdr->stash_n;
+      s_n = n < (uint32_t)kCuckooStash ? n : (uint32_t)kCuckooStash;
+      s_seed = hash_fmix32(hdr->seed + 0x9E3779B9u, 0x5BD1E995u + (uint32_t)attempt);
+    }
+    __syncthreads();
+    for (uint32_t i = threadIdx.x; i < s_n; i += blockDim.x) s_stash[i] = tab[2ull * cap + i];
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      hdr->seed = s_seed;
+      hdr->stash_n = 0;
+      hdr->rehashes += 1;
+      __threadfence();
+    }
+    __syncthreads();
+    const uint32_t seed = s_seed;
+    const uint4 empty = make_uint4(kEmptyKey, kEmptyKey, kEmptyKey, kEmptyKey);
+    for (uint64_t s = threadIdx.x; s < 2ull * cap; s += blockDim.x) {
+      const int t = s < cap ? 0 : 1;
+      const uint32_t i = (uint32_t)(s - (uint64_t)t * cap);
+      const uint32_t key = *reinterpret_cast<volatile uint32_t*>(tab + s);
+      if (key == kEmptyKey || cuckoo_h(t, key, seed, cap) == i) continue;
+      const uint4 e = atom_exch_128(tab + s, empty);
+      if (e.x != kEmptyKey) cuckoo_place(hdr, tab, cap, seed, e, kCuckooMaxEvict, false);
+    }
+    for (uint32_t i = threadIdx.x; i < s_n; i += blockDim.x) cuckoo_place(hdr, tab, cap, seed, s_stash[i], kCuckooMaxEvict, false);
+    __threadfence();
+    __syncthreads();
+    if (*reinterpret_cast<volatile uint32_t*>(&hdr->stash_n) == 0) break;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    hdr->collisions = s_coll;
+    if (hdr->stash_n) hdr->error = 1u;   // no seed found: the stash still holds entries (LP_ERR_CAPACITY)
+  }
 }
 
 __global__ void stats_kernel(const uint32_t* ck, int has_hash, int64_t* d_stats) {
@@ -619,7 +681,7 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
   cudaError_t e = cudaMemsetAsync(ck, 0xFF, bytes, st);
   if (e != cudaSuccess) return e;
   if (hi.store != 0) {
-    hash_header_kernel<<<1, 1, 0, st>>>((uint32_t*)ck, hi.cap, hi.seed);
+    hash_header_kernel<<<1, 1, 0, st>>>((uint32_t*)ck, hi.cap, hi.seed, hi.max_evict);
     e = cudaGetLastError();
   }
   return e;
@@ -769,6 +831,11 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const in
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
                               int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st) {
   pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, G, tasks, d_ntasks);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_cuckoo_rehash(void* ck, cudaStream_t st) {
+  cuckoo_rehash_kernel<<<1, 1024, 0, st>>>((uint32_t*)ck);
   return cudaGetLastError();
 }
 

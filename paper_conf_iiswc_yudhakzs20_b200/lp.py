@@ -31,6 +31,7 @@ FLAG_NO_SHUFFLE = 2
 FLAG_NO_PAIRING = 4
 FLAG_NO_FUSED_COMPACT = 8
 FLAG_RECOVER_TILE128 = 16
+FLAG_CUCKOO_SHORT_CHAINS = 32
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
@@ -221,7 +222,7 @@ class LP:
     def __init__(self, region_m: int, region_n: int, cksum="mod|xor", store="array", device: int = 0,
                  body="auto", hash_seed: int = 0x9747B28C,
                  tc_pair: bool = True, shuffle: bool = True, pairing: bool = True, fused_compact: bool = True,
-                 recover_slices: bool = True):
+                 recover_slices: bool = True, cuckoo_short_chains: bool = False):
         self.mask = parse_cksum(cksum)
         self.store = STORE_NAMES[store] if isinstance(store, str) else int(store)
         self.body = BODY_NAMES[body] if isinstance(body, str) else int(body)
@@ -230,7 +231,8 @@ class LP:
         self.cfg = Config(region_m, region_n, self.mask, self.store, device, self.body, hash_seed,
                           (0 if tc_pair else FLAG_TC_1CTA) | (0 if shuffle else FLAG_NO_SHUFFLE) |
                           (0 if pairing else FLAG_NO_PAIRING) | (0 if fused_compact else FLAG_NO_FUSED_COMPACT) |
-                          (0 if recover_slices else FLAG_RECOVER_TILE128))
+                          (0 if recover_slices else FLAG_RECOVER_TILE128) |
+                          (FLAG_CUCKOO_SHORT_CHAINS if cuckoo_short_chains else 0))
         h = ctypes.c_void_p()
         _check(lib().lp_config(ctypes.byref(self.cfg), ctypes.byref(h)))
         self._h = h

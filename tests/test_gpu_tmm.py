@@ -19,9 +19,9 @@ pytestmark = pytest.mark.gpu
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
               store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True, pairing=True,
-              recover_slices=True):
+              recover_slices=True, cuckoo_short_chains=False):
     h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle, pairing=pairing,
-              recover_slices=recover_slices)
+              recover_slices=recover_slices, cuckoo_short_chains=cuckoo_short_chains)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -62,6 +62,11 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
                     tol = 1e-5
                 assert oracle.rel_err(to32(got), ref) <= tol, rid
     # clean validate -> 0 failed
+    if store.startswith("cuckoo"):
+        d_stats = torch.zeros(2, dtype=torch.int64, device=out.device)
+        h.stats(wl, ck, d_stats)
+        assert d_stats[1].item() == 0 and ck_golden[6] == 0        # nothing lost, stash empty after the rehash
+        run_cycle.last_rehashes = int(ck_golden[7])
     h.validate(wl, out, ck, failed, d_n, ws)
     assert int(d_n.item()) == 0
 
@@ -280,3 +285,39 @@ def test_tf32x3_hash_stores(store):
 def test_simt_no_shuffle_ablation(store):
     """The paper's "without parallel reduction" variant (L343): same records, sequential fold."""
     run_cycle(256, 256, 128, 32, 32, "i32", "i32", "int17", "mod|xor", "simt", store=store, frac=0.1, shuffle=False)
+
+
+# ----------------------------------------------------------------------------- cuckoo rehash (L270)
+def test_cuckoo_rehash_after_short_chains():
+    """L270 "When a cycle is detected, the cuckoo hash table performs hash tables rehashing": with the body's
+    eviction bound cut to 16 (test hook), walks at 43% load end in the stash (~20 of 65536 inserts); the rehash
+    kernel rebuilds T1/T2 under a new seed.  Afterwards every rid is found by the oracle's lookup (with the
+    header's new seed) with its oracle record, the stash is empty and the error flag is 0 -- and recovery
+    (which re-inserts) leaves the same state."""
+    run_cycle.last_rehashes = 0
+    run_cycle(8192, 8192, 64, 32, 32, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store="cuckoo", frac=0.05,
+              cuckoo_short_chains=True, check_values=False)
+    assert run_cycle.last_rehashes >= 1
+
+
+@pytest.mark.parametrize("store", ["cuckoo", "cuckoo_lock"])
+def test_cuckoo_full_r262144(store):
+    """at R = 262144 (16384^2 output, 32x32 regions) the 50%-load sizing lost records; with 1.15 R
+    per table + rehash every rid must be found with its oracle record and lp_stats must report no error."""
+    h = lp.LP(32, 32, cksum="mod|xor", store=store)
+    A, B = make_inputs(41, 16384, 16384, 64, "int5", "bf16")
+    a, b = host_to_dev(A, "bf16"), host_to_dev(B, "bf16")
+    wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    d_stats = torch.zeros(2, dtype=torch.int64, device=out.device)
+    h.stats(wl, ck, d_stats)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert d_stats[1].item() == 0
+    assert int(d_n.item()) == 0
+    R = h.num_regions(wl)
+    ck_h = dev_to_host(ck)
+    assert ck_h[6] == 0
+    check_store_table(ck_h, store, R, 2, oracle.records(dev_to_host(out), 32, 32, 3))

@@ -382,9 +382,15 @@ def test_cuckoo_eviction_moves_occupant_to_other_table():
     assert list(oracle.cuckoo_lookup(tab, cap, 1, x, seed)) == [222]
 
 
-def test_cuckoo_roundtrip_at_load_half():
+def _nextprime(c):
+    while c < 2 or any(c % d == 0 for d in range(2, int(c ** 0.5) + 1)):
+        c += 1
+    return c
+
+
+def test_cuckoo_roundtrip_at_library_sizing():
     R, sel, seed = 1000, 2, 9
-    cap = 1009  # per table -> total load 1000 / 2018 < 50% (L270)
+    cap = _nextprime(int(np.ceil(R * 1.15)))  # liblp's per-table sizing: total load 1000 / 2302 = 43% (L270)
     tab = np.full(2 * cap * 4, 0xFFFFFFFF, dtype=np.uint32)
     rng = random.Random(1)
     recs = {k: [rng.getrandbits(32), rng.getrandbits(32)] for k in range(R)}
@@ -414,3 +420,126 @@ def test_cuckoo_reinsert_updates_in_place():
     assert np.sum(keys != 0xFFFFFFFF) == 40   # no duplicates
     for k in range(40):
         assert list(oracle.cuckoo_lookup(tab, cap, 2, k, seed)) == [7 * k, 9]
+
+
+# --------------------------------------------------------------------------- hand-built hash tables (L183)
+def _fmix32(h):
+    h ^= h >> 16
+    h = (h * 0x85EBCA6B) & 0xFFFFFFFF
+    h ^= h >> 13
+    h = (h * 0xC2B2AE35) & 0xFFFFFFFF
+    h ^= h >> 16
+    return h
+
+
+def _records_by_hand(out, RM, RN, mask):
+    """{local rid: record} from Python ints + zlib (no oracle call)."""
+    Q = out.shape[1] // RN
+    return {p * Q + q: _brute_record(np.ascontiguousarray(out[p * RM:(p + 1) * RM, q * RN:(q + 1) * RN]), mask)
+            for p in range(out.shape[0] // RM) for q in range(Q)}
+
+
+def test_validate_cuckoo_hand_built_table():
+    """lpo_validate_cuckoo against a T1/T2 table placed by hand (L269-270, Fig. 4; Reading R24), with a global
+    rid offset: one key missing, one record word wrong, one key living in T2 and one region whose data changed.
+    The expected failed list is written out by hand below."""
+    RM = RN = 4
+    out = gen.generate(21, 16, 16, "uniform", "f32")          # 4 x 4 regions, local rids 0..15
+    mask, sel, seed, cap, off = 3, 2, 0x1234567, 211, 100
+    h2seed = (seed * 0x9E3779B9 + 0x7F4A7C15) & 0xFFFFFFFF
+    tab = np.full((2, cap, 4), 0xFFFFFFFF, dtype=np.uint32)
+    recs = _records_by_hand(out, RM, RN, mask)
+    for rid, rec in recs.items():
+        if rid == 5:                                          # never persisted (missing key)
+            continue
+        key = rid + off                                       # hash stores key on the GLOBAL rid
+        s1, s2 = _fmix32(key ^ seed) % cap, _fmix32(key ^ h2seed) % cap
+        t, s = (1, s2) if (rid == 12 or tab[0, s1, 0] != 0xFFFFFFFF) else (0, s1)   # rid 12 forced into T2
+        assert tab[t, s, 0] == 0xFFFFFFFF
+        tab[t, s] = [key] + rec + [0]
+    def slot_of(key):
+        for t, hs in ((0, seed), (1, h2seed)):
+            s = _fmix32(key ^ hs) % cap
+            if tab[t, s, 0] == key:
+                return t, s
+        return None
+    t9, s9 = slot_of(off + 9)                                 # rid 9: XOR word of its record is wrong
+    tab[t9, s9, 2] ^= 0x10
+    assert slot_of(off + 12)[0] == 1                          # rid 12 lives in T2
+    bad = out.copy()
+    bad.view(np.uint32)[13, 9] ^= np.uint32(1 << 30)         # data of region (3, 2) = local rid 14 changed
+    got = oracle.validate_cuckoo(bad, tab, cap, seed, RM, RN, mask, rid_offset=off)
+    assert list(got) == [105, 109, 114]
+    # the clean image with the completed, correct table validates
+    tab[t9, s9, 2] ^= 0x10
+    s5 = _fmix32(105 ^ seed) % cap
+    t5, s5 = (0, s5) if tab[0, s5, 0] == 0xFFFFFFFF else (1, _fmix32(105 ^ h2seed) % cap)
+    assert tab[t5, s5, 0] == 0xFFFFFFFF
+    tab[t5, s5] = [105] + recs[5] + [0]
+    assert list(oracle.validate_cuckoo(out, tab, cap, seed, RM, RN, mask, rid_offset=off)) == []
+    # keys placed without the offset (a shard that forgot rid_offset) fail every region
+    assert list(oracle.validate_cuckoo(out, tab, cap, seed, RM, RN, mask, rid_offset=0)) == list(range(16))
+
+
+def test_validate_quad_hand_built_table_with_offset():
+    """lpo_validate_quad against a quadratic-probing table placed by hand (home + i^2, L267; Reading R14/R20),
+    global rids = local + 1000: a missing key, a wrong MOD word and a key displaced to its 2nd probe slot."""
+    RM = RN = 8
+    out = gen.generate(22, 32, 16, "uniform", "bf16")   # 4 x 2 regions, local rids 0..7
+    mask, sel, seed, cap, off = 3, 2, 77, 13, 1000
+    tab = np.full((cap, 1 + sel), 0xFFFFFFFF, dtype=np.uint32)
+    recs = _records_by_hand(out, RM, RN, mask)
+    for rid, rec in recs.items():
+        if rid == 6:                                          # never persisted
+            continue
+        key = rid + off
+        h = _fmix32(key ^ seed) % cap
+        for i in range(cap):
+            s = (h + i * i) % cap
+            if tab[s, 0] == 0xFFFFFFFF:
+                tab[s] = [key] + rec
+                break
+    # rid 2's MOD word is wrong
+    h = _fmix32((off + 2) ^ seed) % cap
+    s2 = next((h + i * i) % cap for i in range(cap) if tab[(h + i * i) % cap, 0] == off + 2)
+    tab[s2, 1] += np.uint32(1)
+    got = oracle.validate_quad(out, tab, cap, seed, RM, RN, mask, rid_offset=off)
+    assert list(got) == [1002, 1006]
+    tab[s2, 1] -= np.uint32(1)
+    assert list(oracle.validate_quad(out, tab, cap, seed, RM, RN, mask, rid_offset=off)) == [1006]
+    assert list(oracle.validate_quad(out, tab, cap, seed, RM, RN, mask, rid_offset=0)) == list(range(8))
+
+
+# --------------------------------------------------------------------------- stencil operation order (Reading R19)
+def test_stencil_sum_order_crafted():
+    """((u + d) + l) + r in fp32, then 0.5*c + 0.125*s: a crafted neighbourhood where the four plausible
+    summation orders round differently.  u = 2^24, d = l = 1, r = 2, c = 0 at the centre (1, 1):
+      ((u+d)+l)+r: 2^24+1 -> 2^24 (tie, even), +1 -> 2^24, +2 -> 2^24+2;   * 0.125 -> 2097152.25
+      (u+d)+(l+r): 2^24+3 -> 2^24+4 (tie, even);                            * 0.125 -> 2097152.5
+      ((u+d)+r)+l: 2^24+2, +1 -> 2^24+4 (tie, even);                        * 0.125 -> 2097152.5
+      ((l+r)+u)+d: 3+2^24 -> 2^24+4, +1 -> 2^24+4;                          * 0.125 -> 2097152.5"""
+    x = np.zeros((3, 3), dtype=np.float32)
+    x[0, 1], x[2, 1], x[1, 0], x[1, 2] = 2.0 ** 24, 1.0, 1.0, 2.0
+    assert oracle.stencil5(x)[1, 1] == np.float32(2097152.25)
+    # centre term added after the scaled sum: c = 1 -> 0.5 + 2097152.25 = 2097152.75 (exact, ulp 0.25)
+    x[1, 1] = 1.0
+    assert oracle.stencil5(x)[1, 1] == np.float32(2097152.75)
+    # u and d are the vertical neighbours: swap roles (l = 2^24 horizontally) -> ((1+1)+2^24)+2 = 2^24+2... and
+    # ((u+d)+l)+r with u = d = 1, l = 2^24, r = 2: 2 + 2^24 -> 2^24+2, +2 -> 2^24+4 -> 2097152.5 + 0.5*c
+    y = np.zeros((3, 3), dtype=np.float32)
+    y[0, 1], y[2, 1], y[1, 0], y[1, 2] = 1.0, 1.0, 2.0 ** 24, 2.0
+    assert oracle.stencil5(y)[1, 1] == np.float32(2097152.5)
+
+
+def test_stencil_random_vs_float32_numpy_in_stated_order():
+    """Random fp32 inputs: the oracle equals a numpy float32 evaluation in Reading R19's order (zero outside the
+    domain) element for element -- catches a contraction (FMA), a dropped or doubled neighbour, or an index slip."""
+    x = gen.generate(23, 37, 29, "uniform", "f32") * np.float32(1000.0)
+    p = np.pad(x, 1)
+    u, d, l, r, c = p[:-2, 1:-1], p[2:, 1:-1], p[1:-1, :-2], p[1:-1, 2:], p[1:-1, 1:-1]
+    s = ((u + d) + l) + r
+    ref = np.float32(0.5) * c + np.float32(0.125) * s
+    assert ref.dtype == np.float32
+    assert np.array_equal(oracle.stencil5(x).view(np.uint32), ref.view(np.uint32))
+    alt = np.float32(0.5) * c + np.float32(0.125) * ((u + d) + (l + r))
+    assert not np.array_equal(alt.view(np.uint32), ref.view(np.uint32))   # the input does separate the orders
