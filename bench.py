@@ -9,10 +9,17 @@ batch of the workload:
   the counts] -> a10 selective re-execution -> a11 re-validate -> [all-reduce of
   the summary].
 
-Default workload (N=1) = BASELINE configs[1]: TMM 8192x8192x8192 bf16 -> bf16,
-128x128 regions, MOD|XOR records.  With --gpus N (torchrun, one rank per GPU)
-every rank owns an 8192-row band of a (8192*N) x 8192 output (weak scaling,
-region-row sharding).
+Default workload (N=1) = BASELINE configs[3] (C4): 5-point stencil 32768 x 32768
+fp32 -> fp32 (the paper's 32-bit data, L199/L546; 4 GiB per array, the largest
+single-GPU config), 128x128 regions, MOD|XOR records, 10% of the regions
+corrupted.  With --gpus N every rank owns a 32768-row band of a (32768*N) x 32768
+domain (weak scaling, region-row sharding); the band's input keeps
+its two halo rows (read-only input, generated per rank: no data exchange), and
+the only collective is the NCCL all-reduce of the int64 counts.  When
+WORLD_SIZE is unset and --gpus N > 1, bench.py re-launches itself under
+torch.distributed.run with N ranks.  Other workloads (--workload): the C2 TMM
+8192^3 (bf16 / fp32 via 3xTF32 / checksum sweep), C3 store ablation, C5 TMM
+65536^3, the paper's int32 TMM and the SpMV class.
 
 Reported:
   value      validate+recover throughput, GB/s, summed over ranks / max-rank
@@ -61,9 +68,12 @@ WORKLOADS = {
                              cksum="mod|xor", frac=0.05, store="array", weak=True),
     "tmm8192_bf16_f32out": dict(kind="tmm", M=8192, N=8192, K=8192, in_dt="bf16", out_dt="f32", region=128,
                                 cksum="mod|xor", frac=0.05, store="array", weak=True),
-    # BASELINE configs[3]: stencil 32768^2 fp32, 128x128 regions, 10% injection
+    # BASELINE configs[3] (N=1 default): stencil 32768^2 fp32, 128x128 regions, 10% injection; weak-scaled by
+    # 32768-row bands under torchrun
     "stencil32768": dict(kind="stencil", M=32768, N=32768, K=0, in_dt="f32", out_dt="f32", region=128,
-                         cksum="mod|xor", frac=0.10, store="array", weak=False),
+                         cksum="mod|xor", frac=0.10, store="array", weak=True),
+    "stencil32768_adler": dict(kind="stencil", M=32768, N=32768, K=0, in_dt="f32", out_dt="f32", region=128,
+                               cksum="mod|xor|adler", frac=0.10, store="array", weak=True),
     # BASELINE configs[2]: store ablation on TMM 16384^3
     "tmm16384_array": dict(kind="tmm", M=16384, N=16384, K=16384, in_dt="bf16", out_dt="bf16", region=128,
                            cksum="mod|xor", frac=0.05, store="array", weak=False),
@@ -118,7 +128,7 @@ def parse():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="process-group backend for N>1 (gloo + --same-device: test the N>1 path on one GPU)")
     ap.add_argument("--same-device", action="store_true", help="test hook: put every rank on cuda:0")
-    ap.add_argument("--workload", default="tmm8192_bf16", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="stencil32768", choices=sorted(WORKLOADS))
     ap.add_argument("--overhead-reps", type=int, default=20)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the cpu_baseline sample")
@@ -147,6 +157,7 @@ class ClockSampler:
     def __init__(self, index: int):
         self.index = index
         self.samples = []
+        self.stamped = []
         self.reasons = set()
         self.stop_flag = False
         self.t = None
@@ -171,7 +182,9 @@ class ClockSampler:
         nv = self.nvml
         while not self.stop_flag:
             try:
-                self.samples.append(nv.nvmlDeviceGetClockInfo(self.handle, nv.NVML_CLOCK_SM))
+                mhz = nv.nvmlDeviceGetClockInfo(self.handle, nv.NVML_CLOCK_SM)
+                self.samples.append(mhz)
+                self.stamped.append((time.perf_counter(), mhz))
                 r = nv.nvmlDeviceGetCurrentClocksEventReasons(self.handle)
                 for name, bit in self.REASONS.items():
                     if r & bit:
@@ -179,6 +192,11 @@ class ClockSampler:
             except Exception:
                 pass
             time.sleep(0.01)
+
+    def median_between(self, t0, t1):
+        """Median SM clock of the samples taken in [t0, t1] (host perf_counter), or None."""
+        xs = [m for t, m in list(self.stamped) if t0 <= t <= t1]
+        return statistics.median(xs) if xs else None
 
     def wait_first(self, timeout=2.0):
         t0 = time.time()
@@ -204,6 +222,43 @@ def peaks():
             d = json.load(f)
         return d["hbm_gbs"], d["bf16_tflops"], d.get("bf16_tflops_sustained"), "measured"
     return 6650.0, 1590.0, 1400.0, "fallback (B200_PROFILING.md)"
+
+
+def measure_tf32_peak(dev, long_kernel=False):
+    """TF32 dense tensor peak, measured here: cuBLAS fp32 GEMM 8192^3 with TF32 allowed (torch.matmul), best of
+    10 CUDA-event timings (burst); for a multi-ms kernel timed inside a long run, the same GEMM back to back for
+    ~3 s (sustained, median of the last half).  Returns (TFLOP/s, description)."""
+    import torch
+
+    prev = torch.backends.cuda.matmul.allow_tf32
+    torch.backends.cuda.matmul.allow_tf32 = True
+    try:
+        n = 8192
+        x = torch.randn((n, n), device=dev, dtype=torch.float32)
+        y = torch.randn((n, n), device=dev, dtype=torch.float32)
+        z = torch.empty((n, n), device=dev, dtype=torch.float32)
+        for _ in range(3):
+            torch.matmul(x, y, out=z)
+        ts = []
+        t_end = time.perf_counter() + (3.0 if long_kernel else 0.0)
+        while len(ts) < 10 or time.perf_counter() < t_end:
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            torch.matmul(x, y, out=z)
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        flop = 2.0 * n ** 3
+        if long_kernel:
+            t = statistics.median(ts[len(ts) // 2:])
+            how = "sustained: median of the last half of ~3 s back to back"
+        else:
+            t = min(ts)
+            how = "burst: best of 10"
+        return flop / (t * 1e-3) / 1e12, (f"measured in this run: cuBLAS fp32 GEMM 8192^3 with TF32 allowed "
+                                          f"(torch.matmul), {how}")
+    finally:
+        torch.backends.cuda.matmul.allow_tf32 = prev
 
 
 def ncu_traffic(kernel_key: str, workload: str):
@@ -279,15 +334,18 @@ def run_ours(args):
         wl = lp.Workload.spmv(vals_d, x_d.view(-1), rp_d, cols_d)
         body_flops = 2.0 * float(rp_host[-1])
     else:
-        gM = W["M"]
-        if world > 1:
-            raise SystemExit("stencil workload is single-GPU (no halo exchange in round 1)")
-        sh = shard.plan(gM, W["N"], RM, RN, 1, 0)
-        M, N, K = W["M"], W["N"], 0
-        a = torch.empty((M, N), dtype=torch.float32, device=dev)
-        lpsynth.device_fill(a, 1, "uniform", "f32")
+        # row band of a (M * world) x N domain; the band's input keeps its halo rows (the neighbouring ranks'
+        # boundary rows of the read-only input, generated here from the same counter formula: no exchange)
+        gM = W["M"] * (world if W["weak"] else 1)
+        sh = shard.plan(gM, W["N"], RM, RN, world, rank)
+        M, N, K = sh.rows, W["N"], 0
+        lo = max(0, sh.row_offset - 1)
+        hi = min(gM, sh.row_offset + M + 1)
+        band = torch.empty((hi - lo, N), dtype=torch.float32, device=dev)
+        lpsynth.device_fill(band, 1, "uniform", "f32", row0=lo, ncols_global=N)
+        a = band[sh.row_offset - lo:sh.row_offset - lo + M]
         b = None
-        wl = lp.Workload.stencil(a)
+        wl = lp.Workload.stencil(a, row_offset=sh.row_offset, global_m=gM)
         body_flops = 0.0
     h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
               shuffle=not args.no_shuffle, pairing=not args.no_pairing, recover_slices=not args.recover_tile128)
@@ -470,9 +528,17 @@ def run_ours(args):
         t_validate = report.median(diffs)
         del gs
 
-    # ---- LP overhead: protected vs unprotected twin, interleaved, cold L2
-    tp, tu = [], []
+    # ---- LP overhead: protected vs unprotected twin, interleaved, cold L2.  Every protected rep starts from a
+    # freshly initialised table (a hash store then measures fresh-table inserts, as Fig. 5 / Table IV do); the
+    # twin gets a memset of the same size on a scratch buffer, so both sides do identical untimed preparation.
+    ck_twin_scratch = torch.empty_like(ck)
+    tp, tu, pair_clk = [], [], []
     for i in range(args.overhead_reps * 2):
+        if i % 2 == 0:
+            h.cksum_init(wl, ck)
+            tw0 = time.perf_counter()
+        else:
+            ck_twin_scratch.fill_(-1)
         l2_flush()
         e0, e1 = ev(), ev()
         if i % 2 == 0:
@@ -485,10 +551,22 @@ def run_ours(args):
             e1.record(st)
         torch.cuda.synchronize()
         (tp if i % 2 == 0 else tu).append(e0.elapsed_time(e1))
+        if i % 2 == 1:
+            pair_clk.append(clk.median_between(tw0, time.perf_counter()))
     t_prot, t_unprot = report.median(tp), report.median(tu)
     # overhead from adjacent (protected, unprotected) pairs: robust to clock drift under the power cap
     pair_ratios = [a / b for a, b in zip(tp, tu)]
     overhead_pairs = 100.0 * (report.median(pair_ratios) - 1.0)
+    q25, q75 = report.quantile(pair_ratios, 0.25), report.quantile(pair_ratios, 0.75)
+    pclk = [c for c in pair_clk if c is not None]
+    overhead_detail = {
+        "pairs": len(pair_ratios),
+        "iqr_pct": [round(100.0 * (q25 - 1.0), 3), round(100.0 * (q75 - 1.0), 3)],
+        "t_protected_ms_min_max": [round(min(tp), 4), round(max(tp), 4)],
+        "t_unprotected_ms_min_max": [round(min(tu), 4), round(max(tu), 4)],
+        "pair_sm_mhz_min_median_max": ([min(pclk), statistics.median(pclk), max(pclk)] if pclk else None),
+        "table_init": "cksum_init before every protected rep (fresh table), same-size memset before every twin rep",
+    }
     clocks = clk.stop()
     # hash-store statistics of one fresh protected run (collisions = sum of extra probes, Table II analog)
     d_stats = torch.zeros(2, dtype=torch.int64, device=dev)
@@ -545,6 +623,9 @@ def run_ours(args):
     value = bytes_vr_total * args.steps / (sum_vr * 1e-3) / 1e9
     e2e_value = bytes_vr_total / (t_e2e * 1e-3) / 1e9
     hbm, bf16, bf16_s, peak_src = peaks()
+    tf32_peak_measured = None
+    if rank == 0 and W["kind"] == "tmm" and W["in_dt"] == "f32" and W.get("body") != "simt":
+        tf32_peak_measured = measure_tf32_peak(dev, long_kernel=t_prot > 2.0)
 
     line = None
     if rank == 0:
@@ -562,13 +643,19 @@ def run_ours(args):
         elif W["kind"] == "tmm":
             if W.get("body") == "simt":
                 kname = "tmm_simt_kernel"
-                # FP32 FFMA peak: 148 SMs x 128 FMA/clk x 2 flop x max SM clock (guide unit counts);
-                # the int32 body uses IMAD on the same pipe (taken at the same rate)
-                peak = 148 * 128 * 2 * 1.965e9 / 1e12
+                if W["in_dt"] == "i32":
+                    # int32 multiply-add runs as IMAD at half the FFMA rate: 64 per SM per clock
+                    peak = 148 * 64 * 2 * 1.965e9 / 1e12
+                    psrc = "derived: 148 SM x 64 IMAD/clk (half the FFMA rate) x 2 x 1965 MHz"
+                else:
+                    # FP32 FFMA peak: 148 SMs x 128 FMA/clk x 2 flop x max SM clock (guide unit counts)
+                    peak = 148 * 128 * 2 * 1.965e9 / 1e12
+                    psrc = "derived: 148 SM x 128 FP32 FMA/clk x 2 x 1965 MHz"
                 achieved = body_flops / (t_prot * 1e-3) / 1e12
                 roof = {"bound": "alu", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 2),
-                        "peak": round(peak, 1), "unit": "TFLOP/s", "frac": round(achieved / peak, 4),
-                        "peak_source": "derived: 148 SM x 128 FP32 FMA/clk x 2 x 1965 MHz",
+                        "peak": round(peak, 1), "unit": "TOP/s" if W["in_dt"] == "i32" else "TFLOP/s",
+                        "frac": round(achieved / peak, 4),
+                        "peak_source": psrc,
                         "algorithmic_per_launch": f"2*M*N*K = {body_flops:.4g} flop",
                         "traffic": ncu_traffic(kname, args.workload)}
             elif W["in_dt"] == "bf16":
@@ -587,20 +674,18 @@ def run_ours(args):
             else:
                 kname = "tmm_tf32x3_kernel"
                 achieved = 3.0 * body_flops / (t_prot * 1e-3) / 1e12   # 3 tf32 MMAs per fp32 MAC
-                base = bf16_s if (t_prot > 2.0 and bf16_s is not None and achieved <= 0.5 * bf16_s) else bf16
-                tf32_peak = base * (1.125 / 2.25)   # measured bf16 x nominal tf32/bf16 dense ratio (guide table)
+                tf32_peak, tf32_src = tf32_peak_measured
                 roof = {"bound": "tensor", "kernel": f"{kname} (protected, {W['cksum']})", "achieved": round(achieved, 1),
                         "peak": round(tf32_peak, 1), "unit": "TFLOP/s (tf32 tensor work)",
                         "frac": round(achieved / tf32_peak, 4),
-                        "peak_source": f"{peak_src} bf16 {'sustained' if base != bf16 else 'burst'} x 0.5 "
-                                       "(nominal tf32/bf16 dense ratio)",
+                        "peak_source": tf32_src,
                         "algorithmic_per_launch": f"3 x 2*M*N*K = {3 * body_flops:.4g} tf32 flop "
                                                   f"(fp32-equivalent {body_flops / (t_prot * 1e-3) / 1e12:.1f} TFLOP/s)",
                         "traffic": ncu_traffic(kname, args.workload)}
         else:
             sb = 2.0 * out_bytes
             achieved = sb / (t_prot * 1e-3) / 1e9
-            roof = {"bound": "hbm", "kernel": "stencil5_ldg_kernel (protected, MOD|XOR)", "achieved": round(achieved, 1),
+            roof = {"bound": "hbm", "kernel": f"stencil5_ldg_kernel (protected, {W['cksum']})", "achieved": round(achieved, 1),
                     "peak": hbm, "unit": "GB/s", "frac": round(achieved / hbm, 4),
                     "peak_source": f"{peak_src} HBM copy", "algorithmic_per_launch": f"8 B/elem = {sb:.4g} B",
                     "traffic": ncu_traffic("stencil5_ldg_kernel", args.workload)}
@@ -623,12 +708,13 @@ def run_ours(args):
             "config": {"workload": args.workload, "M_global": gM, "N": N, "K": K, "region": [RM, RN],
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
-                       "recovery": recovery_desc(args, RM),
+                       "recovery": recovery_desc(args, RM, W),
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write, then 2x L2 read of another buffer: clean lines) before every recovery phase and every isolated kernel rep",
                        "launch": "CUDA graph replay per step segment" if args.graph else "eager"},
             "lp_overhead_pct": round(overhead_pairs, 3),
             "lp_overhead_pct_of_medians": round(report.overhead_pct(t_prot, t_unprot), 3),
+            "lp_overhead_detail": overhead_detail,
             "lp_overhead_method": f"median over {len(pair_ratios)} adjacent (protected, unprotected) run pairs of "
                                   "t_prot/t_unprot - 1, L2 flushed before every run",
             "t_protected_ms": round(t_prot, 4),
@@ -828,7 +914,11 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
-def recovery_desc(args, RM):
+def recovery_desc(args, RM, W):
+    if W["kind"] == "stencil":
+        return "failed 128x128 regions re-executed in list mode by persistent CTAs (one region per CTA pass)"
+    if W["kind"] == "spmv" or W.get("body") == "simt":
+        return "failed regions re-executed in list mode (one region per CTA pass)"
     if args.no_pairing:
         return "one 128x128 tile per failed tile"
     if RM == 32 and not args.recover_tile128:
@@ -836,8 +926,26 @@ def recovery_desc(args, RM):
     return "same-row failed tiles paired into 128x256 tasks (when > #SM)"
 
 
+def self_launch(args) -> int:
+    """`python bench.py --gpus N` with N > 1 outside torchrun: re-run this command under torch.distributed.run
+    with N ranks on this node (rendezvous on 127.0.0.1, a free port); returns its exit code."""
+    import socket
+
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        port = so.getsockname()[1]
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd, cwd=ROOT)
+
+
 def main():
     args = parse()
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        sys.exit(self_launch(args))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}: launch one rank per GPU")
     if args.impl == "reference":
         run_reference(args)
     else:

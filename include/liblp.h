@@ -152,7 +152,11 @@ typedef struct {
   int64_t ldb;
   int64_t ldc;       /* out row pitch in elements */
   int64_t row_offset, global_m; /* shard: rows [row_offset, row_offset+m) of global_m.
-                                   STENCIL5 requires row_offset = 0, global_m = m. */
+                                   STENCIL5 shards: a points at the input element of global row
+                                   row_offset, column 0; the halo rows a - lda (when row_offset > 0) and
+                                   a + m*lda (when row_offset + m < global_m) must be readable -- they are
+                                   the neighbouring shards' boundary rows, which the caller holds (the
+                                   input is read-only, so no exchange happens inside liblp). */
   /* SPMV only (ignored otherwise): m = rows of A (= length of y = out), n = columns
    * (= length of x = b), a = values (f32 [nnz]), b = x (f32 [n]), row_ptr (int64
    * [m + 1], absolute offsets into a / col_idx for this shard's rows), col_idx

@@ -121,7 +121,6 @@ lp_status check_wl(const lp_ctx* h, const lp_workload_t* wl, lp::RegionGeom* g) 
     if (wl->k <= 0) return fail(LP_ERR_INVALID_ARG, "k must be positive");
   } else {
     if (wl->in_dtype != LP_F32 || wl->out_dtype != LP_F32) return fail(LP_ERR_UNSUPPORTED, "stencil is fp32 -> fp32");
-    if (wl->row_offset != 0 || wl->global_m != wl->m) return fail(LP_ERR_UNSUPPORTED, "stencil shards are not supported");
   }
   g->M = wl->m;
   g->N = wl->n;
@@ -220,6 +219,13 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
 
 size_t workspace_bytes(const lp::RegionGeom& g) { return ws_layout(g).total; }
 
+// Row shard of the stencil: the caller's input pointer is the shard's first row; the halo rows
+// above / below exist (and are read) only where the global domain continues (zero padding outside).
+void stencil_rows(const lp_workload_t* wl, lp::StencilArgs* a) {
+  a->row_lo = wl->row_offset > 0 ? -1 : 0;
+  a->row_span = (int)(wl->m + (wl->row_offset + wl->m < wl->global_m ? 1 : 0) - a->row_lo);
+}
+
 // Body dispatch shared by run_protected and recover (list = null for a full run).
 lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
                    const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr) {
@@ -238,6 +244,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.ldo = wl->ldc;
     a.H = wl->m;
     a.W = wl->n;
+    stencil_rows(wl, &a);
     a.RM = g.RM;
     a.RN = g.RN;
     a.mask = h->mask;
@@ -530,6 +537,7 @@ lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void
   a.ldo = wl->ldc;
   a.H = wl->m;
   a.W = wl->n;
+  stencil_rows(wl, &a);
   a.RM = g.RM;
   a.RN = g.RN;
   a.mask = h->mask;

@@ -101,6 +101,8 @@ struct StencilArgs {
   float* out;
   int64_t ldo;
   int64_t H, W;
+  int row_lo, row_span;  // readable input rows, relative to this shard's first row: [row_lo, row_lo + row_span)
+                         // = the shard plus its halo rows inside the global domain (zero outside it)
   int RM, RN;
   uint32_t mask;
   HashInfo hash;

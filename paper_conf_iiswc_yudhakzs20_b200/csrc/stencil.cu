@@ -59,7 +59,8 @@ __device__ __forceinline__ float ldg_nc_f(const float* p) {
 
 template <uint32_t MASK, int STORE, int COMBINE>
 __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __restrict__ in, int64_t ldi,
-                                                              float* __restrict__ out, int64_t ldo, int H, int W,
+                                                              float* __restrict__ out, int64_t ldo, int row_lo,
+                                                              int row_span, int W,
                                                               int64_t Q, int64_t R, uint32_t* __restrict__ ck,
                                                               int64_t rid_offset, const int64_t* __restrict__ list,
                                                               const int64_t* __restrict__ d_n) {
@@ -116,7 +117,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
 #pragma unroll
     for (int r = 0; r < kRowsW + 2; ++r) {
       const int i = i0 - 1 + r;
-      v[r] = ((unsigned)i < (unsigned)H) ? ldg_nc_v4(in + (int64_t)i * ldi + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+      v[r] = ((unsigned)(i - row_lo) < (unsigned)row_span) ? ldg_nc_v4(in + (int64_t)i * ldi + j) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
 #pragma unroll
     for (int r = 0; r < kRowsW; ++r) edge[r] = eok ? ldg_nc_f(in + (int64_t)(i0 + r) * ldi + je) : 0.f;
@@ -198,12 +199,12 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
 #define LP_LCASE(M, S)                                                                                          \
   case M * 5 + S:                                                                                               \
     if (a.list)                                                                                                 \
-      stencil5_ldg_kernel<M, S, 0><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H,         \
-                                                                   (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
+      stencil5_ldg_kernel<M, S, 0><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo,          \
+                                                                   a.row_span, (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
                                                                    a.d_n);                                      \
     else                                                                                                        \
-      stencil5_ldg_kernel<M, S, 1><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H,         \
-                                                                   (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
+      stencil5_ldg_kernel<M, S, 1><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo,          \
+                                                                   a.row_span, (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
                                                                    a.d_n);                                      \
     break;
 #define LP_LCASE3(M) LP_LCASE(M, 0)
@@ -234,7 +235,8 @@ cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recove
   switch (a.mask * 5 + sk) {
 #define LP_CCASE(M, S)                                                                                          \
   case M * 5 + S:                                                                                               \
-    stencil5_ldg_kernel<M, S, 2><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, (int)a.H, (int)a.W, Q,  \
+    stencil5_ldg_kernel<M, S, 2><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo, a.row_span,  \
+                                                              (int)a.W, Q,                                      \
                                                               R, a.ck, a.rid_offset, nullptr, d_recovered);     \
     break;
 #define LP_CCASE3(M) LP_CCASE(M, 0)

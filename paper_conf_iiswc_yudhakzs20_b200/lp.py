@@ -188,13 +188,16 @@ class Workload:
                         global_m if global_m is not None else row_offset + m)
 
     @staticmethod
-    def stencil(inp, H=None, W=None) -> "Workload":
+    def stencil(inp, H=None, W=None, row_offset=0, global_m=None) -> "Workload":
+        """out = 5-point stencil of inp (Reading R19).  Row shard: inp = rows [row_offset, row_offset + H) of a
+        global_m-row input, as a view whose neighbouring rows (the halo) are readable where the domain continues."""
         if inp is not None:
             H, W = inp.shape
             lda = inp.stride(0)
         else:
             lda = W
-        return Workload(WL_STENCIL5, H, W, 0, inp, None, F32, F32, lda, 0, W, 0, H)
+        return Workload(WL_STENCIL5, H, W, 0, inp, None, F32, F32, lda, 0, W, row_offset,
+                        global_m if global_m is not None else row_offset + H)
 
     @staticmethod
     def spmv(values, x, row_ptr, col_idx, m=None, row_offset=0, global_m=None) -> "Workload":

@@ -30,3 +30,14 @@ def median(xs):
     s = sorted(xs)
     n = len(s)
     return s[n // 2] if n % 2 else 0.5 * (s[n // 2 - 1] + s[n // 2])
+
+
+def quantile(xs, q: float) -> float:
+    """Linear-interpolation quantile (numpy's default 'linear' method), q in [0, 1]."""
+    s = sorted(xs)
+    if not s:
+        raise ValueError("empty sample")
+    pos = q * (len(s) - 1)
+    lo = int(math.floor(pos))
+    hi = min(lo + 1, len(s) - 1)
+    return s[lo] + (s[hi] - s[lo]) * (pos - lo)

@@ -19,7 +19,8 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 def test_two_rank_bench_same_device():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", "29541", "bench.py", "--gpus", "2", "--steps", "2",
-           "--warmup", "3", "--overhead-reps", "2", "--no-cpu-baseline", "--dist-backend", "gloo", "--same-device"]
+           "--warmup", "3", "--overhead-reps", "2", "--no-cpu-baseline", "--dist-backend", "gloo", "--same-device",
+           "--workload", "tmm8192_bf16"]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
@@ -30,6 +31,24 @@ def test_two_rank_bench_same_device():
     assert d["n_failed_per_step"] == 2 * round(0.05 * d["config"]["regions_per_rank"])
     assert d["value"] > 0 and d["roofline"]["achieved"] > 0
     assert d["per_rank"]["n_failed"]["min"] == d["per_rank"]["n_failed"]["max"] == round(0.05 * d["config"]["regions_per_rank"])
+
+
+def test_self_launch_two_rank_stencil_same_device():
+    """`python bench.py --gpus 2` without torchrun re-launches itself with 2 ranks; default
+    workload = C4 stencil, weak-scaled by 32768-row bands with read-only halo rows."""
+    cmd = [sys.executable, "bench.py", "--gpus", "2", "--steps", "2", "--warmup", "3", "--overhead-reps", "2",
+           "--no-cpu-baseline", "--dist-backend", "gloo", "--same-device"]
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["n_failed_after_recover"] == 0 and d["scaling"] == "weak"
+    assert d["config"]["workload"] == "stencil32768" and d["config"]["M_global"] == 65536
+    assert d["config"]["regions_per_rank"] == 256 * 256
+    assert d["n_failed_per_step"] == 2 * round(0.10 * 256 * 256)
+    assert d["dtype"].startswith("f32->f32")
 
 
 def test_inject_skips_rids_of_other_shards():

@@ -103,3 +103,42 @@ def test_same_grid_check_and_recover(frac, store):
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0
+
+
+@pytest.mark.parametrize("shard", [0, 1, 2, 3])
+def test_stencil_row_shard(shard):
+    """Row shard s of 4 (SURVEY §8e for the stencil): the shard's input view keeps the neighbouring rows
+    readable as its halo; its output rows, records (GLOBAL rids) and the failed set after injection equal the
+    oracle's on the full domain's rows [s*H/4, (s+1)*H/4); recovery restores the golden bytes."""
+    H, W, G = 1024, 512, 4
+    m = H // G
+    r0 = shard * m
+    X = gen.generate(9, H, W, "uniform", "f32")
+    full_in = host_to_dev(X, "f32")
+    x = full_in[r0:r0 + m]                                  # view into the full input: halo rows readable
+    h = lp.LP(128, 128, cksum="mod|xor")
+    wl = lp.Workload.stencil(x, row_offset=r0, global_m=H)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = host_to_dev(gen.generate(509, m, W, "bits", "f32"), "f32")
+    out.copy_(stale)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    torch.cuda.synchronize()
+    golden = dev_to_host(out)
+    exp_out = oracle.stencil5_block(X, r0, 0, m, W)
+    assert np.array_equal(golden.view(np.uint32), exp_out.view(np.uint32))
+    R = h.num_regions(wl)
+    assert np.array_equal(dev_to_host(ck)[:R * 2].reshape(R, 2), oracle.records(exp_out, 128, 128, 3))
+    rid0 = (r0 // 128) * (W // 128)
+    inj = torch.from_numpy(lp.choose_regions(R, 0.3, 77 + shard) + rid0).cuda()   # global rids
+    h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=77)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    nf = int(d_n.item())
+    exp = oracle.validate_array(dev_to_host(out), dev_to_host(ck)[:R * 2], 128, 128, 3, rid_offset=rid0)
+    assert nf > 0 and np.array_equal(failed[:nf].cpu().numpy(), exp)
+    h.recover(wl, out, ck, failed, d_n, ws)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+    assert np.array_equal(dev_to_host(out).view(np.uint32), golden.view(np.uint32))

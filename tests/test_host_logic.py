@@ -180,3 +180,31 @@ def test_spmv_and_stencil_shape_errors():
     h3 = lp.LP(1, 1024, cksum="mod")
     assert _status(lambda: h3.num_regions(lp.Workload.spmv(None, None, None, None, m=1000))) == lp.LP_ERR_INVALID_ARG
     assert h3.num_regions(lp.Workload.spmv(None, None, None, None, m=4096)) == 4
+
+
+def test_quantile_matches_numpy():
+    import numpy as np
+    rng = np.random.default_rng(3)
+    for n in [1, 2, 5, 40]:
+        xs = rng.standard_normal(n).tolist()
+        for q in [0.0, 0.25, 0.5, 0.75, 1.0]:
+            assert report.quantile(xs, q) == pytest.approx(float(np.quantile(xs, q)))
+
+
+def test_bench_self_launch_reference_two_ranks():
+    """`bench.py --impl reference --gpus 2` outside torchrun re-launches itself with 2 ranks; rank 0 alone runs the
+    oracle and prints one line, the other rank exits 0 (no GPU needed)."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = {k: v for k, v in os.environ.items() if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK")}
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--steps", "1",
+                        "--warmup", "0", "--workload", "tmm8192_bf16"], cwd=root, capture_output=True, text=True,
+                       timeout=300, env=env)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["value"] > 0
