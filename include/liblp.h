@@ -229,11 +229,19 @@ LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, voi
                             const int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 
 /* The paper's own recovery form (Listing 7; NEXT row N2): ONE kernel
- * with the grid of the original kernel, in which every CTA validates its region
- * and, if the check fails, re-executes the region in place (data and record).
- * *d_n_recovered (device int64, zeroed by the call) receives the number of
- * re-executed regions.  No failed list is produced.  STENCIL5 workloads only
- * (LP_ERR_UNSUPPORTED otherwise). */
+ * with the grid of the original kernel, in which every CTA validates its regions
+ * and, if a check fails, re-executes in place (data and record).
+ * *d_n_recovered (device int64, zeroed by the call) receives the number of failed
+ * (re-executed) regions.  No failed list is produced.
+ *  - STENCIL5: one CTA per region.
+ *  - TMM (bf16 input, tcgen05 CTA-pair body: m, n % 256 == 0, k % 64 == 0,
+ *    128x128 or 32x32 regions): the persistent CTA pairs walk the tile schedule of
+ *    lp_run_protected; each CTA first validates its 128-row halves of its pair's
+ *    256x256 tiles (all warps, coalesced streaming reads), the pair merges its two
+ *    failed-tile bitmasks through distributed shared memory, and the pair's
+ *    TMA/MMA/epilogue pipeline then recomputes only the tiles holding a failed
+ *    region (every region of such a tile is rewritten with identical bits).
+ * Other workloads / bodies: LP_ERR_UNSUPPORTED. */
 LP_API lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
                                   int64_t* d_n_recovered, lp_stream_t stream);
 

@@ -226,6 +226,39 @@ void stencil_rows(const lp_workload_t* wl, lp::StencilArgs* a) {
   a->row_span = (int)(wl->m + (wl->row_offset + wl->m < wl->global_m ? 1 : 0) - a->row_lo);
 }
 
+lp::TmmArgs tmm_args(const lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
+                     const int64_t* list, const int64_t* d_n) {
+  lp::TmmArgs a;
+  a.A = wl->a;
+  a.lda = wl->lda;
+  a.B = wl->b;
+  a.ldb = wl->ldb;
+  a.C = out;
+  a.ldc = wl->ldc;
+  a.M = wl->m;
+  a.N = wl->n;
+  a.K = wl->k;
+  a.in_bf16 = wl->in_dtype == LP_BF16;
+  a.out_bf16 = wl->out_dtype == LP_BF16;
+  a.i32 = wl->in_dtype == LP_I32;
+  a.RM = g.RM;
+  a.RN = g.RN;
+  a.mask = h->mask;
+  a.hash = hash_info(h, g);
+  a.ck = (uint32_t*)ck;
+  a.rid_offset = g.rid_offset;
+  a.list = list;
+  a.d_n = d_n;
+  a.list_is_tiles = 0;
+  a.slice64 = 0;
+  a.tasks = nullptr;
+  a.d_ntasks = nullptr;
+  a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
+  a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
+  a.sm_count = h->sm_count;
+  return a;
+}
+
 // Body dispatch shared by run_protected and recover (list = null for a full run).
 lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
                    const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr) {
@@ -285,34 +318,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
   }
   if (!wl->a || !wl->b) return fail(LP_ERR_INVALID_ARG, "null A or B");
   if (wl->lda < wl->k || wl->ldb < wl->n) return fail(LP_ERR_INVALID_ARG, "lda < k or ldb < n");
-  lp::TmmArgs a;
-  a.A = wl->a;
-  a.lda = wl->lda;
-  a.B = wl->b;
-  a.ldb = wl->ldb;
-  a.C = out;
-  a.ldc = wl->ldc;
-  a.M = wl->m;
-  a.N = wl->n;
-  a.K = wl->k;
-  a.in_bf16 = wl->in_dtype == LP_BF16;
-  a.out_bf16 = wl->out_dtype == LP_BF16;
-  a.i32 = wl->in_dtype == LP_I32;
-  a.RM = g.RM;
-  a.RN = g.RN;
-  a.mask = h->mask;
-  a.hash = hi;
-  a.ck = (uint32_t*)ck;
-  a.rid_offset = g.rid_offset;
-  a.list = list;
-  a.d_n = d_n;
-  a.list_is_tiles = 0;
-  a.slice64 = 0;
-  a.tasks = nullptr;
-  a.d_ntasks = nullptr;
-  a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
-  a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
-  a.sm_count = h->sm_count;
+  lp::TmmArgs a = tmm_args(h, wl, g, out, ck, list, d_n);
   const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, wl->lda, wl->ldb, wl->ldc,
                                           wl->a, wl->b, out);
   const bool tf_ok = !a.i32 && lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, a.in_bf16, a.out_bf16,
@@ -523,9 +529,29 @@ lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void
   lp::RegionGeom g;
   lp_status s = check_wl(h, wl, &g);
   if (s) return s;
-  if (wl->kind != LP_WL_STENCIL5) return fail(LP_ERR_UNSUPPORTED, "same-grid check-and-recover: STENCIL5 only");
+  if (wl->kind == LP_WL_SPMV) return fail(LP_ERR_UNSUPPORTED, "same-grid check-and-recover: STENCIL5 and TMM only");
   if (h->mask == 0) return fail(LP_ERR_STATE, "check-and-recover needs a checksum (cfg.cksum != 0)");
   if (!out || !cksum || !d_n_recovered || !wl->a) return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (wl->kind == LP_WL_TMM) {
+    if (!wl->b) return fail(LP_ERR_INVALID_ARG, "null B");
+    if (wl->lda < wl->k || wl->ldb < wl->n) return fail(LP_ERR_INVALID_ARG, "lda < k or ldb < n");
+    if (h->cfg.body == LP_BODY_SIMT || (h->cfg.flags & (LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE)) ||
+        !lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, wl->in_dtype == LP_BF16, wl->lda, wl->ldb, wl->ldc,
+                              wl->a, wl->b, out) ||
+        !lp::tmm_tc_check_supported(wl->m, wl->n))
+      return fail(LP_ERR_UNSUPPORTED,
+                  "TMM check-and-recover runs on the tcgen05 CTA-pair body: bf16 input, m, n %% 256 == 0, k %% 64 == 0, "
+                  "128x128 or 32x32 regions");
+    if (!aligned16(cksum)) return fail(LP_ERR_INVALID_ARG, "cksum must be 16-B aligned");
+    if ((s = check_device(h))) return s;
+    DeviceGuard dg(h->cfg.device);
+    const lp::TmmArgs a = tmm_args(h, wl, g, out, cksum, nullptr, nullptr);
+    const char* why = nullptr;
+    cudaError_t e = lp::launch_tmm_tc_check_recover(a, d_n_recovered, (cudaStream_t)stream, &why);
+    if (e != cudaSuccess) return why ? fail(LP_ERR_UNSUPPORTED, "check-and-recover: %s", why) : cuda_fail(e, "check-and-recover launch");
+    if ((s = cuckoo_rehash(h, cksum, (cudaStream_t)stream))) return s;
+    return ok();
+  }
   if (!lp::stencil_supported(g.RM, g.RN)) return fail(LP_ERR_UNSUPPORTED, "stencil supports 128x128 regions");
   if (!aligned16(wl->a) || !aligned16(out) || (wl->lda * 4) % 16) return fail(LP_ERR_INVALID_ARG, "stencil buffers must be 16-B aligned");
   if ((s = check_device(h))) return s;

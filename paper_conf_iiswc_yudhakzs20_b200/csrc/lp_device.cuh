@@ -91,6 +91,23 @@ __device__ __forceinline__ CkRecord warp_reduce(const CkPartial<MASK>& p, uint32
   return r;
 }
 
+// Reduction over aligned groups of 2^lg_log2 lanes (every lane of a group ends with its group's record).
+template <uint32_t MASK>
+__device__ __forceinline__ CkRecord segment_reduce(const CkPartial<MASK>& p, int lg_log2) {
+  if (lg_log2 == 5) return warp_reduce<MASK>(p);
+  CkRecord r{p.mod, p.xr, p.s, 0u};
+  if constexpr ((MASK & kAdler) != 0) r.wmod = (uint32_t)(p.w % kAdlerBase);
+  for (int o = (1 << lg_log2) >> 1; o > 0; o >>= 1) {
+    if constexpr ((MASK & kMod) != 0) r.mod += __shfl_xor_sync(0xFFFFFFFFu, r.mod, o);
+    if constexpr ((MASK & kXor) != 0) r.xr ^= __shfl_xor_sync(0xFFFFFFFFu, r.xr, o);
+    if constexpr ((MASK & kAdler) != 0) {
+      r.s += __shfl_xor_sync(0xFFFFFFFFu, r.s, o);
+      r.wmod += __shfl_xor_sync(0xFFFFFFFFu, r.wmod, o);
+    }
+  }
+  return r;
+}
+
 __device__ __forceinline__ CkRecord combine(CkRecord a, const CkRecord& b) {
   a.mod += b.mod;
   a.xr ^= b.xr;

@@ -88,6 +88,11 @@ cudaError_t launch_tmm_simt(const TmmArgs& a, cudaStream_t st);
 bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int64_t lda, int64_t ldb,
                       int64_t ldc, const void* A, const void* B, const void* C);
 cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why);
+// Listing 7's same-grid check-and-recover on the CTA-pair kernel (M, N % 256 == 0): every CTA validates
+// its halves of its pair's tiles, then recomputes in place only the tiles with a failed region;
+// *d_rec (zeroed here) counts the failed regions.
+bool tmm_tc_check_supported(int64_t M, int64_t N);
+cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why);
 
 // ---- tmm_tf32.cu : fp32 in/out via 3xTF32 on tcgen05 (CTA pair)
 bool tmm_tf32_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int out_bf16, int64_t lda,

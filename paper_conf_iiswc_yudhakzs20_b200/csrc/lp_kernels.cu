@@ -27,21 +27,6 @@ constexpr int kValUnroll = 8;
 // checksum (the B200 form of Listing 4's shfl_down ladder, L244-258); narrower
 // groups use an xor butterfly of log2(group) shuffles.  Adler's W is reduced
 // mod 65521 per lane first so the u32 sums cannot wrap (<= 32 * 65520).
-template <uint32_t MASK>
-__device__ __forceinline__ CkRecord segment_reduce(const CkPartial<MASK>& p, int lg_log2) {
-  if (lg_log2 == 5) return warp_reduce<MASK>(p);
-  CkRecord r{p.mod, p.xr, p.s, 0u};
-  if constexpr ((MASK & kAdler) != 0) r.wmod = (uint32_t)(p.w % kAdlerBase);
-  for (int o = (1 << lg_log2) >> 1; o > 0; o >>= 1) {
-    if constexpr ((MASK & kMod) != 0) r.mod += __shfl_xor_sync(0xFFFFFFFFu, r.mod, o);
-    if constexpr ((MASK & kXor) != 0) r.xr ^= __shfl_xor_sync(0xFFFFFFFFu, r.xr, o);
-    if constexpr ((MASK & kAdler) != 0) {
-      r.s += __shfl_xor_sync(0xFFFFFFFFu, r.s, o);
-      r.wmod += __shfl_xor_sync(0xFFFFFFFFu, r.wmod, o);
-    }
-  }
-  return r;
-}
 
 
 // Fused ordered compaction (a9) for small tables: every validate CTA bumps a ticket after

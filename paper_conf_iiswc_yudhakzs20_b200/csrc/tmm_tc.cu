@@ -285,11 +285,97 @@ constexpr int kB2Bytes = kBK * 128 * 2;   // 16 KiB: this CTA's 128 columns of B
 constexpr int kStage2Bytes = kA2Bytes + kB2Bytes;
 constexpr int kSmem2Bytes = kStages2 * kStage2Bytes + 1024 + 1024;
 
+// ---------------------------------------------------------------------------- Listing 7 check phase
+// Same-grid check-and-recover (Listing 7; NEXT row N2): before its mainloop, every CTA
+// validates its 128-row half of each 256x256 tile its pair owns in the ordinary persistent
+// schedule (L183: "fetching the corresponding data from memory, computing their checksums, and
+// then comparing them with the ones stored in the checksum table").  Work item = one 32-row band
+// (32x32 regions) or a whole 128-row half (128x128 regions) of a tile; the 6 warps take items
+// round robin, lane l reads 16-byte chunk l (+32) of every row (coalesced 512-B rows), each lane's
+// chunks stay inside one region column, so a segmented warp reduction yields the records.  A
+// failed region sets its tile's bit in this CTA's shared bitmask and bumps *d_rec.
+constexpr int kCheckUnroll = 8;
+
+__device__ __forceinline__ uint4 ld_u4_noalloc(const void* p) {
+  uint4 r;
+  asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
 template <typename OutT, uint32_t MASK, int REG, int STORE>
+__device__ __forceinline__ void check_tiles(const OutT* __restrict__ C, int64_t ldc, const uint32_t* __restrict__ ck,
+                                            int64_t ntiles, int64_t pair, int64_t npairs, int64_t num_m,
+                                            int64_t num_n, int64_t Qr, int64_t rid_offset, uint32_t rank,
+                                            uint32_t* s_fail, int64_t* d_rec) {
+  constexpr int ES = (int)sizeof(OutT);
+  constexpr int S = selem_of(MASK);
+  constexpr int CPR = 256 * ES / 16;            // 16-byte chunks per tile-half row (32 bf16 / 64 fp32)
+  constexpr int U = CPR / 32;                   // chunks per lane per row
+  constexpr int CPRR = REG * ES / 16;           // chunks per region row
+  constexpr int LGL = CPRR >= 32 ? 5 : (CPRR == 16 ? 4 : (CPRR == 8 ? 3 : 2));
+  constexpr int RB = REG == 32 ? 32 : 128;      // rows per work item
+  constexpr int NB = 128 / RB;                  // items per tile half
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t nloc = (ntiles - pair + npairs - 1) / npairs;
+  for (int64_t it = warp; it < nloc * NB; it += kThreads / 32) {
+    const int64_t lt = it / NB;
+    const int band = (int)(it - lt * NB);
+    int64_t mb, nb;
+    tile_coords(pair + lt * npairs, num_m, num_n, mb, nb);
+    const int64_t row0 = (mb * 2 + rank) * 128 + band * RB;
+    const uint8_t* base = reinterpret_cast<const uint8_t*>(C + row0 * ldc + nb * 256);
+    CkPartial<MASK> part[U];
+#pragma unroll 1
+    for (int r0 = 0; r0 < RB; r0 += kCheckUnroll) {
+      uint4 v[kCheckUnroll][U];
+#pragma unroll
+      for (int r = 0; r < kCheckUnroll; ++r)
+#pragma unroll
+        for (int u = 0; u < U; ++u) v[r][u] = ld_u4_noalloc(base + (int64_t)(r0 + r) * ldc * ES + (lane + 32 * u) * 16);
+#pragma unroll
+      for (int r = 0; r < kCheckUnroll; ++r)
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int c = lane + 32 * u;
+          const uint32_t pos = (uint32_t)(((r0 + r) % REG) * REG * ES + (c % CPRR) * 16 + 1);
+          part[u].add4(v[r][u].x, v[r][u].y, v[r][u].z, v[r][u].w, pos);
+        }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const CkRecord rec = segment_reduce<MASK>(part[u], LGL);
+      const int c = lane + 32 * u;
+      if ((c % CPRR) == 0) {
+        const int64_t p = row0 / REG, q = nb * (256 / REG) + c / CPRR;
+        const int64_t rid = p * Qr + q;
+        uint32_t w[3];
+        record_words<MASK>(rec, (uint64_t)REG * REG * ES, w);
+        bool bad = false;
+        if constexpr (STORE == 0) {
+#pragma unroll
+          for (int s2 = 0; s2 < S; ++s2) bad |= (ck[rid * S + s2] != w[s2]);
+        } else {
+          uint32_t stored[3];
+          bad = !store_lookup<S, STORE>(ck, (uint32_t)(rid + rid_offset), stored);
+#pragma unroll
+          for (int s2 = 0; s2 < S; ++s2) bad |= (!bad && stored[s2] != w[s2]);
+        }
+        if (bad) {
+          atomicOr(&s_fail[lt >> 5], 1u << (lt & 31));
+          atomicAdd(reinterpret_cast<unsigned long long*>(d_rec), 1ull);
+        }
+      }
+    }
+  }
+}
+
+template <typename OutT, uint32_t MASK, int REG, int STORE, bool CHECK = false>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     tmm_tc2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
                    OutT* __restrict__ C, int64_t ldc, int64_t K, int64_t num_m, int64_t num_n, int64_t Qr,
-                   int64_t rid_offset, uint32_t* __restrict__ ck) {
+                   int64_t rid_offset, uint32_t* __restrict__ ck, int64_t* __restrict__ d_rec) {
   constexpr int BN = 256;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -331,12 +417,32 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   const uint32_t tmem_base = *tmem_holder;
   const int64_t ntiles = num_m * num_n;
   const int nkb = (int)(K / kBK);
+  // Listing 7 form: failed-tile bitmask of this pair's local tile sequence (own half | peer half)
+  uint32_t* s_fail = reinterpret_cast<uint32_t*>(srec + 16);
+  const int64_t nloc = (ntiles - pair + npairs - 1) / npairs;
+  const int nwords = (int)((nloc + 31) >> 5);
+  uint32_t* s_todo = s_fail + nwords;
+  if constexpr (CHECK) {
+    for (int i = threadIdx.x; i < nwords; i += kThreads) s_fail[i] = 0u;
+    __syncthreads();
+    check_tiles<OutT, MASK, REG, STORE>(C, ldc, ck, ntiles, pair, npairs, num_m, num_n, Qr, rid_offset, rank, s_fail,
+                                        d_rec);
+    cluster_sync_all();  // both halves checked; the peer's bitmask is final
+    uint32_t peer;
+    for (int i = threadIdx.x; i < nwords; i += kThreads) {
+      asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(peer) : "r"(mapa_peer(&s_fail[i], rank ^ 1u)) : "memory");
+      s_todo[i] = s_fail[i] | peer;
+    }
+    __syncthreads();
+  }
+  auto skip = [&](int64_t lt) -> bool { return CHECK && !((s_todo[lt >> 5] >> (lt & 31)) & 1u); };
 
   if (warp == 0) {
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int64_t t = pair; t < ntiles; t += npairs) {
+      for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
+        if (skip(lt)) continue;
         int64_t mb, nb;
         tile_coords(t, num_m, num_n, mb, nb);
         const int m0 = (int)(mb * 256 + rank * 128), n0 = (int)(nb * 256 + rank * 128);
@@ -366,7 +472,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int64_t t = pair; t < ntiles; t += npairs) {
+      for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
+        if (skip(lt)) continue;
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -398,7 +505,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const int wq = warp & 3;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int64_t t = pair; t < ntiles; t += npairs) {
+    for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
+      if (skip(lt)) continue;
       int64_t mb, nb;
       tile_coords(t, num_m, num_n, mb, nb);
       mbar_wait(&tfull[acc], acc_phase);
@@ -540,7 +648,7 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2Bytes);                \
     if (e != cudaSuccess) return e;                                                                         \
     kfn<<<(unsigned)grid, kThreads, kSmem2Bytes, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr,    \
-                                                       a.rid_offset, a.ck);                                 \
+                                                       a.rid_offset, a.ck, nullptr);                        \
     break;                                                                                                  \
   }
 #define LP_TC2_CASE3(M) LP_TC2_CASE(M, 0)
@@ -556,6 +664,56 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
 #undef LP_TC2_CASE3
 #undef LP_TC2_CASE5
 #undef LP_TC2_CASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+template <typename OutT, int REG>
+cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why) {
+  CUtensorMap ma, mb;
+  if (!make_map_2d(&ma, a.A, (uint64_t)a.K, (uint64_t)a.M, (uint64_t)a.lda, kBK, kBM) ||
+      !make_map_2d(&mb, a.B, (uint64_t)a.N, (uint64_t)a.K, (uint64_t)a.ldb, 64, kBK)) {
+    *why = "cuTensorMapEncodeTiled failed";
+    return cudaErrorInvalidValue;
+  }
+  const int64_t num_m = a.M / 256, num_n = a.N / 256;
+  int64_t grid = 2 * num_m * num_n;
+  const int64_t cap = a.sm_count & ~1;
+  if (grid > cap) grid = cap;
+  if (grid < 2) grid = 2;
+  const int64_t nloc = (num_m * num_n + grid / 2 - 1) / (grid / 2);
+  const int smem = kSmem2Bytes + (int)(2 * ((nloc + 31) / 32) * 4);
+  if (smem > 227 * 1024) {
+    *why = "too many tiles per CTA pair for the check-and-recover bitmask";
+    return cudaErrorInvalidValue;
+  }
+  const int64_t Qr = a.N / REG;
+  cudaError_t e = cudaMemsetAsync(d_rec, 0, sizeof(int64_t), st);
+  if (e != cudaSuccess) return e;
+  switch (a.mask * 5 + a.hash.store) {
+#define LP_TC2C_CASE(M, S)                                                                                  \
+  case M * 5 + S: {                                                                                         \
+    auto kfn = tmm_tc2_kernel<OutT, M, REG, S, true>;                                                      \
+    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
+    if (e != cudaSuccess) return e;                                                                         \
+    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr, a.rid_offset, \
+                                                a.ck, d_rec);                                               \
+    break;                                                                                                  \
+  }
+#define LP_TC2C_CASE3(M) LP_TC2C_CASE(M, 0)
+#define LP_TC2C_CASE5(M) LP_TC2C_CASE(M, 0) LP_TC2C_CASE(M, 1) LP_TC2C_CASE(M, 2) LP_TC2C_CASE(M, 3) LP_TC2C_CASE(M, 4)
+    LP_TC2C_CASE5(1)
+    LP_TC2C_CASE3(2)
+    LP_TC2C_CASE5(3)
+    LP_TC2C_CASE3(4)
+    LP_TC2C_CASE3(5)
+    LP_TC2C_CASE3(6)
+    LP_TC2C_CASE3(7)
+#undef LP_TC2C_CASE3
+#undef LP_TC2C_CASE5
+#undef LP_TC2C_CASE
     default:
       return cudaErrorInvalidValue;
   }
@@ -584,6 +742,17 @@ bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf
   if ((((uintptr_t)A) & 15u) || (((uintptr_t)B) & 15u) || (((uintptr_t)C) & 15u)) return false;
   if (M > (int64_t)INT32_MAX || N > (int64_t)INT32_MAX || K > (int64_t)INT32_MAX) return false;
   return true;
+}
+
+bool tmm_tc_check_supported(int64_t M, int64_t N) { return M % 256 == 0 && N % 256 == 0; }
+
+cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why) {
+  if (a.mask == 0 || a.list || !tmm_tc_check_supported(a.M, a.N)) return cudaErrorInvalidValue;
+  if (a.RM == 128)
+    return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 128>(a, d_rec, st, why)
+                      : launch_pair_check<float, 128>(a, d_rec, st, why);
+  return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 32>(a, d_rec, st, why)
+                    : launch_pair_check<float, 32>(a, d_rec, st, why);
 }
 
 cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why) {

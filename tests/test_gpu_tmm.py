@@ -321,3 +321,71 @@ def test_cuckoo_full_r262144(store):
     ck_h = dev_to_host(ck)
     assert ck_h[6] == 0
     check_store_table(ck_h, store, R, 2, oracle.records(dev_to_host(out), 32, 32, 3))
+
+
+# ----------------------------------------------------------------------------- Listing 7 on the TMM (N2)
+@pytest.mark.parametrize("reg,out_dt,store", [(128, "bf16", "array"), (32, "bf16", "array"), (128, "f32", "array"),
+                                              (32, "f32", "quad_cas"), (128, "bf16", "cuckoo")])
+@pytest.mark.parametrize("frac", [0.01, 0.10, 0.50])
+def test_tmm_same_grid_check_and_recover(reg, out_dt, store, frac):
+    """Listing 7 (L565-578) on the tcgen05 CTA-pair TMM: one kernel validates every region of its tiles and
+    recomputes in place only the tiles holding a failed region.  The count equals the oracle's failed set on
+    the corrupted image, the recovered bytes equal the golden run, and a re-validate finds nothing."""
+    M, N, K = 1024, 1536, 128          # 24 tiles of 256x256 over the CTA pairs; ragged per-pair counts
+    h = lp.LP(reg, reg, cksum="mod|xor", store=store)
+    A, B = make_inputs(13, M, N, K, "uniform", "bf16")
+    a, b = host_to_dev(A, "bf16"), host_to_dev(B, "bf16")
+    wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    stale = host_to_dev(stale_image(13, M, N, out_dt), out_dt)
+    out.copy_(stale)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    torch.cuda.synchronize()
+    golden = dev_to_host(out)
+    R = h.num_regions(wl)
+    # clean image: nothing fails, nothing is recomputed
+    d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+    h.check_recover(wl, out, ck, d_rec)
+    torch.cuda.synchronize()
+    assert int(d_rec.item()) == 0
+    inj = torch.from_numpy(lp.choose_regions(R, frac, 500 + reg)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=501)
+    torch.cuda.synchronize()
+    exp = oracle_validate(dev_to_host(out), dev_to_host(ck), store, reg, reg, h.mask)
+    assert len(exp) > 0
+    h.check_recover(wl, out, ck, d_rec)
+    torch.cuda.synchronize()
+    assert int(d_rec.item()) == len(exp)
+    assert np.array_equal(dev_to_host(out).view(np.uint8), golden.view(np.uint8))
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(d_n.item()) == 0
+
+
+def test_tmm_check_and_recover_full_8192():
+    """BASELINE configs[1] shape: 8192^3 bf16, 128x128 regions, 5% STALE_WORDS: check-and-recover restores the
+    golden bytes; the count equals the oracle's failed set recomputed from the corrupted image."""
+    from lpsynth import device_fill
+    M = N = K = 8192
+    a = torch.empty((M, K), dtype=torch.bfloat16, device="cuda")
+    b = torch.empty((K, N), dtype=torch.bfloat16, device="cuda")
+    device_fill(a, 1, "uniform", "bf16")
+    device_fill(b, 2, "uniform", "bf16")
+    h = lp.LP(128, 128, cksum="mod|xor")
+    wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    golden = out.clone()
+    stale = torch.zeros_like(out)
+    R = h.num_regions(wl)
+    inj = torch.from_numpy(lp.choose_regions(R, 0.05, 1001)).cuda()
+    h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=1001)
+    torch.cuda.synchronize()
+    exp = oracle_validate(dev_to_host(out), dev_to_host(ck), "array", 128, 128, h.mask)
+    d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+    h.check_recover(wl, out, ck, d_rec)
+    torch.cuda.synchronize()
+    assert int(d_rec.item()) == len(exp) > 0
+    assert torch.equal(out.view(torch.int16), golden.view(torch.int16))

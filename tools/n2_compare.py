@@ -1,7 +1,14 @@
 #!/usr/bin/env python
-"""N2: the paper's same-grid check-and-recover kernel (Listing 7) vs validate -> compact -> list-mode
-relaunch, on the C4 stencil (32768^2 fp32, 128x128 regions, MOD|XOR) at 1/10/50% STALE_REGION crashes.
-Times are CUDA-event medians of 7 reps, L2 flushed; each rep starts from the same corrupted image."""
+"""N2: the paper's same-grid check-and-recover kernel (Listing 7) vs validate -> compact ->
+list-mode relaunch, at 1/10/50% crashed regions.
+
+  --workload stencil : C4 stencil 32768^2 fp32, 128x128 regions, MOD|XOR, STALE_REGION crashes
+  --workload tmm128  : C2 TMM 8192^3 bf16, 128x128 regions, MOD|XOR, STALE_WORDS crashes
+  --workload tmm32   : C2 TMM 8192^3 bf16, 32x32 regions, MOD|XOR, STALE_WORDS crashes
+
+Times are CUDA-event medians of 7 reps, L2 flushed before each; each rep starts from the same corrupted
+image, and the recovered output is asserted equal to the golden one after every rep."""
+import argparse
 import sys
 
 import torch
@@ -10,31 +17,52 @@ sys.path.insert(0, ".")
 import lpsynth  # noqa: E402
 from paper_conf_iiswc_yudhakzs20_b200 import lp  # noqa: E402
 
-H = W = 32768
-x = torch.empty((H, W), dtype=torch.float32, device="cuda")
-lpsynth.device_fill(x, 1, "uniform", "f32")
-h = lp.LP(128, 128, cksum="mod|xor")
-wl = lp.Workload.stencil(x)
+ap = argparse.ArgumentParser()
+ap.add_argument("--workload", default="stencil", choices=["stencil", "tmm128", "tmm32"])
+args = ap.parse_args()
+
+if args.workload == "stencil":
+    H = W = 32768
+    x = torch.empty((H, W), dtype=torch.float32, device="cuda")
+    lpsynth.device_fill(x, 1, "uniform", "f32")
+    h = lp.LP(128, 128, cksum="mod|xor")
+    wl = lp.Workload.stencil(x)
+    mode = "stale_region"
+else:
+    n = 8192
+    reg = 128 if args.workload == "tmm128" else 32
+    a = torch.empty((n, n), dtype=torch.bfloat16, device="cuda")
+    b = torch.empty((n, n), dtype=torch.bfloat16, device="cuda")
+    lpsynth.device_fill(a, 1, "uniform", "bf16")
+    lpsynth.device_fill(b, 2, "uniform", "bf16")
+    h = lp.LP(reg, reg, cksum="mod|xor")
+    wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+    mode = "stale_words"
 out, ck, failed, d_n, ws = h.alloc(wl)
 h.cksum_init(wl, ck)
 h.run_protected(wl, out, ck)
 golden = out.clone()
 stale = torch.empty_like(out)
-lpsynth.device_fill(stale.view(torch.int32), 3, "bits", "u32")
+if out.dtype == torch.float32:
+    lpsynth.device_fill(stale.view(torch.int32), 3, "bits", "u32")
+else:
+    lpsynth.device_fill(stale, 3, "bits", "bf16")
 R = h.num_regions(wl)
 flush = torch.empty(512 << 20, dtype=torch.uint8, device="cuda")
 bad_img = torch.empty_like(out)
 ck_img = torch.empty_like(ck)
 d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+print(f"workload {args.workload}: R = {R}")
 print("| crash fraction | failed regions | validate + compact + relaunch (ms) | same-grid check-and-recover (ms) | ratio |")
 print("|---|---|---|---|---|")
 for frac in (0.01, 0.10, 0.50):
     inj = torch.from_numpy(lp.choose_regions(R, frac, 77)).cuda()
     out.copy_(golden)
-    h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=77)
+    h.inject(wl, out, ck, stale, inj, mode=mode, seed=77)
     bad_img.copy_(out)
     ck_img.copy_(ck)
     res = {}
+    nfail = {}
     for name in ("ours", "listing7"):
         ts = []
         for _ in range(7):
@@ -51,8 +79,10 @@ for frac in (0.01, 0.10, 0.50):
             e1.record()
             torch.cuda.synchronize()
             ts.append(e0.elapsed_time(e1))
-            assert torch.equal(out, golden)
+            assert torch.equal(out.view(torch.int16) if out.dtype == torch.bfloat16 else out.view(torch.int32),
+                               golden.view(torch.int16) if out.dtype == torch.bfloat16 else golden.view(torch.int32))
+            nfail[name] = int(d_n.item()) if name == "ours" else int(d_rec.item())
         res[name] = sorted(ts)[3]
-    n = int(d_n.item())
-    print(f"| {frac:.0%} | {n} | {res['ours']:.3f} | {res['listing7']:.3f} | {res['listing7'] / res['ours']:.2f} |",
-          flush=True)
+    assert nfail["ours"] == nfail["listing7"], nfail
+    print(f"| {frac:.0%} | {nfail['ours']} | {res['ours']:.3f} | {res['listing7']:.3f} | "
+          f"{res['listing7'] / res['ours']:.2f} |", flush=True)
