@@ -107,7 +107,8 @@ WORKLOADS = {
 def kernels_per_step(W, store, R):
     """Our kernels launched by one step (init memset is not a kernel): protected body (+ hash header),
     inject, 2 x validate (+ the ordered-compaction scatter when R > 16384; smaller tables are compacted
-    by the last validate CTA), recovery (+ tile de-dup / pairing kernels)."""
+    by the last validate CTA), recovery (+ tile de-dup / pairing kernels, + the recovered-count kernel,
+    + the cuckoo rehash check)."""
     body = 1 + (1 if store != "array" else 0)
     val = 1 if R <= 16384 else 2
     if W["kind"] == "tmm" and W["in_dt"] == "bf16" and W.get("body") != "simt":
@@ -116,6 +117,10 @@ def kernels_per_step(W, store, R):
         rec = 4                                        # tile mark, count, scatter, 3xTF32 list mode
     else:
         rec = 1
+    rec += 1                                           # recovered-region count (lp_recover_count)
+    if store.startswith("cuckoo"):
+        body += 1                                      # cuckoo rehash check after the body (and after recovery)
+        rec += 1
     return body + 1 + 2 * val + rec
 
 
@@ -141,6 +146,9 @@ def parse():
                     help="override the workload's injected fraction of regions (design-space runs)")
     ap.add_argument("--recover-tile128", action="store_true",
                     help="tcgen05 recovery of 32x32 regions: 128x128 tiles instead of 128x64 slices -- A/B switch")
+    ap.add_argument("--nvls-count", action="store_true",
+                    help="N>1 over NCCL: all-reduce the failed count inside lp_validate through an NVSwitch multicast "
+                         "counter (multimem.red, lp_attach_nvls_count) instead of an NCCL all-reduce")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch the step eagerly instead of replaying captured CUDA graphs")
     return ap.parse_args()
@@ -347,8 +355,21 @@ def run_ours(args):
         b = None
         wl = lp.Workload.stencil(a, row_offset=sh.row_offset, global_m=gM)
         body_flops = 0.0
+    nvls_mc, nvls_buf, nvls_note = None, None, None
+    if args.nvls_count:
+        if world > 1 and args.dist_backend == "nccl":
+            nvls_mc, nvls_buf = shard.nvls_counter(dev)
+            if nvls_mc is None:
+                nvls_note, nvls_buf = f"unavailable ({nvls_buf}); NCCL all-reduce used", None
+            else:
+                nvls_note = "failed count all-reduced by multimem.red from the CTA that finalises it"
+        else:
+            nvls_note = "needs N > 1 over NCCL; NCCL/no all-reduce used"
     h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
-              shuffle=not args.no_shuffle, pairing=not args.no_pairing, recover_slices=not args.recover_tile128)
+              shuffle=not args.no_shuffle, pairing=not args.no_pairing, recover_slices=not args.recover_tile128,
+              nvls_count=nvls_mc is not None)
+    if nvls_mc is not None:
+        h.attach_nvls_count(nvls_mc, nvls_buf, world)
     h0 = lp.LP(RM, RN, cksum=0, device=local, body=W.get("body", "auto"))   # unprotected twin (overhead denominator)
     out, ck, failed, d_n, ws = h.alloc(wl)
     out_twin = torch.empty_like(out)
@@ -404,15 +425,23 @@ def run_ours(args):
     def seg_inject():
         h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=1000 + rank)
 
+    # counts = {n_failed, n_recovered (regions the recovery kernels rewrote), n_failed_after}; with the NVLS
+    # counter, lp_validate itself leaves the all-rank failed count in slot 4 of the multicast buffer
     def seg_validate():
         h.validate(wl, out, ck, failed, d_n, ws)
-        counts[0:1].copy_(d_n)
-        counts[1:2].copy_(d_n)
+        counts[0:1].copy_(nvls_buf[4:5] if nvls_buf is not None else d_n)
 
     def seg_recover():
-        h.recover(wl, out, ck, failed, d_n, ws)
+        h.recover(wl, out, ck, failed, d_n, ws, d_n_recovered=counts[1:2])
         h.validate(wl, out, ck, failed, d_n, ws)
-        counts[2:3].copy_(d_n)
+        counts[2:3].copy_(nvls_buf[4:5] if nvls_buf is not None else d_n)
+
+    def reduce_failed():
+        if nvls_buf is None:
+            shard.allreduce_counts(counts[0:1])
+
+    def reduce_summary():
+        shard.allreduce_counts(counts[1:2] if nvls_buf is not None else counts[1:3])
 
     runners = {"body": seg_body, "inject": seg_inject, "validate": seg_validate, "recover": seg_recover}
 
@@ -438,9 +467,9 @@ def run_ours(args):
         l2_flush()                    # cold L2 for the recovery phase (not timed)
         e[3].record(st)
         runners["validate"]()
-        shard.allreduce_counts(counts[0:2])
+        reduce_failed()
         runners["recover"]()
-        shard.allreduce_counts(counts[2:3])
+        reduce_summary()
         e[4].record(st)
         return e
 
@@ -474,6 +503,7 @@ def run_ours(args):
     t_inj = [s[1] for s in segs]
     t_vr = [s[2] for s in segs]
     n_failed = int(counts[0].item())
+    n_recovered = int(counts[1].item())
     n_after = int(counts[2].item())
     assert n_after == 0, f"re-validation left {n_after} failed regions"
     n_failed_local = int(d_n.item())  # after re-validate: 0
@@ -532,6 +562,8 @@ def run_ours(args):
     # freshly initialised table (a hash store then measures fresh-table inserts, as Fig. 5 / Table IV do); the
     # twin gets a memset of the same size on a scratch buffer, so both sides do identical untimed preparation.
     ck_twin_scratch = torch.empty_like(ck)
+    h0.run_protected(wl, out_twin, None)      # first call of the twin (module load) outside the timed reps
+    torch.cuda.synchronize()
     tp, tu, pair_clk = [], [], []
     for i in range(args.overhead_reps * 2):
         if i % 2 == 0:
@@ -593,9 +625,9 @@ def run_ours(args):
         out.copy_(out_host, non_blocking=True)
         ck.copy_(ck_host, non_blocking=True)
         runners["validate"]()
-        shard.allreduce_counts(counts[0:2])
+        reduce_failed()
         runners["recover"]()
-        shard.allreduce_counts(counts[2:3])
+        reduce_summary()
         summary_host.copy_(counts, non_blocking=True)
         e1.record(st)
         torch.cuda.synchronize()
@@ -726,6 +758,10 @@ def run_ours(args):
                                      if args.graph else "events around one eager call")),
             "t_recovery_phase_ms": round(sum_vr / args.steps, 4),
             "n_failed_per_step": n_failed,
+            "n_recovered_per_step": n_recovered,
+            "count_allreduce": (nvls_note if args.nvls_count else
+                                ("NCCL all_reduce(SUM) of int64 counts on the compute stream" if world > 1
+                                 else "none (N = 1)")),
             "n_failed_after_recover": n_after,
             "per_rank": spread,
             "hash_collisions": hash_stats[0] if W["store"] != "array" else None,

@@ -136,8 +136,10 @@ typedef enum {
   LP_FLAG_RECOVER_TILE128 = 16u, /* tcgen05 bf16 recovery of 32x32 regions: de-duplicate failed regions into 128x128
                                    tiles (paired into 128x256 tasks) instead of 128x64 slices paired into 128x128
                                    tasks (A/B switch; both re-execute every failed region, L51-57) */
-  LP_FLAG_CUCKOO_SHORT_CHAINS = 32u /* cuckoo stores, test hook: the body's inserts give up after 16 evictions
+  LP_FLAG_CUCKOO_SHORT_CHAINS = 32u, /* cuckoo stores, test hook: the body's inserts give up after 16 evictions
                                        instead of 128, so entries reach the stash and the rehash (L270) runs */
+  LP_FLAG_NVLS_COUNT = 64u /* allow lp_attach_nvls_count: lp_validate all-reduces the failed count through an
+                              NVSwitch multicast counter (multimem.red) from the CTA that finalises it */
 } lp_config_flags;
 
 typedef struct {
@@ -228,6 +230,16 @@ LP_API lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* o
 LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
                             const int64_t* d_n_failed, void* workspace, lp_stream_t stream);
 
+/* lp_recover that also reports, in *d_n_recovered (device int64; may be NULL), the number of
+ * regions whose data and record the recovery kernels rewrote: the entries of the list the kernel
+ * consumed times the regions per entry -- *d_n_failed without de-duplication, and (de-duplicated
+ * tiles or slices) x (32x32 regions per tile / slice) when several failed 32x32 regions share a
+ * tensor-core tile, in which case it can exceed *d_n_failed.  Written on the device after the
+ * re-execution kernel, in stream order. */
+LP_API lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
+                                  const int64_t* failed_list, const int64_t* d_n_failed, void* workspace,
+                                  int64_t* d_n_recovered, lp_stream_t stream);
+
 /* The paper's own recovery form (Listing 7; NEXT row N2): ONE kernel
  * with the grid of the original kernel, in which every CTA validates its regions
  * and, if a check fails, re-executes in place (data and record).
@@ -244,6 +256,20 @@ LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, voi
  * Other workloads / bodies: LP_ERR_UNSUPPORTED. */
 LP_API lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
                                   int64_t* d_n_recovered, lp_stream_t stream);
+
+/* NVLS-fused failed-count all-reduce (needs cfg.flags & LP_FLAG_NVLS_COUNT).
+ * mc_counter = the multicast (NVLS) address and uc_counter = this rank's unicast address of the same
+ * 64-byte-aligned, >= 64-byte counter buffer, bound to a multicast object on every one of the
+ * world_size ranks and zero-filled on all of them before the first lp_validate (e.g. torch symmetric
+ * memory: rendezvous(...).multicast_ptr / buffer_ptrs[rank]).  Afterwards every lp_validate on this
+ * handle ends with the CTA that writes *d_n_failed adding the shard's count with
+ * multimem.red.add.u64 into every rank's copy, signalling its arrival the same way and waiting for all
+ * ranks of this epoch; ((uint64_t*)uc_counter)[4] then holds the all-rank failed count (the local list
+ * and *d_n_failed are unchanged).  Every rank must call lp_validate the same number of times.
+ * mc_counter == uc_counter with world_size == 1 is a single-GPU emulation (plain atomics) that
+ * exercises the epoch logic; NULL, NULL detaches.  The multimem path itself needs >= 2 GPUs on an
+ * NVSwitch fabric: a 1-device multicast object cannot be created (cuMulticastCreate -> invalid value). */
+LP_API lp_status lp_attach_nvls_count(lp_handle h, void* mc_counter, void* uc_counter, int32_t world_size);
 
 /* Records of every region of `out` (uint32 [R][selem], order MOD, XOR, ADLER)
  * without comparing -- for parity tests against the oracle. */

@@ -25,6 +25,7 @@ struct lp_ctx {
   int selem;
   int dev_checked;  // 0 = not yet, 1 = ok
   int sm_count;
+  lp::NvlsCount nvls;  // NVLS-fused failed count (lp_attach_nvls_count); mc == nullptr: off
 };
 
 namespace {
@@ -261,7 +262,8 @@ lp::TmmArgs tmm_args(const lp_ctx* h, const lp_workload_t* wl, const lp::RegionG
 
 // Body dispatch shared by run_protected and recover (list = null for a full run).
 lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, void* out, void* ck,
-                   const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr) {
+                   const int64_t* list, const int64_t* d_n, cudaStream_t st, void* workspace = nullptr,
+                   int64_t* d_rec = nullptr) {
   const lp::HashInfo hi = hash_info(h, g);
   if ((h->cfg.flags & LP_FLAG_NO_SHUFFLE) && wl->kind == LP_WL_STENCIL5)
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is not built for the stencil body");
@@ -288,6 +290,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.d_n = d_n;
     a.sm_count = h->sm_count;
     cudaError_t e = lp::launch_stencil(a, st);
+    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
     return e == cudaSuccess ? ok() : cuda_fail(e, "stencil launch");
   }
   if (wl->kind == LP_WL_SPMV) {
@@ -314,6 +317,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
     a.sm_count = h->sm_count;
     cudaError_t e = lp::launch_spmv(a, st);
+    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
     return e == cudaSuccess ? ok() : cuda_fail(e, "SPMV launch");
   }
   if (!wl->a || !wl->b) return fail(LP_ERR_INVALID_ARG, "null A or B");
@@ -366,12 +370,21 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     const char* why = nullptr;
     cudaError_t e = tc_ok ? lp::launch_tmm_tc(a, st, &why) : lp::launch_tmm_tf32(a, st, &why);
     if (e != cudaSuccess) return why ? fail(LP_ERR_CUDA, "tcgen05 launch: %s", why) : cuda_fail(e, "tcgen05 launch");
+    if (list && d_rec) {
+      // regions rewritten = entries of the list the kernel consumed x regions per entry (a de-duplicated
+      // tile / slice rewrites every region inside it)
+      // (without a workspace every listed region recomputes its whole E x E tile)
+      const int64_t per = (int64_t)(E / g.RM) * ((a.list_is_tiles ? EN : E) / g.RN);
+      e = lp::launch_scale_count(a.d_n, per, d_rec, st);
+      if (e != cudaSuccess) return cuda_fail(e, "recovered-count launch");
+    }
     return ok();
   }
   if (!lp::tmm_simt_supported(g.RM, g.RN, a.in_bf16, a.out_bf16))
     return fail(LP_ERR_UNSUPPORTED, "SIMT body supports 32x32, 64x64 and 128x128 regions");
   if (wl->k % 16) return fail(LP_ERR_UNSUPPORTED, "SIMT body needs k %% 16 == 0");
   cudaError_t e = lp::launch_tmm_simt(a, st);
+  if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
   return e == cudaSuccess ? ok() : cuda_fail(e, "SIMT TMM launch");
 }
 
@@ -403,7 +416,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING | LP_FLAG_NO_FUSED_COMPACT |
-                                 LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS))
+                                 LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS | LP_FLAG_NVLS_COUNT))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");
@@ -415,6 +428,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   h->selem = lp::selem_of(cfg->cksum);
   h->dev_checked = 0;
   h->sm_count = 0;
+  h->nvls = lp::NvlsCount{nullptr, nullptr, 1};
   *out = h;
   return ok();
 }
@@ -506,12 +520,17 @@ lp_status lp_validate(lp_handle h, const lp_workload_t* wl, const void* out, con
   cudaStream_t st = (cudaStream_t)stream;
   uint32_t* ticket = (h->cfg.flags & LP_FLAG_NO_FUSED_COMPACT) ? nullptr : (uint32_t*)((uint8_t*)workspace + w.ticket);
   cudaError_t e = lp::launch_validate(g, h->mask, hash_info(h, g), out, cksum, flags, nullptr, h->sm_count, st, counts,
-                                      failed_list, d_n_failed, ticket);
+                                      failed_list, d_n_failed, ticket, h->nvls.uc ? &h->nvls : nullptr);
   return e == cudaSuccess ? ok() : cuda_fail(e, "validate launch");
 }
 
 lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
                      const int64_t* d_n_failed, void* workspace, lp_stream_t stream) {
+  return lp_recover_count(h, wl, out, cksum, failed_list, d_n_failed, workspace, nullptr, stream);
+}
+
+lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, const int64_t* failed_list,
+                           const int64_t* d_n_failed, void* workspace, int64_t* d_n_recovered, lp_stream_t stream) {
   lp::RegionGeom g;
   lp_status s = check_wl(h, wl, &g);
   if (s) return s;
@@ -520,7 +539,8 @@ lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksu
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
   if (workspace && !aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
-  if ((s = run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace))) return s;
+  if ((s = run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace, d_n_recovered)))
+    return s;
   return cuckoo_rehash(h, cksum, (cudaStream_t)stream);
 }
 
@@ -575,6 +595,23 @@ lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void
   a.sm_count = h->sm_count;
   cudaError_t e = lp::launch_stencil_check_recover(a, d_n_recovered, (cudaStream_t)stream);
   return e == cudaSuccess ? ok() : cuda_fail(e, "check-and-recover launch");
+}
+
+lp_status lp_attach_nvls_count(lp_handle h, void* mc_counter, void* uc_counter, int32_t world_size) {
+  if (!h) return fail(LP_ERR_INVALID_ARG, "null handle");
+  if (!mc_counter && !uc_counter) {
+    h->nvls = lp::NvlsCount{nullptr, nullptr, 1};
+    return ok();
+  }
+  if (!(h->cfg.flags & LP_FLAG_NVLS_COUNT)) return fail(LP_ERR_STATE, "lp_config_t.flags lacks LP_FLAG_NVLS_COUNT");
+  if (!mc_counter || !uc_counter) return fail(LP_ERR_INVALID_ARG, "both the multicast and the unicast address are needed");
+  if ((((uintptr_t)mc_counter) & 63u) || (((uintptr_t)uc_counter) & 63u))
+    return fail(LP_ERR_INVALID_ARG, "counter buffers must be 64-B aligned");
+  if (world_size < 1) return fail(LP_ERR_INVALID_ARG, "world_size must be >= 1");
+  if (mc_counter == uc_counter && world_size != 1)
+    return fail(LP_ERR_INVALID_ARG, "mc == uc (single-GPU emulation) needs world_size == 1");
+  h->nvls = lp::NvlsCount{(unsigned long long*)mc_counter, (unsigned long long*)uc_counter, world_size};
+  return ok();
 }
 
 lp_status lp_region_checksums(lp_handle h, const lp_workload_t* wl, const void* out, uint32_t* records,

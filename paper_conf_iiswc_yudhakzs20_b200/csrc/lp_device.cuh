@@ -407,6 +407,50 @@ __device__ __forceinline__ bool store_lookup(const uint32_t* ck, uint32_t global
   }
 }
 
+// ---------------------------------------------------------------------------
+// NVLS-fused failed count: the CTA that finalises a shard's failed
+// count also adds it, with multimem.red, into a counter bound to a multicast object that every
+// rank maps (NVSwitch performs the reduction into each GPU's copy), bumps an arrival counter the
+// same way, and waits until all world_size ranks of this epoch have arrived: every rank then
+// holds the all-rank count without a separate NCCL all-reduce launch.  Counter buffer (u64,
+// zero-filled once on every rank, symmetric): [0],[1] cumulative counts by epoch parity,
+// [2] arrivals, [3] this rank's epoch, [4] RESULT (the all-rank count of the latest epoch),
+// [5],[6] last cumulative value by parity.  mc == uc with world == 1 is the single-GPU
+// emulation (plain atomics on the local copy) that tests the epoch logic without NVLink.
+struct NvlsCount {
+  unsigned long long* mc;  // multicast address of the counter buffer (null: feature off)
+  unsigned long long* uc;  // this rank's unicast address of the same buffer
+  int world;
+};
+
+__device__ __forceinline__ void nvls_publish(const NvlsCount& nv, int64_t n) {
+  if (nv.uc == nullptr) return;
+  volatile unsigned long long* uc = nv.uc;
+  const unsigned long long e = uc[3] + 1ull;
+  uc[3] = e;
+  const int par = (int)(e & 1ull);
+  if (nv.mc == nv.uc) {
+    atomicAdd(nv.uc + par, (unsigned long long)n);
+    __threadfence();
+    atomicAdd(nv.uc + 2, 1ull);
+  } else {
+    asm volatile("multimem.red.relaxed.sys.global.add.u64 [%0], %1;" ::"l"(nv.mc + par), "l"((unsigned long long)n)
+                 : "memory");
+    asm volatile("multimem.red.release.sys.global.add.u64 [%0], %1;" ::"l"(nv.mc + 2), "l"(1ull) : "memory");
+  }
+  const unsigned long long target = e * (unsigned long long)nv.world;
+  unsigned long long arrived;
+  for (;;) {
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(arrived) : "l"(nv.uc + 2) : "memory");
+    if (arrived >= target) break;
+    __nanosleep(64);
+  }
+  unsigned long long cum;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(cum) : "l"(nv.uc + par) : "memory");
+  uc[4] = cum - uc[5 + par];
+  uc[5 + par] = cum;
+}
+
 // Streaming 16-byte load that does not allocate in L1 (validate reads `out` once).
 __device__ __forceinline__ uint4 ld_stream_u4(const void* p) {
   uint4 r;

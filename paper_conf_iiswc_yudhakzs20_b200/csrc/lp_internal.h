@@ -7,6 +7,8 @@
 
 namespace lp {
 
+struct NvlsCount;  // lp_device.cuh
+
 // Geometry of one output matrix split into regions.
 struct RegionGeom {
   int64_t M, N;        // output rows / cols of this shard
@@ -34,7 +36,8 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
 constexpr int64_t kFusedCompactMaxR = 16384;
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
                             uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
-                            int64_t* list, int64_t* d_n, uint32_t* ticket = nullptr);
+                            int64_t* list, int64_t* d_n, uint32_t* ticket = nullptr,
+                            const NvlsCount* nv = nullptr);
 size_t validate_counts_bytes(const RegionGeom& g, int sm_count);
 cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* block_counts, int64_t* list,
                            int64_t* d_n, cudaStream_t st);
@@ -49,6 +52,8 @@ cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t o
                               int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
 // cuckoo stores: rebuild T1/T2 with a new seed if the stash is non-empty (no-op otherwise)
 cudaError_t launch_cuckoo_rehash(void* ck, cudaStream_t st);
+// *dst = *src * per on the device (recovered-region count of a list-mode recovery)
+cudaError_t launch_scale_count(const int64_t* src, int64_t per, int64_t* dst, cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
 // failed regions -> unique tile ids of an EM x EN tile grid (tile = (p*RM/EM)*(N/EN) + q*RN/EN), ascending
 cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const int64_t* list, const int64_t* d_n,

@@ -36,7 +36,8 @@ constexpr int kValUnroll = 8;
 // ticket RMW by thread 0 (cumulative: the CTA's flag stores are visible before the
 // ticket moves); the last CTA fences again before reading the flags (L2: ld.global.cg).
 __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int64_t R, int64_t rid_offset,
-                                                      uint32_t* ticket, int64_t* list, int64_t* d_n) {
+                                                      uint32_t* ticket, int64_t* list, int64_t* d_n,
+                                                      NvlsCount nvc) {
   __shared__ int s_last;
   __shared__ int s_warp[kValWarps];
   if (threadIdx.x == 0) {
@@ -104,6 +105,7 @@ __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int6
   if (threadIdx.x == 0) {
     *d_n = total;
     *ticket = 0u;
+    nvls_publish(nvc, total);
   }
 }
 
@@ -128,7 +130,8 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
                                                                 uint32_t* __restrict__ records, int64_t rpc,
                                                                 uint32_t* __restrict__ cta_counts,
                                                                 uint32_t* __restrict__ ticket,
-                                                                int64_t* __restrict__ list, int64_t* __restrict__ d_n) {
+                                                                int64_t* __restrict__ list, int64_t* __restrict__ d_n,
+                                                                NvlsCount nv) {
   constexpr int S = selem_of(MASK);
   __shared__ uint32_t s_fail;
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -194,7 +197,7 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
   if constexpr (MODE != 2) {
     __syncthreads();
     if (threadIdx.x == 0) cta_counts[blockIdx.x] = s_fail;
-    if (ticket) fused_compact_if_last(flags, R, rid_offset, ticket, list, d_n);
+    if (ticket) fused_compact_if_last(flags, R, rid_offset, ticket, list, d_n, nv);
   }
 }
 
@@ -208,11 +211,12 @@ template <uint32_t MASK>
 cudaError_t validate_dispatch_mode(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
                                    int64_t ldc_bytes, int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2,
                                    const uint32_t* ck, int64_t rid_offset, uint8_t* flags, uint32_t* records,
-                                   uint32_t* counts, uint32_t* ticket, int64_t* list, int64_t* d_n) {
+                                   uint32_t* counts, uint32_t* ticket, int64_t* list, int64_t* d_n,
+                                   const NvlsCount& nv) {
 #define LP_VLAUNCH(MD)                                                                                    \
   validate_kernel<MASK, MD><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2,     \
                                                             L.g_log2, ck, rid_offset, flags, records, L.rpc, counts, \
-                                                            ticket, list, d_n)
+                                                            ticket, list, d_n, nv)
   if (mode == 0) LP_VLAUNCH(0);
   else if (mode == 1) LP_VLAUNCH(1);
   else if (mode == 3) LP_VLAUNCH(3);
@@ -296,7 +300,7 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
                                                                           int nblocks, int64_t chunk, int per_block,
                                                                           int64_t rid_offset,
                                                                           int64_t* __restrict__ list,
-                                                                          int64_t* __restrict__ d_n) {
+                                                                          int64_t* __restrict__ d_n, NvlsCount nv) {
   // counting block i (i < nblocks) owns flags [i*chunk, (i+1)*chunk); this scatter block
   // owns counting blocks [b*per_block, (b+1)*per_block).  Its output offset is the sum of
   // the counts before its first counting block (block 0 also publishes the total).
@@ -329,7 +333,10 @@ __global__ void __launch_bounds__(kCompactThreads) compact_scatter_kernel(const 
       a += red[1][w];
     }
     s_base = m;
-    if (blockIdx.x == 0) *d_n = a;
+    if (blockIdx.x == 0) {
+      *d_n = a;
+      nvls_publish(nv, a);
+    }
   }
   __syncthreads();
   long long base = s_base;
@@ -713,8 +720,10 @@ size_t validate_counts_bytes(const RegionGeom& g, int sm_count) {
 
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
                             uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
-                            int64_t* list, int64_t* d_n, uint32_t* ticket) {
+                            int64_t* list, int64_t* d_n, uint32_t* ticket, const NvlsCount* nvc) {
   const int row_bytes = g.RN * g.es;
+  NvlsCount nv{nullptr, nullptr, 1};
+  if (nvc && !records) nv = *nvc;
   const int cpr = row_bytes / 16;
   int cpr_log2 = 0;
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
@@ -729,7 +738,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
 #define LP_VCASE(M)                                                                                          \
   case M:                                                                                                    \
     e = validate_dispatch_mode<M>(mode, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                \
-                                  (const uint32_t*)ck, g.rid_offset, flags, records, counts, tk, list, d_n);\
+                                  (const uint32_t*)ck, g.rid_offset, flags, records, counts, tk, list, d_n, nv);\
     break;
     LP_VCASE(1)
     LP_VCASE(2)
@@ -759,7 +768,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   cfg.numAttrs = 1;
   return cudaLaunchKernelEx(&cfg, compact_scatter_kernel, (const uint8_t*)flags, (int64_t)g.R,
                             (const uint32_t*)counts, (int)L.grid.x, (int64_t)L.rpc, per, (int64_t)g.rid_offset,
-                            list, d_n);
+                            list, d_n, nv);
 }
 
 size_t compact_scratch_bytes(int64_t R) {
@@ -777,7 +786,7 @@ cudaError_t launch_compact(const RegionGeom& g, const uint8_t* flags, uint32_t* 
   int sg, per;
   scatter_grid(nb, sg, per);
   compact_scatter_kernel<<<sg, kCompactThreads, 0, st>>>(flags, g.R, block_counts, (int)nb, kCompactChunk, per,
-                                                         g.rid_offset, list, d_n);
+                                                         g.rid_offset, list, d_n, NvlsCount{nullptr, nullptr, 1});
   return cudaGetLastError();
 }
 
@@ -811,6 +820,16 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const in
   tg.R = T;
   tg.rid_offset = 0;
   return launch_compact(tg, tile_flags, block_counts, tile_list, d_ntiles, st);
+}
+
+__global__ void scale_count_kernel(const int64_t* __restrict__ src, int64_t per, int64_t* __restrict__ dst) {
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+  *dst = *src * per;
+}
+
+cudaError_t launch_scale_count(const int64_t* src, int64_t per, int64_t* dst, cudaStream_t st) {
+  scale_count_kernel<<<1, 1, 0, st>>>(src, per, dst);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,

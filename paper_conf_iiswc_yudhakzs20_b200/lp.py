@@ -32,6 +32,7 @@ FLAG_NO_PAIRING = 4
 FLAG_NO_FUSED_COMPACT = 8
 FLAG_RECOVER_TILE128 = 16
 FLAG_CUCKOO_SHORT_CHAINS = 32
+FLAG_NVLS_COUNT = 64
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
@@ -40,7 +41,8 @@ BODY_NAMES = {"auto": 0, "simt": 1, "tcgen05": 2}
 INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 3}
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",
             "lp_run_protected", "lp_validate", "lp_recover", "lp_region_checksums", "lp_inject", "lp_stats",
-            "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study", "lp_check_recover"]
+            "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study", "lp_check_recover",
+            "lp_attach_nvls_count", "lp_recover_count"]
 
 
 def parse_cksum(spec) -> int:
@@ -100,11 +102,13 @@ def lib():
             "lp_run_protected": [P, pw, P, P, P],
             "lp_validate": [P, pw, P, P, P, I64, P, P, P],
             "lp_recover": [P, pw, P, P, P, P, P, P],
+            "lp_recover_count": [P, pw, P, P, P, P, P, P, P],
             "lp_region_checksums": [P, pw, P, P, P],
             "lp_inject": [P, pw, P, P, P, P, I64, U32, U64, P],
             "lp_stats": [P, pw, P, P, P],
             "lp_fn_study": [P, U32, ctypes.c_int32, I64, U64, I64, P, P, I64, P],
             "lp_check_recover": [P, pw, P, P, P, P],
+            "lp_attach_nvls_count": [P, P, P, ctypes.c_int32],
         }
         for name, args in sig.items():
             f = getattr(L, name)
@@ -225,7 +229,7 @@ class LP:
     def __init__(self, region_m: int, region_n: int, cksum="mod|xor", store="array", device: int = 0,
                  body="auto", hash_seed: int = 0x9747B28C,
                  tc_pair: bool = True, shuffle: bool = True, pairing: bool = True, fused_compact: bool = True,
-                 recover_slices: bool = True, cuckoo_short_chains: bool = False):
+                 recover_slices: bool = True, cuckoo_short_chains: bool = False, nvls_count: bool = False):
         self.mask = parse_cksum(cksum)
         self.store = STORE_NAMES[store] if isinstance(store, str) else int(store)
         self.body = BODY_NAMES[body] if isinstance(body, str) else int(body)
@@ -235,7 +239,8 @@ class LP:
                           (0 if tc_pair else FLAG_TC_1CTA) | (0 if shuffle else FLAG_NO_SHUFFLE) |
                           (0 if pairing else FLAG_NO_PAIRING) | (0 if fused_compact else FLAG_NO_FUSED_COMPACT) |
                           (0 if recover_slices else FLAG_RECOVER_TILE128) |
-                          (FLAG_CUCKOO_SHORT_CHAINS if cuckoo_short_chains else 0))
+                          (FLAG_CUCKOO_SHORT_CHAINS if cuckoo_short_chains else 0) |
+                          (FLAG_NVLS_COUNT if nvls_count else 0))
         h = ctypes.c_void_p()
         _check(lib().lp_config(ctypes.byref(self.cfg), ctypes.byref(h)))
         self._h = h
@@ -280,14 +285,23 @@ class LP:
         _check(lib().lp_validate(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), failed.numel(),
                                  _ptr(d_n), _ptr(workspace), _stream(stream)))
 
-    def recover(self, wl, out, ck, failed, d_n, workspace=None, stream=None):
-        _check(lib().lp_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), _ptr(d_n),
-                                _ptr(workspace), _stream(stream)))
+    def recover(self, wl, out, ck, failed, d_n, workspace=None, stream=None, d_n_recovered=None):
+        """lp_recover; with d_n_recovered (device int64[1]) lp_recover_count: regions rewritten."""
+        if d_n_recovered is None:
+            _check(lib().lp_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), _ptr(d_n),
+                                    _ptr(workspace), _stream(stream)))
+        else:
+            _check(lib().lp_recover_count(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed),
+                                          _ptr(d_n), _ptr(workspace), _ptr(d_n_recovered), _stream(stream)))
 
     def check_recover(self, wl, out, ck, d_n_recovered, stream=None):
         """Listing 7's same-grid check-and-recover (N2): validate + in-place re-execution in one kernel."""
         _check(lib().lp_check_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(d_n_recovered),
                                       _stream(stream)))
+
+    def attach_nvls_count(self, mc_ptr, uc_ptr, world_size: int):
+        """NVLS-fused all-rank failed count (lp_attach_nvls_count); pointers are ints or tensors (None, None: off)."""
+        _check(lib().lp_attach_nvls_count(self._h, _ptr(mc_ptr), _ptr(uc_ptr), int(world_size)))
 
     def region_checksums(self, wl, out, records, stream=None):
         _check(lib().lp_region_checksums(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(records), _stream(stream)))

@@ -62,3 +62,24 @@ def gather_failed(local_failed, group=None):
     outs = [torch.empty_like(pad) for _ in sizes]
     dist.all_gather(outs, pad, group=group)
     return torch.cat([o[:int(s.item())] for o, s in zip(outs, sizes)])
+
+
+def nvls_counter(device, group=None):
+    """A 16 x int64 counter buffer in torch symmetric memory, bound to an NVSwitch multicast object on every
+    rank (the NVLS-fused failed count, lp_attach_nvls_count).  Returns (multicast_ptr, local tensor) or
+    (None, reason) when the fabric offers no multicast (e.g. one GPU, or no NVSwitch)."""
+    import torch
+    import torch.distributed as dist
+    import torch.distributed._symmetric_memory as symm_mem
+
+    try:
+        t = symm_mem.empty(16, dtype=torch.int64, device=device)
+        t.zero_()
+        hdl = symm_mem.rendezvous(t, group if group is not None else dist.group.WORLD)
+        if not getattr(hdl, "has_multicast_support", lambda: False)() or not hdl.multicast_ptr:
+            return None, "symmetric memory without multicast support on this fabric"
+        torch.cuda.synchronize(device)
+        hdl.barrier()
+        return int(hdl.multicast_ptr), t
+    except Exception as e:  # noqa: BLE001 -- reported in the bench line, the NCCL all-reduce stays in place
+        return None, f"{type(e).__name__}: {e}"

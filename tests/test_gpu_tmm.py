@@ -85,7 +85,23 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     if mode in ("bitflip",):
         assert set(got_failed.tolist()) == injected          # a bit flip always changes MOD and XOR
     # (8) recover -> out == golden byte-for-byte, records == golden, re-validate == 0
-    h.recover(wl, out, ck, failed, d_n, ws if recover_ws else None)
+    d_rec = torch.full((1,), -1, dtype=torch.int64, device=out.device)
+    h.recover(wl, out, ck, failed, d_n, ws if recover_ws else None, d_n_recovered=d_rec)
+    torch.cuda.synchronize()
+    # regions rewritten (lp_recover_count): failed regions, or whole de-duplicated tiles / slices
+    tc = body == "tcgen05" or (body == "auto" and in_dt != "i32")
+    if not tc or (RM == 128 and in_dt == "bf16"):
+        exp_rec = nf
+    else:
+        EM = 128 if in_dt == "bf16" else 256
+        EN = 64 if (in_dt == "bf16" and RM == 32 and pairing and recover_slices) else EM
+        if not recover_ws:
+            exp_rec = nf * (EM // RM) * (EM // RN)
+        else:
+            Q = N // RN
+            tiles = {((r // Q) * RM // EM, (r % Q) * RN // EN) for r in got_failed.tolist()}
+            exp_rec = len(tiles) * (EM // RM) * (EN // RN)
+    assert int(d_rec.item()) == exp_rec, (int(d_rec.item()), exp_rec, nf)
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0

@@ -131,3 +131,41 @@ def test_validate_graph_replay_and_large_table():
             torch.cuda.synchronize()
             n = int(d_n.item())
             assert n == 37 and np.array_equal(failed[:n].cpu().numpy(), bad), (M, reg)
+
+
+@pytest.mark.parametrize("R_big", [False, True])
+def test_nvls_count_single_gpu_emulation(R_big):
+    """lp_attach_nvls_count in its single-GPU emulation (mc == uc, world 1): the CTA that finalises the failed
+    count (fused last-CTA compaction for R <= 16384, the scatter launch above) publishes it into the counter
+    buffer with the epoch / parity / arrival protocol of the NVLS path; slot 4 must equal the count of every
+    successive validate, slot 3 the epoch.  (The multimem.red path itself needs >= 2 NVSwitch-connected GPUs:
+    a 1-device multicast object cannot be created.)"""
+    from lpsynth import device_fill
+    M, N = (2048, 2048) if not R_big else (8192, 8192)
+    reg = 32 if R_big else 128
+    a = torch.empty((M, 64), dtype=torch.bfloat16, device="cuda")
+    b = torch.empty((64, N), dtype=torch.bfloat16, device="cuda")
+    device_fill(a, 1, "uniform", "bf16")
+    device_fill(b, 2, "uniform", "bf16")
+    h = lp.LP(reg, reg, cksum="mod|xor", nvls_count=True)
+    wl = lp.Workload.tmm(a, b, out_dtype="bf16")
+    out, ck, failed, d_n, ws = h.alloc(wl)
+    cnt = torch.zeros(16, dtype=torch.int64, device="cuda")
+    h.attach_nvls_count(cnt, cnt, 1)
+    h.cksum_init(wl, ck)
+    h.run_protected(wl, out, ck)
+    R = h.num_regions(wl)
+    assert (R > 16384) == R_big
+    stale = torch.zeros_like(out)
+    for epoch, frac in enumerate([0.0, 0.05, 0.01, 0.2], start=1):
+        if frac:
+            inj = torch.from_numpy(lp.choose_regions(R, frac, 40 + epoch)).cuda()
+            h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=epoch)
+        h.validate(wl, out, ck, failed, d_n, ws)
+        torch.cuda.synchronize()
+        assert int(cnt[4].item()) == int(d_n.item()) and int(cnt[3].item()) == epoch
+        h.recover(wl, out, ck, failed, d_n, ws)
+    h.attach_nvls_count(None, None, 1)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    torch.cuda.synchronize()
+    assert int(cnt[3].item()) == 4 and int(d_n.item()) == 0

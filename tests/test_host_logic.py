@@ -208,3 +208,18 @@ def test_bench_self_launch_reference_two_ranks():
     assert len(lines) == 1
     d = json.loads(lines[0])
     assert d["impl"] == "reference" and d["n_gpus"] == 2 and d["value"] > 0
+
+
+def test_nvls_attach_argument_errors():
+    """lp_attach_nvls_count is host-checked (no GPU needed): the config flag is required, both addresses are
+    needed, 64-B alignment, the single-GPU emulation only with world 1; NULL, NULL detaches."""
+    from paper_conf_iiswc_yudhakzs20_b200 import lp
+    h = lp.LP(128, 128, cksum="mod|xor")
+    with pytest.raises(lp.LPError):
+        h.attach_nvls_count(4096, 4096, 1)                 # flag missing
+    h2 = lp.LP(128, 128, cksum="mod|xor", nvls_count=True)
+    for args in [(4096, None, 2), (4096, 8192 + 8, 2), (4096, 4096, 2), (4096, 8192, 0)]:
+        with pytest.raises(lp.LPError):
+            h2.attach_nvls_count(*args)
+    h2.attach_nvls_count(4096, 8192, 8)                    # accepted (no device access at attach time)
+    h2.attach_nvls_count(None, None, 1)
