@@ -117,7 +117,8 @@ def kernels_per_step(W, store, R):
         rec = 4                                        # tile mark, count, scatter, 3xTF32 list mode
     else:
         rec = 1
-    rec += 1                                           # recovered-region count (lp_recover_count)
+    if not (W["kind"] == "tmm" and W["in_dt"] == "bf16" and W.get("body") != "simt"):
+        rec += 1                                       # recovered-region count (lp_recover_count) launch
     if store.startswith("cuckoo"):
         body += 1                                      # cuckoo rehash check after the body (and after recovery)
         rec += 1
@@ -144,6 +145,8 @@ def parse():
                     help="tcgen05 recovery: one 128x128 tile per failed tile (no same-row pairing) -- A/B switch")
     ap.add_argument("--inject-frac", type=float, default=None,
                     help="override the workload's injected fraction of regions (design-space runs)")
+    ap.add_argument("--recover-slices128", action="store_true",
+                    help="tcgen05 recovery of 128x128 regions: 128x64 slice tasks instead of paired tiles -- A/B switch")
     ap.add_argument("--recover-tile128", action="store_true",
                     help="tcgen05 recovery of 32x32 regions: 128x128 tiles instead of 128x64 slices -- A/B switch")
     ap.add_argument("--nvls-count", action="store_true",
@@ -367,7 +370,7 @@ def run_ours(args):
             nvls_note = "needs N > 1 over NCCL; NCCL/no all-reduce used"
     h = lp.LP(RM, RN, cksum=W["cksum"], store=W["store"], device=local, body=W.get("body", "auto"),
               shuffle=not args.no_shuffle, pairing=not args.no_pairing, recover_slices=not args.recover_tile128,
-              nvls_count=nvls_mc is not None)
+              nvls_count=nvls_mc is not None, recover_slices128=args.recover_slices128)
     if nvls_mc is not None:
         h.attach_nvls_count(nvls_mc, nvls_buf, world)
     h0 = lp.LP(RM, RN, cksum=0, device=local, body=W.get("body", "auto"))   # unprotected twin (overhead denominator)

@@ -138,8 +138,11 @@ typedef enum {
                                    tasks (A/B switch; both re-execute every failed region, L51-57) */
   LP_FLAG_CUCKOO_SHORT_CHAINS = 32u, /* cuckoo stores, test hook: the body's inserts give up after 16 evictions
                                        instead of 128, so entries reach the stash and the rehash (L270) runs */
-  LP_FLAG_NVLS_COUNT = 64u /* allow lp_attach_nvls_count: lp_validate all-reduces the failed count through an
+  LP_FLAG_NVLS_COUNT = 64u, /* allow lp_attach_nvls_count: lp_validate all-reduces the failed count through an
                               NVSwitch multicast counter (multimem.red) from the CTA that finalises it */
+  LP_FLAG_RECOVER_SLICES128 = 128u /* tcgen05 bf16 recovery of 128x128 regions: two 128x64 slices per failed region,
+                                      grouped 1-4 per task (finer load balance; the two slice partial records are
+                                      combined across tasks) instead of same-row pairs of 128x128 tiles (A/B switch) */
 } lp_config_flags;
 
 typedef struct {

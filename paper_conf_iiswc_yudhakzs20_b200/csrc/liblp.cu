@@ -196,7 +196,8 @@ int64_t dedupe_capacity(const lp::RegionGeom& g) {
 }
 
 struct WsLayout {
-  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, d_ntasks, ticket, total;
+  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, tasks_tmp, d_ntasks, part, cnt, ticket,
+      total;
 };
 
 WsLayout ws_layout(const lp::RegionGeom& g) {
@@ -211,9 +212,16 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   w.tile_counts = w.tile_flags + al((size_t)T);
   w.tile_list = w.tile_counts + al(lp::compact_scratch_bytes(T));
   w.d_ntiles = w.tile_list + al((size_t)T * 8);
-  w.tasks = w.d_ntiles + 256;                       // paired recovery tasks: int32[max(R, T)]
-  w.d_ntasks = w.tasks + al((size_t)(g.R > T ? g.R : T) * 4);
-  w.ticket = w.d_ntasks + 256;                      // fused-compaction ticket (u32; zero-initialised, kept at 0)
+  const size_t ntask_bytes = al((size_t)(g.R > T ? g.R : T) * 4);
+  w.tasks = w.d_ntiles + 256;                       // recovery tasks, size-sorted + snake order: int32[max(R, T)]
+  w.tasks_tmp = w.tasks + ntask_bytes;              // the same tasks in row order (grouping output)
+  w.d_ntasks = w.tasks_tmp + ntask_bytes;
+  // 128x128 regions recovered as 128x64 slices: per-region slice partials {2 x CkRecord} + arrival counter
+  // (zero-initialised, reset by the finishing slice)
+  const size_t npart = g.RM == 128 ? (size_t)g.R : 0;
+  w.part = w.d_ntasks + 256;
+  w.cnt = w.part + al(npart * 32);
+  w.ticket = w.cnt + al(npart * 4);                 // fused-compaction ticket (u32; zero-initialised, kept at 0)
   w.total = w.ticket + 256;
   return w;
 }
@@ -252,6 +260,8 @@ lp::TmmArgs tmm_args(const lp_ctx* h, const lp_workload_t* wl, const lp::RegionG
   a.d_n = d_n;
   a.list_is_tiles = 0;
   a.slice64 = 0;
+  a.slice_part = nullptr;
+  a.slice_cnt = nullptr;
   a.tasks = nullptr;
   a.d_ntasks = nullptr;
   a.force_1cta = (h->cfg.flags & LP_FLAG_TC_1CTA) ? 1 : 0;
@@ -290,7 +300,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.d_n = d_n;
     a.sm_count = h->sm_count;
     cudaError_t e = lp::launch_stencil(a, st);
-    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
+    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, 1, d_rec, st);
     return e == cudaSuccess ? ok() : cuda_fail(e, "stencil launch");
   }
   if (wl->kind == LP_WL_SPMV) {
@@ -317,7 +327,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     a.no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) ? 1 : 0;
     a.sm_count = h->sm_count;
     cudaError_t e = lp::launch_spmv(a, st);
-    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
+    if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, 1, d_rec, st);
     return e == cudaSuccess ? ok() : cuda_fail(e, "SPMV launch");
   }
   if (!wl->a || !wl->b) return fail(LP_ERR_INVALID_ARG, "null A or B");
@@ -335,11 +345,17 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
                   "tcgen05 body needs 16-B aligned pitches, region 128x128 or 32x32, and either bf16 input with "
                   "m%%128 == 0, n%%128 == 0, k%%64 == 0, or fp32 input/output with m, n %% 256 == 0, k %% 32 == 0");
     const int E = tc_ok ? 128 : 256;  // tile edge of the list-mode kernel
-    const bool need_dedupe = tf_ok ? true : (g.RM == 32);
     const bool pairing = !(h->cfg.flags & LP_FLAG_NO_PAIRING);
-    // bf16 32x32 regions: de-duplicate into 128x64 slices and group up to four slices of a row band per
-    // N = 256 task (1.7x less re-executed work than 128x128 tiles at 5% failed regions, same A panel reuse)
-    const bool slices = tc_ok && g.RM == 32 && pairing && !(h->cfg.flags & LP_FLAG_RECOVER_TILE128);
+    // bf16: failed regions become 128x64 slices, grouped 1-4 per N = 64..256 task of one row band.
+    //  - 32x32 regions: de-duplicated (1.7x less re-executed work than 128x128 tiles at 5% failed);
+    //  - 128x128 regions, with LP_FLAG_RECOVER_SLICES128 (A/B switch; measured slower): two
+    //    slices each, so k-slice tasks can fill every SM (205 failed regions on 148 SMs: 410 slices in tasks
+    //    of 3 instead of 103 paired 128x256 tasks); a region's two slice partial records are combined
+    //    across tasks in the workspace (epi_finish_slice128).  Default: paired 128x128 tiles.
+    const bool slices = tc_ok && pairing &&
+                        ((g.RM == 32 && !(h->cfg.flags & LP_FLAG_RECOVER_TILE128)) ||
+                         (g.RM == 128 && h->mask != 0 && (h->cfg.flags & LP_FLAG_RECOVER_SLICES128)));
+    const bool need_dedupe = tf_ok ? true : (g.RM == 32 || slices);
     const int EN = slices ? 64 : E;
     if (list && workspace && need_dedupe && dedupe_tiles(g, E, EN) > 0) {
       // several failed regions may share one tensor-core tile: recompute each tile once
@@ -353,16 +369,27 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
       a.d_n = (const int64_t*)(ws + w.d_ntiles);
       a.list_is_tiles = 1;
       a.slice64 = slices ? 1 : 0;
+      if (slices && g.RM == 128) {
+        a.slice_part = (void*)(ws + w.part);
+        a.slice_cnt = (uint32_t*)(ws + w.cnt);
+      }
     }
+    // regions rewritten = entries of the list the kernel consumes x regions per entry (a de-duplicated
+    // tile / slice rewrites every region inside it; without a workspace every listed region recomputes its
+    // whole E x E tile): reported by the grouping kernel when it runs, else by a one-thread launch
+    const int64_t rec_num = (int64_t)E * (a.list_is_tiles ? EN : E), rec_den = (int64_t)g.RM * g.RN;
+    bool rec_done = false;
     if (list && workspace && tc_ok && (a.list_is_tiles || g.RM == 128) && pairing) {
       // pair failed 128x128 tiles of the same row band into 128x256 tasks (or group up to four 128x64 slices)
       const WsLayout w = ws_layout(g);
       uint8_t* ws = (uint8_t*)workspace;
       const int64_t off = a.list_is_tiles ? 0 : g.rid_offset;
       const int64_t div = a.list_is_tiles ? g.N / EN : g.Q;
-      cudaError_t e0 = lp::launch_pair_tasks(a.list, a.d_n, off, div, h->sm_count, a.slice64 ? 4 : 2,
-                                             (int32_t*)(ws + w.tasks),
-                                             (int64_t*)(ws + w.d_ntasks), st);
+      const int grid = (int)(g.R < h->sm_count ? g.R : h->sm_count);  // the re-execution grid (launch_cfg)
+      cudaError_t e0 = lp::launch_pair_tasks(a.list, a.d_n, off, div, h->sm_count, a.slice64 ? 4 : 2, grid,
+                                             (int32_t*)(ws + w.tasks_tmp), (int32_t*)(ws + w.tasks),
+                                             (int64_t*)(ws + w.d_ntasks), d_rec, rec_num, rec_den, st);
+      rec_done = d_rec != nullptr;
       if (e0 != cudaSuccess) return cuda_fail(e0, "recovery pairing");
       a.tasks = (const int32_t*)(ws + w.tasks);
       a.d_ntasks = (const int64_t*)(ws + w.d_ntasks);
@@ -370,12 +397,8 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     const char* why = nullptr;
     cudaError_t e = tc_ok ? lp::launch_tmm_tc(a, st, &why) : lp::launch_tmm_tf32(a, st, &why);
     if (e != cudaSuccess) return why ? fail(LP_ERR_CUDA, "tcgen05 launch: %s", why) : cuda_fail(e, "tcgen05 launch");
-    if (list && d_rec) {
-      // regions rewritten = entries of the list the kernel consumed x regions per entry (a de-duplicated
-      // tile / slice rewrites every region inside it)
-      // (without a workspace every listed region recomputes its whole E x E tile)
-      const int64_t per = (int64_t)(E / g.RM) * ((a.list_is_tiles ? EN : E) / g.RN);
-      e = lp::launch_scale_count(a.d_n, per, d_rec, st);
+    if (list && d_rec && !rec_done) {
+      e = lp::launch_scale_count(a.d_n, rec_num, rec_den, d_rec, st);
       if (e != cudaSuccess) return cuda_fail(e, "recovered-count launch");
     }
     return ok();
@@ -384,7 +407,7 @@ lp_status run_body(lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, 
     return fail(LP_ERR_UNSUPPORTED, "SIMT body supports 32x32, 64x64 and 128x128 regions");
   if (wl->k % 16) return fail(LP_ERR_UNSUPPORTED, "SIMT body needs k %% 16 == 0");
   cudaError_t e = lp::launch_tmm_simt(a, st);
-  if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, d_rec, st);
+  if (e == cudaSuccess && list && d_rec) e = lp::launch_scale_count(d_n, 1, 1, d_rec, st);
   return e == cudaSuccess ? ok() : cuda_fail(e, "SIMT TMM launch");
 }
 
@@ -416,7 +439,8 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->body < LP_BODY_AUTO || cfg->body > LP_BODY_TCGEN05) return fail(LP_ERR_INVALID_ARG, "unknown body %d", cfg->body);
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING | LP_FLAG_NO_FUSED_COMPACT |
-                                 LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS | LP_FLAG_NVLS_COUNT))
+                                 LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS | LP_FLAG_NVLS_COUNT |
+                                 LP_FLAG_RECOVER_SLICES128))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");

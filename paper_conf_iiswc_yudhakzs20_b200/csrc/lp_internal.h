@@ -48,12 +48,17 @@ cudaError_t launch_inject(const RegionGeom& g, uint32_t mask, const HashInfo& hi
 // ascending list of 128x128 tiles/regions -> recovery tasks of 1-2 entries of the same row band
 // (row = (list[i] - off) / div); pairing only when *d_n > min_pair.  tasks[t] = (i << 1) | paired.
 // G = 4: tasks of up to four entries (128x64 slices), tasks[t] = (i << 2) | (count - 1).
+// The tasks are then ordered by size (largest first) and dealt to the `grid` persistent CTAs of the
+// re-execution kernel in alternating direction (CTA i runs positions i, i + grid, ...): an LPT-like static
+// schedule.  tasks_tmp: scratch of the same size as tasks.  d_rec (optional) <- *d_n * rec_num / rec_den,
+// the regions the re-execution will rewrite (lp_recover_count), so no separate count launch is needed.
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
-                              int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st);
+                              int G, int grid, int32_t* tasks_tmp, int32_t* tasks, int64_t* d_ntasks,
+                              int64_t* d_rec, int64_t rec_num, int64_t rec_den, cudaStream_t st);
 // cuckoo stores: rebuild T1/T2 with a new seed if the stash is non-empty (no-op otherwise)
 cudaError_t launch_cuckoo_rehash(void* ck, cudaStream_t st);
-// *dst = *src * per on the device (recovered-region count of a list-mode recovery)
-cudaError_t launch_scale_count(const int64_t* src, int64_t per, int64_t* dst, cudaStream_t st);
+// *dst = *src * num / den on the device (recovered-region count of a list-mode recovery)
+cudaError_t launch_scale_count(const int64_t* src, int64_t num, int64_t den, int64_t* dst, cudaStream_t st);
 cudaError_t launch_stats(const HashInfo& hi, const void* ck, int64_t* d_stats, cudaStream_t st);
 // failed regions -> unique tile ids of an EM x EN tile grid (tile = (p*RM/EM)*(N/EN) + q*RN/EN), ascending
 cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const int64_t* list, const int64_t* d_n,
@@ -80,6 +85,8 @@ struct TmmArgs {
   const int64_t* d_n;
   int list_is_tiles;    // list holds 128x128 tile ids (de-duplicated recovery of 32x32 regions)
   int slice64;          // with list_is_tiles: ids are 128x64 slices, a task is 1-4 slices of one row band (N = 64..256)
+  void* slice_part;     // 128x128 regions as slices: per-region {2 x CkRecord} partials (workspace)
+  uint32_t* slice_cnt;  //   and per-region arrival counters (zero-initialised, self-resetting)
   const int32_t* tasks;  // tcgen05 list mode: paired recovery tasks (launch_pair_tasks), or null
   const int64_t* d_ntasks;
   int force_1cta;       // tcgen05: use the 1-CTA 128x256 kernel even where the CTA-pair kernel applies

@@ -9,6 +9,8 @@
 // recovery re-executes only those.
 #include <cuda_runtime.h>
 #include <stdint.h>
+
+#include <cstdlib>
 #include <stdlib.h>
 
 #include "lp_device.cuh"
@@ -379,14 +381,19 @@ static void scatter_grid(int64_t nblocks, int& grid, int& per_block) {
 }
 
 // ---------------------------------------------------------------------------
+// Every tile of the EM x EN grid that a failed RM x RN region overlaps (a region may hold several tiles --
+// 128x128 regions as two 128x64 slices -- or a tile several regions -- 32x32 regions in a 128x64 slice).
 __global__ void tile_mark_kernel(const int64_t* __restrict__ list, const int64_t* __restrict__ d_n,
-                                 int64_t rid_offset, int64_t Q, int64_t tiles_per_row, int per_m, int per_n,
+                                 int64_t rid_offset, int64_t Q, int64_t tiles_per_row, int RM, int RN, int EM, int EN,
                                  uint8_t* __restrict__ tile_flags) {
   const int64_t n = *d_n;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t rid = list[i] - rid_offset;
     const int64_t p = rid / Q, q = rid - p * Q;
-    tile_flags[(p / per_m) * tiles_per_row + q / per_n] = 1;  // idempotent plain store
+    const int64_t r0 = p * RM / EM, r1 = (p * RM + RM - 1) / EM;
+    const int64_t c0 = q * RN / EN, c1 = (q * RN + RN - 1) / EN;
+    for (int64_t r = r0; r <= r1; ++r)
+      for (int64_t c = c0; c <= c1; ++c) tile_flags[r * tiles_per_row + c] = 1;  // idempotent plain store
   }
 }
 
@@ -461,7 +468,10 @@ constexpr int kPairPer = 4;  // entries per thread per block pass (4096 per pass
 
 __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t* __restrict__ list,
                                                                   const int64_t* __restrict__ d_n, int64_t off,
-                                                                  int64_t div, int64_t min_pair, int G,
+                                                                  int64_t div, int64_t min_pair, int G, int grid,
+                                                                  int lpt, int64_t* __restrict__ d_rec,
+                                                                  int64_t rec_num, int64_t rec_den,
+                                                                  int32_t* __restrict__ tasks_tmp,
                                                                   int32_t* __restrict__ tasks,
                                                                   int64_t* __restrict__ d_ntasks) {
   __shared__ int64_t s_max[32];
@@ -470,6 +480,7 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
   // the re-execution grid that follows may start its prologue now (it waits for this grid to finish)
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const int64_t n = *d_n;
+  if (d_rec && threadIdx.x == 0) *d_rec = n * rec_num / rec_den;  // regions the re-execution will rewrite
   const bool pairing = n > min_pair;
   const int sh = G == 4 ? 2 : 1;
   // slice grouping (G = 4): as many entries per task as it takes to fill the SMs once, 2..4
@@ -514,11 +525,71 @@ __global__ void __launch_bounds__(kPairThreads) pair_tasks_kernel(const int64_t*
     }
     int tot;
     const int idx = block_scan_excl_sum(nh, s_sum, &tot);
-    for (int k = 0; k < nh; ++k) tasks[carry_t + idx + k] = w[k];
+    for (int k = 0; k < nh; ++k) tasks_tmp[carry_t + idx + k] = w[k];
     carry_t += tot;
     carry_ls = blk_max > carry_ls ? blk_max : carry_ls;
   }
-  if (threadIdx.x == 0) *d_ntasks = carry_t;
+  // Static LPT-like schedule for the persistent re-execution grid (CTA c runs positions c, c + grid, ...):
+  // tasks sorted by entry count, largest first (stable), dealt round by round; the LAST round goes
+  // forward (it may be partial and must land on CTAs 0..L-1) and the rounds alternate direction
+  // backwards from it, so a CTA that got a small task in one round gets a large one in the next.
+  const int64_t T = carry_t;
+  const int mask = (1 << sh) - 1;
+  __shared__ int s_cls[5], s_off[5];
+  if (threadIdx.x < 5) s_cls[threadIdx.x] = 0;
+  __syncthreads();
+  for (int64_t i = threadIdx.x; i < T; i += kPairThreads) atomicAdd(&s_cls[(tasks_tmp[i] & mask) + 1], 1);
+  __syncthreads();
+  if (threadIdx.x == 0) {  // start of each size class in the sorted order (larger classes first)
+    int acc = 0;
+    for (int c = 4; c >= 1; --c) {
+      s_off[c] = acc;
+      acc += s_cls[c];
+    }
+  }
+  __syncthreads();
+  const int64_t nr = (T + grid - 1) / grid;
+  for (int64_t base = 0; base < T; base += kPairThreads) {
+    const int64_t i = base + threadIdx.x;
+    const int32_t w = i < T ? tasks_tmp[i] : 0;
+    const int c = i < T ? (w & mask) + 1 : 0;
+    // stable rank inside the size class (one ballot-based block scan over the 4 class flags at once:
+    // each class's count fits 10 bits of a packed 64-bit word)
+    const unsigned long long f = c ? (1ull << (16 * (c - 1))) : 0ull;
+    unsigned long long x = f;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(0xFFFFFFFFu, x, o);
+      if (lane >= o) x += y;
+    }
+    __shared__ unsigned long long s_w[32];
+    if (lane == 31) s_w[wid] = x;
+    __syncthreads();
+    if (wid == 0) {
+      unsigned long long t = s_w[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long y = __shfl_up_sync(0xFFFFFFFFu, t, o);
+        if (lane >= o) t += y;
+      }
+      s_w[lane] = t;
+    }
+    __syncthreads();
+    const unsigned long long excl = (wid ? s_w[wid - 1] : 0ull) + x - f;
+    const unsigned long long tot = s_w[31];
+    if (i < T) {
+      const int rank = (int)((excl >> (16 * (c - 1))) & 0xFFFFull);
+      const int64_t srt = s_off[c] + rank;  // position in the sorted order
+      const int64_t r = srt / grid, k = srt - r * grid;
+      const int64_t cta = ((nr - 1 - r) & 1) ? (grid - 1 - k) : k;
+      tasks[lpt ? r * grid + cta : i] = w;
+    }
+    __syncthreads();
+    if (threadIdx.x < 4) s_off[threadIdx.x + 1] += (int)((tot >> (16 * threadIdx.x)) & 0xFFFFull);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) *d_ntasks = T;
 }
 
 __global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed, uint32_t max_evict) {
@@ -813,7 +884,7 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const in
   cudaError_t e = cudaMemsetAsync(tile_flags, 0, (size_t)T, st);
   if (e != cudaSuccess) return e;
   tile_mark_kernel<<<(unsigned)(g.R < 148 * 4 * 256 ? (g.R + 255) / 256 : 148 * 4), 256, 0, st>>>(
-      list, d_n, g.rid_offset, g.Q, g.N / EN, EM / g.RM, EN / g.RN, tile_flags);
+      list, d_n, g.rid_offset, g.Q, g.N / EN, g.RM, g.RN, EM, EN, tile_flags);
   e = cudaGetLastError();
   if (e != cudaSuccess) return e;
   RegionGeom tg = g;
@@ -822,19 +893,26 @@ cudaError_t launch_tiles_of_failed(const RegionGeom& g, int EM, int EN, const in
   return launch_compact(tg, tile_flags, block_counts, tile_list, d_ntiles, st);
 }
 
-__global__ void scale_count_kernel(const int64_t* __restrict__ src, int64_t per, int64_t* __restrict__ dst) {
+__global__ void scale_count_kernel(const int64_t* __restrict__ src, int64_t num, int64_t den,
+                                   int64_t* __restrict__ dst) {
   asm volatile("griddepcontrol.wait;" ::: "memory");
-  *dst = *src * per;
+  *dst = *src * num / den;
 }
 
-cudaError_t launch_scale_count(const int64_t* src, int64_t per, int64_t* dst, cudaStream_t st) {
-  scale_count_kernel<<<1, 1, 0, st>>>(src, per, dst);
+cudaError_t launch_scale_count(const int64_t* src, int64_t num, int64_t den, int64_t* dst, cudaStream_t st) {
+  scale_count_kernel<<<1, 1, 0, st>>>(src, num, den, dst);
   return cudaGetLastError();
 }
 
 cudaError_t launch_pair_tasks(const int64_t* list, const int64_t* d_n, int64_t off, int64_t div, int64_t min_pair,
-                              int G, int32_t* tasks, int64_t* d_ntasks, cudaStream_t st) {
-  pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, G, tasks, d_ntasks);
+                              int G, int grid, int32_t* tasks_tmp, int32_t* tasks, int64_t* d_ntasks,
+                              int64_t* d_rec, int64_t rec_num, int64_t rec_den, cudaStream_t st) {
+  static const int lpt = [] {  // LP_TASK_ORDER=row keeps the grouping's row order (A/B runs)
+    const char* e = getenv("LP_TASK_ORDER");
+    return (e && e[0] == 'r') ? 0 : 1;
+  }();
+  pair_tasks_kernel<<<1, kPairThreads, 0, st>>>(list, d_n, off, div, min_pair, G, grid < 1 ? 1 : grid, lpt, d_rec,
+                                                rec_num, rec_den < 1 ? 1 : rec_den, tasks_tmp, tasks, d_ntasks);
   return cudaGetLastError();
 }
 

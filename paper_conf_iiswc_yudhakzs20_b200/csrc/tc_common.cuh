@@ -95,6 +95,9 @@ struct TileSrc {
   int64_t n128;               // 128-column tiles per row (tile-id decoding)
   int slice64;                // list holds 128x64 slice ids (n64 per row); a task is 1-4 slices (slices())
   int64_t n64;
+  int l2_prefetch;            // list mode: k-blocks of the task's operands prefetched into L2 ahead of the ring
+  CkRecord* part;             // 128x128 regions as slices: per-region {2 x CkRecord} partials
+  uint32_t* cnt;              //   per-region arrival counters (epi_finish_slice128)
   __device__ __forceinline__ int64_t count() const {
     return tasks ? *d_ntasks : (list ? *d_n : num_m * num_n);
   }
@@ -207,7 +210,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
       for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
       if constexpr (MASK != 0) {
         // byte position of word 0 of this chunk inside its region's stream
-        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((n0 + ch * 32) & 127) * ES + 1)
                                          : (uint32_t)(lane * 32 * ES + 1);
 #pragma unroll
         for (int i = 0; i < 4; ++i) part.add4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3], pos0 + 16 * i);
@@ -237,7 +240,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
       for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
       if (!final_pass) continue;
       if constexpr (MASK != 0) {
-        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((ch * 32) & 127) * ES + 1)
+        const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((n0 + ch * 32) & 127) * ES + 1)
                                          : (uint32_t)(lane * 32 * ES + 1);
 #pragma unroll
         for (int i = 0; i < 8; ++i) part.add4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3], pos0 + 16 * i);
@@ -255,8 +258,8 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
           store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
         }
         part = CkPartial<MASK>();
-      } else if ((ch & 3) == 3) {
-        // end of a 128-column region: warp partial -> shared slot
+      } else if ((ch & 3) == 3 || ch == NCH - 1) {
+        // end of a 128-column region (or of a 64-column slice of one): warp partial -> shared slot
         const CkRecord rec = warp_reduce<MASK>(part);
         if (lane == 0) srec_acc[(ch / 4) * 4 + wq] = rec;
         part = CkPartial<MASK>();
@@ -302,6 +305,43 @@ __device__ __forceinline__ void epi_finish_halves(int warp, int lane, const CkRe
     uint32_t words[3];
     record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
     store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+  }
+}
+
+// One 128x64 slice of a 128x128 region (recovery of 128x128 regions as slices): combine the 4 warp
+// partials of the slice, publish them as half h of the region's partial record in the workspace, and
+// let the second of the region's two slices to finish -- in this task or another CTA's -- combine both
+// halves and store the record (the record words depend only on the combined sums, not on the order).
+// Ordering: partial store, gpu-scope fence, arrival RMW; the finisher fences before reading the other
+// half through L2 and resets the counter for the next recovery.
+template <typename OutT, uint32_t MASK, int STORE>
+__device__ __forceinline__ void epi_finish_slice128(int warp, int lane, const CkRecord* srec_slot,
+                                                    uint32_t* __restrict__ ck, int64_t m128, int64_t n0, int64_t Qr,
+                                                    int64_t rid_offset, CkRecord* part, uint32_t* cnt) {
+  constexpr int ES = (int)sizeof(OutT);
+  named_bar_epi();
+  if (warp == kEpiWarp0 && lane == 0) {
+    CkRecord rr = srec_slot[0];
+#pragma unroll
+    for (int w = 1; w < 4; ++w) rr = combine(rr, srec_slot[w]);
+    const int64_t rid = m128 * Qr + n0 / 128;
+    const int h = (int)((n0 >> 6) & 1);
+    volatile uint32_t* dst = reinterpret_cast<volatile uint32_t*>(part + 2 * rid + h);
+    dst[0] = rr.mod;
+    dst[1] = rr.xr;
+    dst[2] = rr.s;
+    dst[3] = rr.wmod;
+    __threadfence();
+    if (atomicAdd(cnt + rid, 1u) == 1u) {
+      __threadfence();
+      const volatile uint32_t* o = reinterpret_cast<const volatile uint32_t*>(part + 2 * rid + (h ^ 1));
+      const CkRecord other{o[0], o[1], o[2], o[3]};
+      rr = combine(rr, other);
+      cnt[rid] = 0u;
+      uint32_t words[3];
+      record_words<MASK>(rr, (uint64_t)128 * 128 * ES, words);
+      store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+    }
   }
 }
 

@@ -31,6 +31,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "lp_device.cuh"
 #include "lp_internal.h"
 #include "lp_ptx.cuh"
@@ -143,7 +145,18 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         const int m0 = (int)(mb * kBM);
         const uint32_t bytes = Cfg::kABytes + nch * (kBK * 128);
+        // recovery reads cold operands (random failed tiles, L2 flushed): keep l2_prefetch k-blocks of this
+        // task's A and B boxes in flight into L2 beyond the smem ring, so the ring's TMA loads hit L2
+        const int pf = src.l2_prefetch;
+        auto prefetch = [&](int kb) {
+          tma_prefetch_2d(&tmap_a, kb * kBK, m0);
+#pragma unroll
+          for (int c = 0; c < BN / 64; ++c)
+            if (c < nch) tma_prefetch_2d(&tmap_b, (int)col[c], kb * kBK);
+        };
+        for (int kb = 0; kb < pf && kb < nkb; ++kb) prefetch(kb);
         for (int kb = 0; kb < nkb; ++kb) {
+          if (pf && kb + pf < nkb) prefetch(kb + pf);
           mbar_wait(&empty[stage], phase ^ 1);
           mbar_expect_tx(&full[stage], bytes);
           tma_load_2d(&tmap_a, &full[stage], sA + stage * Cfg::kABytes, kb * kBK, m0);
@@ -217,6 +230,34 @@ __global__ void __launch_bounds__(kThreads, 1)
       tc_fence_after();
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
       CkRecord* srec_acc = srec + acc * (BN / 128) * 4;
+      if constexpr (REG == 128 && BN == 256 && MASK != 0) {
+        if (src.slice64) {
+          // slice task of 128x128 regions: accumulator columns [64c, 64c+64) = half of region (mb, nc[c] / 128);
+          // the two warp-partial slot sets alternate so the next slice cannot overwrite a set before the
+          // combining warp has read it (it passes the next slice's named barrier only after reading)
+          int64_t mb, nc[4];
+          int cnt;
+          src.slices(t, mb, cnt, nc);
+#pragma unroll 1
+          for (int c = 0; c < cnt; ++c) {
+            CkRecord* slot = srec_acc + (c & 1) * 4;
+            epi_store<OutT, MASK, REG, 64, STORE>(t_row + 64 * c, C, ldc, mb, nc[c], wq, lane, slot, ck, src.Qr,
+                                                  src.rid_offset);
+            if (c == cnt - 1) {
+              tc_fence_before();
+              __syncwarp();
+              if (lane == 0) mbar_arrive(&tempty[acc]);
+            }
+            epi_finish_slice128<OutT, MASK, STORE>(warp, lane, slot, ck, mb, nc[c], src.Qr, src.rid_offset, src.part,
+                                                   src.cnt);
+          }
+          if (++acc == 2) {
+            acc = 0;
+            acc_phase ^= 1;
+          }
+          continue;
+        }
+      }
       if constexpr (REG == 32 && BN == 256) {
         if (src.slice64) {
           // accumulator columns [64c, 64c+64) -> slice c (32x32 records per 32-column chunk)
@@ -565,6 +606,16 @@ cudaError_t launch_maybe_pdl(Kern kfn, unsigned grid, int smem, cudaStream_t st,
   return cudaLaunchKernelEx(&cfg, kfn, args...);
 }
 
+// k-blocks of L2 prefetch distance in list mode (LP_TC_PREFETCH=<n> for A/B runs; default 0 = off: measured
+// slower at 4/8/16 k-blocks -- the re-execution is bound by the L2 -> SM fabric, not by DRAM latency)
+int l2_prefetch_kblocks() {
+  static int v = [] {
+    const char* e = getenv("LP_TC_PREFETCH");
+    return e ? atoi(e) : 0;
+  }();
+  return v;
+}
+
 template <typename OutT, int REG, int BN>
 cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   using Cfg = TcCfg<BN>;
@@ -588,6 +639,9 @@ cudaError_t launch_cfg(const TmmArgs& a, cudaStream_t st, const char** why) {
   src.n128 = a.N / 128;
   src.slice64 = a.slice64;
   src.n64 = a.N / 64;
+  src.part = reinterpret_cast<CkRecord*>(a.slice_part);
+  src.l2_prefetch = a.list ? l2_prefetch_kblocks() : 0;
+  src.cnt = a.slice_cnt;
   const int64_t R = (a.M / REG) * (a.N / REG);
   int64_t grid = a.list ? (R < a.sm_count ? R : a.sm_count) : src.num_m * src.num_n;
   if (grid > a.sm_count) grid = a.sm_count;

@@ -33,6 +33,7 @@ FLAG_NO_FUSED_COMPACT = 8
 FLAG_RECOVER_TILE128 = 16
 FLAG_CUCKOO_SHORT_CHAINS = 32
 FLAG_NVLS_COUNT = 64
+FLAG_RECOVER_SLICES128 = 128
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
@@ -229,7 +230,8 @@ class LP:
     def __init__(self, region_m: int, region_n: int, cksum="mod|xor", store="array", device: int = 0,
                  body="auto", hash_seed: int = 0x9747B28C,
                  tc_pair: bool = True, shuffle: bool = True, pairing: bool = True, fused_compact: bool = True,
-                 recover_slices: bool = True, cuckoo_short_chains: bool = False, nvls_count: bool = False):
+                 recover_slices: bool = True, cuckoo_short_chains: bool = False, nvls_count: bool = False,
+                 recover_slices128: bool = False):
         self.mask = parse_cksum(cksum)
         self.store = STORE_NAMES[store] if isinstance(store, str) else int(store)
         self.body = BODY_NAMES[body] if isinstance(body, str) else int(body)
@@ -240,7 +242,8 @@ class LP:
                           (0 if pairing else FLAG_NO_PAIRING) | (0 if fused_compact else FLAG_NO_FUSED_COMPACT) |
                           (0 if recover_slices else FLAG_RECOVER_TILE128) |
                           (FLAG_CUCKOO_SHORT_CHAINS if cuckoo_short_chains else 0) |
-                          (FLAG_NVLS_COUNT if nvls_count else 0))
+                          (FLAG_NVLS_COUNT if nvls_count else 0) |
+                          (FLAG_RECOVER_SLICES128 if recover_slices128 else 0))
         h = ctypes.c_void_p()
         _check(lib().lp_config(ctypes.byref(self.cfg), ctypes.byref(h)))
         self._h = h

@@ -19,9 +19,10 @@ pytestmark = pytest.mark.gpu
 
 def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_words", frac=0.05, seed=1,
               store="array", check_values=True, recover_ws=True, tc_pair=True, shuffle=True, pairing=True,
-              recover_slices=True, cuckoo_short_chains=False):
+              recover_slices=True, cuckoo_short_chains=False, recover_slices128=False):
     h = lp.LP(RM, RN, cksum=mask, store=store, body=body, tc_pair=tc_pair, shuffle=shuffle, pairing=pairing,
-              recover_slices=recover_slices, cuckoo_short_chains=cuckoo_short_chains)
+              recover_slices=recover_slices, cuckoo_short_chains=cuckoo_short_chains,
+              recover_slices128=recover_slices128)
     A, B = make_inputs(seed, M, N, K, kind, in_dt)
     a, b = host_to_dev(A, in_dt), host_to_dev(B, in_dt)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
@@ -90,17 +91,19 @@ def run_cycle(M, N, K, RM, RN, in_dt, out_dt, kind, mask, body, mode="stale_word
     torch.cuda.synchronize()
     # regions rewritten (lp_recover_count): failed regions, or whole de-duplicated tiles / slices
     tc = body == "tcgen05" or (body == "auto" and in_dt != "i32")
-    if not tc or (RM == 128 and in_dt == "bf16"):
+    if not tc or (RM == 128 and in_dt == "bf16" and not (recover_slices128 and pairing and recover_ws)):
         exp_rec = nf
     else:
         EM = 128 if in_dt == "bf16" else 256
-        EN = 64 if (in_dt == "bf16" and RM == 32 and pairing and recover_slices) else EM
+        EN = 64 if (in_dt == "bf16" and pairing and ((RM == 32 and recover_slices) or
+                                                       (RM == 128 and recover_slices128))) else EM
         if not recover_ws:
             exp_rec = nf * (EM // RM) * (EM // RN)
         else:
             Q = N // RN
-            tiles = {((r // Q) * RM // EM, (r % Q) * RN // EN) for r in got_failed.tolist()}
-            exp_rec = len(tiles) * (EM // RM) * (EN // RN)
+            tiles = {((r // Q) * RM // EM, c) for r in got_failed.tolist()
+                     for c in range((r % Q) * RN // EN, ((r % Q) * RN + RN - 1) // EN + 1)}
+            exp_rec = len(tiles) * EM * EN // (RM * RN)
     assert int(d_rec.item()) == exp_rec, (int(d_rec.item()), exp_rec, nf)
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
@@ -405,3 +408,15 @@ def test_tmm_check_and_recover_full_8192():
     torch.cuda.synchronize()
     assert int(d_rec.item()) == len(exp) > 0
     assert torch.equal(out.view(torch.int16), golden.view(torch.int16))
+
+
+@pytest.mark.parametrize("frac", [0.02, 0.3, 1.0])
+@pytest.mark.parametrize("out_dt", ["bf16", "f32"])
+@pytest.mark.parametrize("store", ["array", "quad_cas"])
+def test_tc_recovery_slices128(frac, out_dt, store):
+    """LP_FLAG_RECOVER_SLICES128 (A/B switch): failed 128x128 regions re-executed as two 128x64 slices grouped
+    1-4 per task in size-sorted snake order; each region's record is combined from its two slice partials,
+    possibly computed by different CTAs.  Recovered bytes and records must equal the golden run."""
+    _, nf = run_cycle(2048, 2560, 256, 128, 128, "bf16", out_dt, "uniform", "mod|xor|adler" if store == "array"
+                      else "mod|xor", "tcgen05", mode="stale_words", frac=frac, store=store, recover_slices128=True)
+    assert nf > 0
