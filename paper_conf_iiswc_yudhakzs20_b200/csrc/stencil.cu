@@ -44,6 +44,33 @@ __device__ __forceinline__ float st5(float c, float u, float d, float l, float r
   return __fadd_rn(__fmul_rn(0.5f, c), __fmul_rn(0.125f, s));
 }
 
+// Adler-32 partials of one lane's column of 16-byte vectors, one vector per region row (kRowsW rows, row
+// pitch row_bytes inside the region's byte stream).  Instead of a 64-bit position multiply per vector
+// (CkPartial::add4), the row index is folded in with a running-sum trick: S chains the byte sums through
+// dp4a, T accumulates S after every row (T = sum_r (n - r) * bs_r), Wl chains the in-vector weights
+// 0..15 through dp4a; then  W = base * S + row_bytes * (n * S - T) + Wl  with base = the 1-based stream
+// position of this lane's first byte.  Exactly the sums of add4 (integer arithmetic), 9 ops per row.
+struct AdlerRows {
+  uint32_t S = 0, T = 0, Wl = 0;
+  __device__ __forceinline__ void add_row(uint32_t x, uint32_t y, uint32_t z, uint32_t v) {
+    S = (uint32_t)__dp4a(x, 0x01010101u, __dp4a(y, 0x01010101u, __dp4a(z, 0x01010101u, __dp4a(v, 0x01010101u, S))));
+    Wl = (uint32_t)__dp4a(x, 0x03020100u, __dp4a(y, 0x07060504u, __dp4a(z, 0x0B0A0908u, __dp4a(v, 0x0F0E0D0Cu, Wl))));
+    T += S;
+  }
+  template <uint32_t MASK>
+  __device__ __forceinline__ void fold(CkPartial<MASK>& p, uint32_t base, uint32_t nrows, uint32_t row_bytes) const {
+    p.s += S;
+    p.w += (uint64_t)base * S + (uint64_t)row_bytes * (uint64_t)(nrows * S - T) + Wl;
+  }
+};
+
+// MOD / XOR part of CkPartial::add4 (the Adler part goes through AdlerRows)
+template <uint32_t MASK>
+__device__ __forceinline__ void add4_modxor(CkPartial<MASK>& p, uint32_t x, uint32_t y, uint32_t z, uint32_t v) {
+  if constexpr ((MASK & kMod) != 0) p.mod += (x + y) + (z + v);
+  if constexpr ((MASK & kXor) != 0) p.xr ^= x ^ y ^ z ^ v;
+}
+
 __device__ __forceinline__ float4 ldg_nc_v4(const float* p) {
   float4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
@@ -78,12 +105,15 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       // Listing 7 (L565-578): check-and-recover in the same grid as the original kernel --
       // validate this region from memory (L183), re-execute it only if the check fails.
       CkPartial<MASK> vp;
+      AdlerRows vad;
 #pragma unroll
       for (int r = 0; r < kRowsW; ++r) {
         const uint4 w4 = ld_stream_u4(out + (int64_t)(i0 + r) * ldo + j);
-        const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
-        vp.add4(w4.x, w4.y, w4.z, w4.w, pos);
+        add4_modxor(vp, w4.x, w4.y, w4.z, w4.w);
+        if constexpr ((MASK & kAdler) != 0) vad.add_row(w4.x, w4.y, w4.z, w4.w);
       }
+      if constexpr ((MASK & kAdler) != 0)
+        vad.fold(vp, (uint32_t)(wid * kRowsW * kRN * 4 + lane * 16 + 1), kRowsW, kRN * 4);
       const CkRecord vr = warp_reduce<MASK>(vp);
       if (lane == 0) warp_rec[wid] = vr;
       __syncthreads();
@@ -122,6 +152,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
 #pragma unroll
     for (int r = 0; r < kRowsW; ++r) edge[r] = eok ? ldg_nc_f(in + (int64_t)(i0 + r) * ldi + je) : 0.f;
     CkPartial<MASK> part;
+    AdlerRows ad;
 #pragma unroll
     for (int r = 0; r < kRowsW; ++r) {
       const float4 u = v[r], c = v[r + 1], d = v[r + 2];
@@ -136,10 +167,12 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       o.w = st5(c.w, u.w, d.w, c.z, right);
       __stcs(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
       if constexpr (MASK != 0) {
-        const uint32_t pos = (uint32_t)((wid * kRowsW + r) * kRN * 4 + lane * 16 + 1);
-        part.add4(__float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w), pos);
+        add4_modxor(part, __float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
+        if constexpr ((MASK & kAdler) != 0)
+          ad.add_row(__float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
       }
     }
+    if constexpr ((MASK & kAdler) != 0) ad.fold(part, (uint32_t)(wid * kRowsW * kRN * 4 + lane * 16 + 1), kRowsW, kRN * 4);
     if constexpr (MASK != 0 && COMBINE == 1) {
       // split-barrier combine (one region per CTA): every warp parks its partial in shared memory and
       // ARRIVES on named barrier 2 without waiting; only warp 0 waits (bar.sync) and then combines the
