@@ -72,9 +72,27 @@ __device__ __forceinline__ uint64_t smem_desc(uint32_t saddr, uint32_t lbo, uint
 
 __device__ __forceinline__ void named_bar_epi() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
-// Tile order: groups of 16 M-blocks, M fastest inside a group (L2 reuse of B panels).
+// C tile stores: evict-first (streaming) so the output does not push the A / B panels the next tiles
+// re-read out of L2 (LP_C_STORE_CS=0 builds plain stores for A/B runs)
+#ifndef LP_C_STORE_CS
+#define LP_C_STORE_CS 1
+#endif
+__device__ __forceinline__ void st_c16(uint4* p, uint4 v) {
+#if LP_C_STORE_CS
+  __stcs(p, v);
+#else
+  *p = v;
+#endif
+}
+
+// Tile order: groups of LP_TILE_GROUP M-blocks, M fastest inside a group (L2 reuse of B panels).  8: a
+// wave of 74 CTA-pair tiles spans 8 A panels x ~9 B panels (the smallest footprint; 16 and 4 measured
+// 1.23 / 1.56 GB of DRAM reads per 8192^3 body vs 1.05 GB, profiles/r02/ab_raster.txt).
+#ifndef LP_TILE_GROUP
+#define LP_TILE_GROUP 8
+#endif
 __device__ __forceinline__ void tile_coords(int64_t t, int64_t num_m, int64_t num_n, int64_t& mb, int64_t& nb) {
-  constexpr int64_t G = 16;
+  constexpr int64_t G = LP_TILE_GROUP;
   const int64_t per_group = G * num_n;
   const int64_t g = t / per_group, w = t - g * per_group;
   const int64_t rows = (num_m - g * G) < G ? (num_m - g * G) : G;
@@ -207,7 +225,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
       }
       uint4* dst = reinterpret_cast<uint4*>(crow + ch * 32);
 #pragma unroll
-      for (int i = 0; i < 4; ++i) dst[i] = make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]);
+      for (int i = 0; i < 4; ++i) st_c16(dst + i, make_uint4(w[4 * i], w[4 * i + 1], w[4 * i + 2], w[4 * i + 3]));
       if constexpr (MASK != 0) {
         // byte position of word 0 of this chunk inside its region's stream
         const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((n0 + ch * 32) & 127) * ES + 1)
@@ -237,7 +255,7 @@ __device__ __forceinline__ void epi_store(uint32_t t_row, OutT* __restrict__ C, 
         }
       }
 #pragma unroll
-      for (int i = 0; i < 8; ++i) dst[i] = make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]);
+      for (int i = 0; i < 8; ++i) st_c16(dst + i, make_uint4(r[4 * i], r[4 * i + 1], r[4 * i + 2], r[4 * i + 3]));
       if (!final_pass) continue;
       if constexpr (MASK != 0) {
         const uint32_t pos0 = REG == 128 ? (uint32_t)(row_in_tile * 128 * ES + ((n0 + ch * 32) & 127) * ES + 1)

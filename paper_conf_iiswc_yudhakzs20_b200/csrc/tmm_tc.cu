@@ -75,8 +75,6 @@ __global__ void __launch_bounds__(kThreads, 1)
                   OutT* __restrict__ C, int64_t ldc, int64_t K, TileSrc src, uint32_t* __restrict__ ck) {
   using Cfg = TcCfg<BN>;
   constexpr int S = Cfg::kStages;
-  constexpr int ES = (int)sizeof(OutT);
-  constexpr int NCH = BN / 32;  // 32-column chunks per tile row
 
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
