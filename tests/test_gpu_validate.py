@@ -35,7 +35,7 @@ GEOMS = [
     (16, 1024 * 2, 4, 1024, "bf16"),  # 4 chunks per lane per row
     (2048, 32 * 64, 32, 32, "bf16"),  # many regions: several CTAs, ragged last CTA
     (300 * 7, 128 * 3, 300, 128, "bf16"),  # RM > 256: strip kernel only
-    (1536, 128 * 12, 128, 128, "f32"),     # 64-KiB TMA units, 144 units: one per CTA
+    (1536, 128 * 12, 128, 128, "f32"),     # 144 fp32 128x128 regions (64 KiB each): fewer regions than SMs
     (4096, 32 * 96, 32, 32, "f32"),        # G = 8 units (GC = 64), 1536 units over the SMs
 ]
 
