@@ -16,3 +16,13 @@ $N $F -k regex:tmm_tc_kernel -s 1 -c 1 -o gpurun_out/r02/prof_tmm_tc_recover $B 
 $N $F -k regex:validate_kernel -s 3 -c 1 -o gpurun_out/r02/prof_validate_tmm $B --workload tmm8192_bf16 > gpurun_out/r02/prof_validate_tmm.log 2>&1
 $N $F -k regex:tmm_tf32x3_kernel -s 2 -c 1 -o gpurun_out/r02/prof_tmm_tf32 $B --workload tmm8192_f32 > gpurun_out/r02/prof_tmm_tf32.log 2>&1
 ls -la gpurun_out/r02
+# keep the copy-back small (gpurun merges <= 64 MiB): export every capture to CSV (+ the top SASS lines) and drop
+# the .ncu-rep files
+for r in gpurun_out/r02/*.ncu-rep; do
+  b=${r%.ncu-rep}
+  ncu -i $r --page raw --csv > $b.raw.csv 2>/dev/null
+  ncu -i $r --page details --csv > $b.details.csv 2>/dev/null
+  python tools/ncu_sass_top.py $r 30 > $b.sass_top.txt 2>&1
+  rm -f $r
+done
+du -sh gpurun_out
