@@ -91,6 +91,14 @@ __device__ __forceinline__ void st_c16(uint4* p, uint4 v) {
 #ifndef LP_TILE_GROUP
 #define LP_TILE_GROUP 8
 #endif
+__device__ __forceinline__ void tile_coords_g(int64_t t, int64_t num_m, int64_t num_n, int64_t G, int64_t& mb,
+                                              int64_t& nb) {
+  const int64_t per_group = G * num_n;
+  const int64_t g = t / per_group, w = t - g * per_group;
+  const int64_t rows = (num_m - g * G) < G ? (num_m - g * G) : G;
+  mb = g * G + w % rows;
+  nb = w / rows;
+}
 __device__ __forceinline__ void tile_coords(int64_t t, int64_t num_m, int64_t num_n, int64_t& mb, int64_t& nb) {
   constexpr int64_t G = LP_TILE_GROUP;
   const int64_t per_group = G * num_n;

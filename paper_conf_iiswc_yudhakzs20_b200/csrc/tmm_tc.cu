@@ -580,6 +580,167 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   }
 }
 
+// ---------------------------------------------------------------------------- 256-row CTA-pair kernel
+// Full runs with M % 512 == 0 and N % 256 == 0: each CTA of the pair owns a 256-row band of a 512x256
+// pair tile.  Per k-step the leader issues TWO tcgen05.mma.cta_group::2 256x256x16 (pair rows = CTA rows
+// [0,128) and [128,256)), into accumulators D0 / D1 that together fill the whole TMEM (512 fp32 columns).
+// A is staged as one 256-row TMA box (32 KiB per k-block), B as this CTA's 128 columns (16 KiB): 48 KiB per
+// 256x256x64 MACs per SM instead of 32 KiB per 128x256x64 -- 25% fewer L2 -> SM bytes per flop (the
+// cuBLAS sm_100 kernel's tile shape; C5 runs power-capped, where moved bytes cost clock).  The accumulators
+// cannot be double-buffered, so the epilogue drains D0 first: the next tile's D0 MMAs start while D1 drains.
+constexpr int kStages4 = 4;
+constexpr int kA4Bytes = 256 * kBK * 2;   // 32 KiB: this CTA's 256 rows of A
+constexpr int kB4Bytes = kBK * 128 * 2;   // 16 KiB: this CTA's 128 columns of B
+constexpr int kStage4Bytes = kA4Bytes + kB4Bytes;
+constexpr int kSmem4Bytes = kStages4 * kStage4Bytes + 1024 + 1024;
+
+template <typename OutT, uint32_t MASK, int REG, int STORE>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+    tmm_tc4_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
+                   OutT* __restrict__ C, int64_t ldc, int64_t K, int64_t num_m, int64_t num_n, int64_t group,
+                   int64_t Qr, int64_t rid_offset, uint32_t* __restrict__ ck) {
+  constexpr int BN = 256;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + kStages4 * kA4Bytes;
+  uint64_t* full = (uint64_t*)(smem + kStages4 * kStage4Bytes);
+  uint64_t* empty = full + kStages4;
+  uint64_t* tfull = empty + kStages4;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_holder = (uint32_t*)(tempty + 2);
+  CkRecord* srec = (CkRecord*)(tmem_holder + 4);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = cluster_ctarank();
+  const int64_t pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&tmap_a);
+    prefetch_tmap(&tmap_b);
+    for (int s = 0; s < kStages4; ++s) {
+      mbar_init(&full[s], 2);
+      mbar_init(&empty[s], 1);
+    }
+    for (int s = 0; s < 2; ++s) {
+      mbar_init(&tfull[s], 1);
+      mbar_init(&tempty[s], 8);  // 4 epilogue warps x 2 CTAs, used in rank 0
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_holder)),
+                 "r"(512u)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  cluster_sync_all();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_holder;
+  const int64_t ntiles = num_m * num_n;
+  const int nkb = (int)(K / kBK);
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int64_t t = pair; t < ntiles; t += npairs) {
+        int64_t mb, nb;
+        tile_coords_g(t, num_m, num_n, group, mb, nb);
+        const int m0 = (int)(mb * 512 + rank * 256), n0 = (int)(nb * 256 + rank * 128);
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&empty[stage], phase ^ 1);
+          const uint32_t full0 = mapa_rank0(&full[stage]);
+          if (rank == 0)
+            mbar_expect_tx(&full[stage], 2 * kStage4Bytes);
+          else
+            mbar_arrive_remote(full0);
+          tma_load_2d_pair(&tmap_a, full0, sA + stage * kA4Bytes, kb * kBK, m0);
+          tma_load_2d_pair(&tmap_b, full0, sB + stage * kB4Bytes, n0, kb * kBK);
+          tma_load_2d_pair(&tmap_b, full0, sB + stage * kB4Bytes + kBK * 128, n0 + 64, kb * kBK);
+          if (++stage == kStages4) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {
+      constexpr uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | (0u << 15) | (1u << 16) |
+                                 ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
+      int stage = 0;
+      uint32_t phase = 0;
+      uint32_t acc_phase = 0;
+      for (int64_t t = pair; t < ntiles; t += npairs) {
+        mbar_wait(&tempty[0], acc_phase ^ 1);  // D0 drained by the previous tile's epilogue
+        tc_fence_after();
+        for (int kb = 0; kb < nkb; ++kb) {
+          mbar_wait(&full[stage], phase);
+          tc_fence_after();
+          const uint32_t a_addr = smem_u32(sA + stage * kA4Bytes);
+          const uint32_t b_addr = smem_u32(sB + stage * kB4Bytes);
+#pragma unroll
+          for (int k = 0; k < kBK / kUmmaK; ++k) {
+            const uint64_t bd = smem_desc(b_addr + k * kUmmaK * 128, kBK * 128, 1024);
+            tc_mma_pair(tmem_base, smem_desc(a_addr + k * kUmmaK * 2, 16, 1024), bd, idesc, (kb | k) ? 1u : 0u);
+            if (kb == 0 && k == 0) {
+              mbar_wait(&tempty[1], acc_phase ^ 1);  // D1 drained (overlaps the D0 MMAs above)
+              tc_fence_after();
+            }
+            tc_mma_pair(tmem_base + 256u, smem_desc(a_addr + 128 * 128 + k * kUmmaK * 2, 16, 1024), bd, idesc,
+                        (kb | k) ? 1u : 0u);
+          }
+          tc_commit_pair(&empty[stage]);
+          if (++stage == kStages4) {
+            stage = 0;
+            phase ^= 1;
+          }
+        }
+        tc_commit_pair(&tfull[0]);
+        tc_commit_pair(&tfull[1]);
+        acc_phase ^= 1;
+      }
+    }
+  } else {
+    const int wq = warp & 3;
+    uint32_t acc_phase = 0;
+    for (int64_t t = pair; t < ntiles; t += npairs) {
+      int64_t mb, nb;
+      tile_coords_g(t, num_m, num_n, group, mb, nb);
+#pragma unroll 1
+      for (int d = 0; d < 2; ++d) {
+        mbar_wait(&tfull[d], acc_phase);
+        tc_fence_after();
+        const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(d * BN);
+        CkRecord* srec_d = srec + d * 2 * 4;
+        const int64_t m128 = mb * 4 + rank * 2 + d;
+        epi_store<OutT, MASK, REG, BN, STORE>(t_row, C, ldc, m128, nb * BN, wq, lane, srec_d, ck, Qr, rid_offset);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (rank == 0)
+            mbar_arrive(&tempty[d]);
+          else
+            mbar_arrive_remote(mapa_rank0(&tempty[d]));
+        }
+        if constexpr (MASK != 0 && REG == 128)
+          epi_finish_128<OutT, MASK, BN, STORE>(warp, lane, srec_d, ck, m128, nb * BN, Qr, rid_offset);
+      }
+      acc_phase ^= 1;
+    }
+  }
+
+  tc_fence_before();
+  __syncthreads();
+  cluster_sync_all();
+  tc_fence_after();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "r"(512u) : "memory");
+  }
+}
+
 // ---------------------------------------------------------------------------- host side
 bool make_map_2d(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld_elems,
                  uint32_t box_inner, uint32_t box_outer) {
@@ -722,6 +883,69 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
   return cudaGetLastError();
 }
 
+// LP_TC_TILE=128 forces the 128-row-per-CTA pair kernel for shapes the 256-row one takes (A/B runs);
+// LP_TC4_GROUP=<n> sets its raster group (M-blocks of 512 rows per group)
+int tc4_mode() {
+  static int v = [] {
+    const char* e = getenv("LP_TC_TILE");
+    return (e && atoi(e) == 128) ? 0 : 1;
+  }();
+  return v;
+}
+int64_t tc4_group() {
+  static int64_t v = [] {
+    const char* e = getenv("LP_TC4_GROUP");
+    return e ? (int64_t)atoi(e) : (int64_t)4;
+  }();
+  return v < 1 ? 1 : v;
+}
+
+template <typename OutT, int REG>
+cudaError_t launch_pair4(const TmmArgs& a, cudaStream_t st, const char** why) {
+  CUtensorMap ma, mb;
+  if (!make_map_2d(&ma, a.A, (uint64_t)a.K, (uint64_t)a.M, (uint64_t)a.lda, kBK, 256) ||
+      !make_map_2d(&mb, a.B, (uint64_t)a.N, (uint64_t)a.K, (uint64_t)a.ldb, 64, kBK)) {
+    *why = "cuTensorMapEncodeTiled failed";
+    return cudaErrorInvalidValue;
+  }
+  const int64_t num_m = a.M / 512, num_n = a.N / 256;
+  int64_t grid = 2 * num_m * num_n;
+  const int64_t cap = a.sm_count & ~1;
+  if (grid > cap) grid = cap;
+  if (grid < 2) grid = 2;
+  const int64_t Qr = a.N / REG;
+  const int sk = a.mask ? a.hash.store : 0;
+  const int64_t G = tc4_group();
+  cudaError_t e = cudaSuccess;
+  switch (a.mask * 5 + sk) {
+#define LP_TC4_CASE(M, S)                                                                                   \
+  case M * 5 + S: {                                                                                         \
+    auto kfn = tmm_tc4_kernel<OutT, M, REG, S>;                                                            \
+    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem4Bytes);                \
+    if (e != cudaSuccess) return e;                                                                         \
+    kfn<<<(unsigned)grid, kThreads, kSmem4Bytes, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, G, Qr, \
+                                                       a.rid_offset, a.ck);                                 \
+    break;                                                                                                  \
+  }
+#define LP_TC4_CASE3(M) LP_TC4_CASE(M, 0)
+#define LP_TC4_CASE5(M) LP_TC4_CASE(M, 0) LP_TC4_CASE(M, 1) LP_TC4_CASE(M, 2) LP_TC4_CASE(M, 3) LP_TC4_CASE(M, 4)
+    LP_TC4_CASE(0, 0)
+    LP_TC4_CASE5(1)
+    LP_TC4_CASE3(2)
+    LP_TC4_CASE5(3)
+    LP_TC4_CASE3(4)
+    LP_TC4_CASE3(5)
+    LP_TC4_CASE3(6)
+    LP_TC4_CASE3(7)
+#undef LP_TC4_CASE3
+#undef LP_TC4_CASE5
+#undef LP_TC4_CASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
 template <typename OutT, int REG>
 cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why) {
   CUtensorMap ma, mb;
@@ -774,6 +998,8 @@ cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, cudaStream_t st,
 
 template <typename OutT, int REG>
 cudaError_t launch_reg(const TmmArgs& a, cudaStream_t st, const char** why) {
+  if (!a.list && a.M % 512 == 0 && a.N % 256 == 0 && !a.force_1cta && tc4_mode())
+    return launch_pair4<OutT, REG>(a, st, why);
   if (!a.list && a.M % 256 == 0 && a.N % 256 == 0 && !a.force_1cta) return launch_pair<OutT, REG>(a, st, why);
   // list mode re-executes 128x128 tiles (BN = 128): one 128x128 region, or the
   // 16 32x32 regions of a de-duplicated tile; paired tasks (two such tiles of one

@@ -22,19 +22,20 @@ def cycle(h, wl, out, ck, failed, d_n, ws, stale, frac=0.2):
     assert int(d_n.item()) == 0
 
 
-def tmm(M, N, K, reg, in_dt, out_dt, body, store="array", shuffle=True):
+def tmm(M, N, K, reg, in_dt, out_dt, body, store="array", shuffle=True, **flags):
     tdt = {"bf16": torch.bfloat16, "f32": torch.float32, "i32": torch.int32}[in_dt]
     a = torch.empty((M, K), dtype=tdt, device="cuda")
     b = torch.empty((K, N), dtype=tdt, device="cuda")
     kind = "int5"
     lpsynth.device_fill(a, 1, kind, in_dt)
     lpsynth.device_fill(b, 2, kind, in_dt)
-    h = lp.LP(reg, reg, cksum="mod|xor", store=store, body=body, shuffle=shuffle)
+    h = lp.LP(reg, reg, cksum="mod|xor", store=store, body=body, shuffle=shuffle, **flags)
     wl = lp.Workload.tmm(a, b, out_dtype=out_dt)
     out, ck, failed, d_n, ws = h.alloc(wl)
     stale = torch.zeros_like(out)
     cycle(h, wl, out, ck, failed, d_n, ws, stale)
-    print("ok", M, N, K, reg, in_dt, out_dt, body, store, shuffle, flush=True)
+    print("ok", M, N, K, reg, in_dt, out_dt, body, store, shuffle, flags, flush=True)
+    return h, wl, out, ck, stale
 
 
 def stencil(store="array"):
@@ -90,3 +91,23 @@ stencil("quad_cas")
 tmm(256, 512, 1024, 128, "f32", "f32", "tcgen05")     # 3xTF32: two 512-K chunks through the TMEM running sum
 spmv()
 validate_large_table()
+
+
+# round 2: Listing 7 on the TMM (check phase + DSMEM bitmask merge), cuckoo stash + device rehash,
+# 128x128 regions recovered as slices with cross-task record combine, NVLS count (single-GPU emulation)
+h, wl, out, ck, stale = tmm(512, 768, 128, 128, "bf16", "bf16", "tcgen05")
+inj = torch.from_numpy(lp.choose_regions(h.num_regions(wl), 0.3, 9)).cuda()
+h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=9)
+d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
+h.check_recover(wl, out, ck, d_rec)
+torch.cuda.synchronize()
+print("ok tmm check_recover", int(d_rec.item()), flush=True)
+tmm(1024, 1024, 64, 32, "bf16", "bf16", "tcgen05", store="cuckoo", cuckoo_short_chains=True)
+tmm(512, 1024, 128, 128, "bf16", "bf16", "tcgen05", recover_slices128=True)
+h2, wl2, out2, ck2, stale2 = tmm(512, 512, 64, 128, "bf16", "bf16", "tcgen05", nvls_count=True)
+cnt = torch.zeros(16, dtype=torch.int64, device="cuda")
+h2.attach_nvls_count(cnt, cnt, 1)
+_, _, failed2, d_n2, ws2 = h2.alloc(wl2)
+h2.validate(wl2, out2, ck2, failed2, d_n2, ws2)
+torch.cuda.synchronize()
+print("ok nvls emulation", int(cnt[3].item()), flush=True)
