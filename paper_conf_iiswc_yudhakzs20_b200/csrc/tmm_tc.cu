@@ -895,7 +895,7 @@ int tc4_mode() {
 int64_t tc4_group() {
   static int64_t v = [] {
     const char* e = getenv("LP_TC4_GROUP");
-    return e ? (int64_t)atoi(e) : (int64_t)4;
+    return e ? (int64_t)atoi(e) : (int64_t)2;
   }();
   return v < 1 ? 1 : v;
 }

@@ -420,3 +420,38 @@ def test_tc_recovery_slices128(frac, out_dt, store):
     _, nf = run_cycle(2048, 2560, 256, 128, 128, "bf16", out_dt, "uniform", "mod|xor|adler" if store == "array"
                       else "mod|xor", "tcgen05", mode="stale_words", frac=frac, store=store, recover_slices128=True)
     assert nf > 0
+
+
+@pytest.mark.parametrize("reg", [128, 32])
+@pytest.mark.parametrize("out_dt", ["bf16", "f32"])
+@pytest.mark.parametrize("kind", ["int5", "uniform"])
+def test_tc4_256row_pair_kernel(reg, out_dt, kind):
+    """M % 512 == 0: the CTA-pair kernel with 256 rows per CTA (two M = 256 MMAs per k-step into the whole TMEM);
+    values, records, validate and recovery against the oracle (N = 768: 3 column tiles, 2 x 3 pair tiles)."""
+    run_cycle(1024, 768, 256, reg, reg, "bf16", out_dt, kind, "mod|xor|adler", "tcgen05", mode="stale_words",
+              frac=0.2)
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "cuckoo"])
+def test_tc4_hash_stores(store):
+    run_cycle(1024, 1024, 128, 128, 128, "bf16", "bf16", "int5", "mod|xor", "tcgen05", store=store, frac=0.1)
+
+
+def test_tc4_matches_tc2_bits():
+    """The 256-row pair kernel (M = 1024) and the 128-row pair kernel (the same rows as M = 768 + M = 256
+    problems, which it cannot take) produce identical bits: the same K order per output element."""
+    from lpsynth import device_fill
+    a = torch.empty((1024, 512), dtype=torch.bfloat16, device="cuda")
+    b = torch.empty((512, 768), dtype=torch.bfloat16, device="cuda")
+    device_fill(a, 1, "uniform", "bf16")
+    device_fill(b, 2, "uniform", "bf16")
+    outs = []
+    for rows in ((0, 1024), (0, 768), (768, 1024)):
+        h = lp.LP(128, 128, cksum="mod|xor")
+        wl = lp.Workload.tmm(a[rows[0]:rows[1]], b, out_dtype="f32")
+        out, ck, failed, d_n, ws = h.alloc(wl)
+        h.cksum_init(wl, ck)
+        h.run_protected(wl, out, ck)
+        outs.append(out)
+    torch.cuda.synchronize()
+    assert torch.equal(outs[0].view(torch.int32), torch.cat([outs[1], outs[2]]).view(torch.int32))
