@@ -260,6 +260,15 @@ LP_API lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* ou
 LP_API lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
                                   int64_t* d_n_recovered, lp_stream_t stream);
 
+/* lp_check_recover with a workspace (lp_workspace_bytes bytes; NULL = the static form above).  TMM: the
+ * balanced form -- a cooperative launch (at most the co-resident CTA pairs) whose CTAs publish their
+ * failed tiles to a global bitmask in the workspace and pass a grid barrier after the check phase; the
+ * j-th failed tile then goes to pair j % npairs, so the recompute spreads over every pair instead of
+ * staying on the pairs that own the failed tiles.  Same final state and count.  STENCIL5: as
+ * lp_check_recover. */
+LP_API lp_status lp_check_recover_ws(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
+                                     int64_t* d_n_recovered, void* workspace, lp_stream_t stream);
+
 /* NVLS-fused failed-count all-reduce (needs cfg.flags & LP_FLAG_NVLS_COUNT).
  * mc_counter = the multicast (NVLS) address and uc_counter = this rank's unicast address of the same
  * 64-byte-aligned, >= 64-byte counter buffer, bound to a multicast object on every one of the

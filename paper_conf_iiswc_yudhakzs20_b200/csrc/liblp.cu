@@ -196,8 +196,8 @@ int64_t dedupe_capacity(const lp::RegionGeom& g) {
 }
 
 struct WsLayout {
-  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, tasks_tmp, d_ntasks, part, cnt, ticket,
-      total;
+  size_t flags, counts, tile_flags, tile_counts, tile_list, d_ntiles, tasks, tasks_tmp, d_ntasks, part, cnt, gbits,
+      gbar, ticket, total;
 };
 
 WsLayout ws_layout(const lp::RegionGeom& g) {
@@ -221,7 +221,9 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   const size_t npart = g.RM == 128 ? (size_t)g.R : 0;
   w.part = w.d_ntasks + 256;
   w.cnt = w.part + al(npart * 32);
-  w.ticket = w.cnt + al(npart * 4);                 // fused-compaction ticket (u32; zero-initialised, kept at 0)
+  w.gbits = w.cnt + al(npart * 4);                  // balanced check-and-recover: global failed-tile bitmask
+  w.gbar = w.gbits + al((size_t)(g.R + 31) / 32 * 4);  //   and its grid-barrier counter (cleared per call)
+  w.ticket = w.gbar + 256;                          // fused-compaction ticket (u32; zero-initialised, kept at 0)
   w.total = w.ticket + 256;
   return w;
 }
@@ -570,6 +572,11 @@ lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void
 
 lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, int64_t* d_n_recovered,
                            lp_stream_t stream) {
+  return lp_check_recover_ws(h, wl, out, cksum, d_n_recovered, nullptr, stream);
+}
+
+lp_status lp_check_recover_ws(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, int64_t* d_n_recovered,
+                              void* workspace, lp_stream_t stream) {
   lp::RegionGeom g;
   lp_status s = check_wl(h, wl, &g);
   if (s) return s;
@@ -591,7 +598,11 @@ lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void
     DeviceGuard dg(h->cfg.device);
     const lp::TmmArgs a = tmm_args(h, wl, g, out, cksum, nullptr, nullptr);
     const char* why = nullptr;
-    cudaError_t e = lp::launch_tmm_tc_check_recover(a, d_n_recovered, (cudaStream_t)stream, &why);
+    if (workspace && !aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
+    const WsLayout w = ws_layout(g);
+    uint32_t* gbits = workspace ? (uint32_t*)((uint8_t*)workspace + w.gbits) : nullptr;
+    uint32_t* gbar = workspace ? (uint32_t*)((uint8_t*)workspace + w.gbar) : nullptr;
+    cudaError_t e = lp::launch_tmm_tc_check_recover(a, d_n_recovered, gbits, gbar, (cudaStream_t)stream, &why);
     if (e != cudaSuccess) return why ? fail(LP_ERR_UNSUPPORTED, "check-and-recover: %s", why) : cuda_fail(e, "check-and-recover launch");
     if ((s = cuckoo_rehash(h, cksum, (cudaStream_t)stream))) return s;
     return ok();

@@ -104,7 +104,10 @@ cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why);
 // its halves of its pair's tiles, then recomputes in place only the tiles with a failed region;
 // *d_rec (zeroed here) counts the failed regions.
 bool tmm_tc_check_supported(int64_t M, int64_t N);
-cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why);
+// gbits / gbar (workspace, may be null): balanced form -- a cooperative launch whose CTAs publish their failed
+// tiles to a global bitmask, pass a grid barrier and deal the failed tiles round robin over all pairs.
+cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, uint32_t* gbits, uint32_t* gbar,
+                                        cudaStream_t st, const char** why);
 
 // ---- tmm_tf32.cu : fp32 in/out via 3xTF32 on tcgen05 (CTA pair)
 bool tmm_tf32_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf16, int out_bf16, int64_t lda,

@@ -410,11 +410,56 @@ __device__ __forceinline__ void check_tiles(const OutT* __restrict__ C, int64_t 
   }
 }
 
-template <typename OutT, uint32_t MASK, int REG, int STORE, bool CHECK = false>
+// Tile walk of a CTA pair.  CHECK 0: the persistent schedule t = pair, pair + npairs, ...; 1 (Listing 7,
+// static): the same schedule, skipping tiles whose bit is clear in the pair's merged bitmask `todo`;
+// 2 (Listing 7, balanced): the j-th failed tile of the GLOBAL bitmask (ascending tile index) goes to pair
+// j % npairs -- every role of both CTAs derives the same sequence from the bitmask, no broadcast needed.
+template <int CHECK>
+struct TileWalk {
+  int64_t t, lt, pair, npairs, ntiles;
+  const uint32_t* todo;   // CHECK 1: shared bitmask over local indices
+  const uint32_t* gbits;  // CHECK 2: global bitmask over tile ids
+  int64_t w, nwords, j;
+  uint32_t cur;
+  __device__ __forceinline__ TileWalk(int64_t pair_, int64_t npairs_, int64_t ntiles_, const uint32_t* todo_,
+                                      const uint32_t* gbits_)
+      : t(pair_ - npairs_), lt(-1), pair(pair_), npairs(npairs_), ntiles(ntiles_), todo(todo_), gbits(gbits_), w(-1),
+        nwords((ntiles_ + 31) >> 5), j(0), cur(0u) {}
+  __device__ __forceinline__ bool next(int64_t& out) {
+    if constexpr (CHECK == 2) {
+      for (;;) {
+        while (cur == 0u) {
+          if (++w >= nwords) return false;
+          cur = __ldcg(gbits + w);
+        }
+        const int b = __ffs(cur) - 1;
+        cur &= cur - 1u;
+        const bool mine = (j % npairs) == pair;
+        ++j;
+        if (mine) {
+          out = w * 32 + b;
+          return true;
+        }
+      }
+    } else {
+      for (;;) {
+        t += npairs;
+        ++lt;
+        if (t >= ntiles) return false;
+        if (CHECK == 1 && !((todo[lt >> 5] >> (lt & 31)) & 1u)) continue;
+        out = t;
+        return true;
+      }
+    }
+  }
+};
+
+template <typename OutT, uint32_t MASK, int REG, int STORE, int CHECK = 0>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     tmm_tc2_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
                    OutT* __restrict__ C, int64_t ldc, int64_t K, int64_t num_m, int64_t num_n, int64_t Qr,
-                   int64_t rid_offset, uint32_t* __restrict__ ck, int64_t* __restrict__ d_rec) {
+                   int64_t rid_offset, uint32_t* __restrict__ ck, int64_t* __restrict__ d_rec,
+                   uint32_t* __restrict__ gbits, uint32_t* __restrict__ gbar) {
   constexpr int BN = 256;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -461,27 +506,53 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   const int64_t nloc = (ntiles - pair + npairs - 1) / npairs;
   const int nwords = (int)((nloc + 31) >> 5);
   uint32_t* s_todo = s_fail + nwords;
-  if constexpr (CHECK) {
+  if constexpr (CHECK != 0) {
     for (int i = threadIdx.x; i < nwords; i += kThreads) s_fail[i] = 0u;
     __syncthreads();
     check_tiles<OutT, MASK, REG, STORE>(C, ldc, ck, ntiles, pair, npairs, num_m, num_n, Qr, rid_offset, rank, s_fail,
                                         d_rec);
-    cluster_sync_all();  // both halves checked; the peer's bitmask is final
-    uint32_t peer;
-    for (int i = threadIdx.x; i < nwords; i += kThreads) {
-      asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(peer) : "r"(mapa_peer(&s_fail[i], rank ^ 1u)) : "memory");
-      s_todo[i] = s_fail[i] | peer;
+    if constexpr (CHECK == 1) {
+      cluster_sync_all();  // both halves checked; the peer's bitmask is final
+      uint32_t peer;
+      for (int i = threadIdx.x; i < nwords; i += kThreads) {
+        asm volatile("ld.shared::cluster.u32 %0, [%1];" : "=r"(peer) : "r"(mapa_peer(&s_fail[i], rank ^ 1u)) : "memory");
+        s_todo[i] = s_fail[i] | peer;
+      }
+      __syncthreads();
+    } else {
+      // publish this CTA's failed tiles to the global bitmask, then a grid barrier (cooperative launch:
+      // every CTA is resident); afterwards every pair reads the same global bitmask
+      __syncthreads();
+      for (int i = threadIdx.x; i < nwords; i += kThreads) {
+        uint32_t m = s_fail[i];
+        while (m) {
+          const int64_t lt = (int64_t)i * 32 + (__ffs(m) - 1);
+          m &= m - 1u;
+          const int64_t t = pair + lt * npairs;
+          atomicOr(gbits + (t >> 5), 1u << (t & 31));
+        }
+      }
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(gbar, 1u);
+        uint32_t v;
+        do {
+          __nanosleep(64);
+          asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(gbar) : "memory");
+        } while (v < gridDim.x);
+      }
+      __syncthreads();
     }
-    __syncthreads();
   }
-  auto skip = [&](int64_t lt) -> bool { return CHECK && !((s_todo[lt >> 5] >> (lt & 31)) & 1u); };
 
   if (warp == 0) {
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
-        if (skip(lt)) continue;
+      TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
+      int64_t t;
+      while (walk.next(t)) {
         int64_t mb, nb;
         tile_coords(t, num_m, num_n, mb, nb);
         const int m0 = (int)(mb * 256 + rank * 128), n0 = (int)(nb * 256 + rank * 128);
@@ -511,8 +582,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
-        if (skip(lt)) continue;
+      TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
+      int64_t t;
+      while (walk.next(t)) {
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -544,8 +616,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     const int wq = warp & 3;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int64_t t = pair, lt = 0; t < ntiles; t += npairs, ++lt) {
-      if (skip(lt)) continue;
+    TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
+    int64_t t;
+    while (walk.next(t)) {
       int64_t mb, nb;
       tile_coords(t, num_m, num_n, mb, nb);
       mbar_wait(&tfull[acc], acc_phase);
@@ -861,7 +934,7 @@ cudaError_t launch_pair(const TmmArgs& a, cudaStream_t st, const char** why) {
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2Bytes);                \
     if (e != cudaSuccess) return e;                                                                         \
     kfn<<<(unsigned)grid, kThreads, kSmem2Bytes, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr,    \
-                                                       a.rid_offset, a.ck, nullptr);                        \
+                                                       a.rid_offset, a.ck, nullptr, nullptr, nullptr);     \
     break;                                                                                                  \
   }
 #define LP_TC2_CASE3(M) LP_TC2_CASE(M, 0)
@@ -946,8 +1019,24 @@ cudaError_t launch_pair4(const TmmArgs& a, cudaStream_t st, const char** why) {
   return cudaGetLastError();
 }
 
+template <typename Kern, typename... Args>
+cudaError_t launch_cooperative(Kern kfn, unsigned grid, int smem, cudaStream_t st, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeCooperative;
+  attr[0].val.cooperative = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kfn, args...);
+}
+
 template <typename OutT, int REG>
-cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why) {
+cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, uint32_t* gbits, uint32_t* gbar, cudaStream_t st,
+                              const char** why) {
   CUtensorMap ma, mb;
   if (!make_map_2d(&ma, a.A, (uint64_t)a.K, (uint64_t)a.M, (uint64_t)a.lda, kBK, kBM) ||
       !make_map_2d(&mb, a.B, (uint64_t)a.N, (uint64_t)a.K, (uint64_t)a.ldb, 64, kBK)) {
@@ -959,23 +1048,49 @@ cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, cudaStream_t st,
   const int64_t cap = a.sm_count & ~1;
   if (grid > cap) grid = cap;
   if (grid < 2) grid = 2;
-  const int64_t nloc = (num_m * num_n + grid / 2 - 1) / (grid / 2);
-  const int smem = kSmem2Bytes + (int)(2 * ((nloc + 31) / 32) * 4);
-  if (smem > 227 * 1024) {
-    *why = "too many tiles per CTA pair for the check-and-recover bitmask";
-    return cudaErrorInvalidValue;
-  }
   const int64_t Qr = a.N / REG;
   cudaError_t e = cudaMemsetAsync(d_rec, 0, sizeof(int64_t), st);
   if (e != cudaSuccess) return e;
+  const bool balanced = gbits != nullptr && gbar != nullptr;
+  if (balanced) {  // grid barrier counter + global failed-tile bitmask, cleared in stream order
+    e = cudaMemsetAsync(gbar, 0, sizeof(uint32_t), st);
+    if (e == cudaSuccess) e = cudaMemsetAsync(gbits, 0, (size_t)((num_m * num_n + 31) / 32) * 4, st);
+    if (e != cudaSuccess) return e;
+  }
+  auto smem_for = [&](int64_t g) { return kSmem2Bytes + (int)(2 * (((num_m * num_n + g / 2 - 1) / (g / 2)) + 31) / 32 * 4); };
   switch (a.mask * 5 + a.hash.store) {
 #define LP_TC2C_CASE(M, S)                                                                                  \
   case M * 5 + S: {                                                                                         \
-    auto kfn = tmm_tc2_kernel<OutT, M, REG, S, true>;                                                      \
-    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                       \
+    if (balanced) {                                                                                         \
+      auto kfn = tmm_tc2_kernel<OutT, M, REG, S, 2>;                                                       \
+      /* every CTA must be resident for the grid barrier: at most the co-resident clusters */              \
+      int ncl = 0;                                                                                          \
+      e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_for(2));             \
+      if (e != cudaSuccess) return e;                                                                       \
+      cudaLaunchConfig_t oc = {};                                                                           \
+      oc.gridDim = dim3((unsigned)grid);                                                                    \
+      oc.blockDim = dim3(kThreads);                                                                         \
+      oc.dynamicSmemBytes = (size_t)smem_for(2);                                                            \
+      e = cudaOccupancyMaxActiveClusters(&ncl, kfn, &oc);                                                   \
+      if (e != cudaSuccess) return e;                                                                       \
+      const int64_t g2 = (2 * (int64_t)ncl < grid) ? 2 * (int64_t)ncl : grid;                               \
+      if (g2 < 2) { *why = "no co-resident CTA pair"; return cudaErrorInvalidValue; }                      \
+      const int sm2 = smem_for(g2);                                                                         \
+      if (sm2 > 227 * 1024) { *why = "too many tiles per CTA pair for the bitmask"; return cudaErrorInvalidValue; } \
+      e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, sm2);                      \
+      if (e != cudaSuccess) return e;                                                                       \
+      e = launch_cooperative(kfn, (unsigned)g2, sm2, st, ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr,  \
+                             a.rid_offset, a.ck, d_rec, gbits, gbar);                                       \
+    } else {                                                                                                \
+      const int sm1 = smem_for(grid);                                                                       \
+      if (sm1 > 227 * 1024) { *why = "too many tiles per CTA pair for the bitmask"; return cudaErrorInvalidValue; } \
+      auto kfn = tmm_tc2_kernel<OutT, M, REG, S, 1>;                                                       \
+      e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, sm1);                      \
+      if (e != cudaSuccess) return e;                                                                       \
+      kfn<<<(unsigned)grid, kThreads, sm1, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr,          \
+                                                 a.rid_offset, a.ck, d_rec, nullptr, nullptr);              \
+    }                                                                                                       \
     if (e != cudaSuccess) return e;                                                                         \
-    kfn<<<(unsigned)grid, kThreads, smem, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, Qr, a.rid_offset, \
-                                                a.ck, d_rec);                                               \
     break;                                                                                                  \
   }
 #define LP_TC2C_CASE3(M) LP_TC2C_CASE(M, 0)
@@ -1024,13 +1139,14 @@ bool tmm_tc_supported(int64_t M, int64_t N, int64_t K, int RM, int RN, int in_bf
 
 bool tmm_tc_check_supported(int64_t M, int64_t N) { return M % 256 == 0 && N % 256 == 0; }
 
-cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, cudaStream_t st, const char** why) {
+cudaError_t launch_tmm_tc_check_recover(const TmmArgs& a, int64_t* d_rec, uint32_t* gbits, uint32_t* gbar,
+                                        cudaStream_t st, const char** why) {
   if (a.mask == 0 || a.list || !tmm_tc_check_supported(a.M, a.N)) return cudaErrorInvalidValue;
   if (a.RM == 128)
-    return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 128>(a, d_rec, st, why)
-                      : launch_pair_check<float, 128>(a, d_rec, st, why);
-  return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 32>(a, d_rec, st, why)
-                    : launch_pair_check<float, 32>(a, d_rec, st, why);
+    return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 128>(a, d_rec, gbits, gbar, st, why)
+                      : launch_pair_check<float, 128>(a, d_rec, gbits, gbar, st, why);
+  return a.out_bf16 ? launch_pair_check<__nv_bfloat16, 32>(a, d_rec, gbits, gbar, st, why)
+                    : launch_pair_check<float, 32>(a, d_rec, gbits, gbar, st, why);
 }
 
 cudaError_t launch_tmm_tc(const TmmArgs& a, cudaStream_t st, const char** why) {

@@ -43,7 +43,7 @@ INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",
             "lp_run_protected", "lp_validate", "lp_recover", "lp_region_checksums", "lp_inject", "lp_stats",
             "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study", "lp_check_recover",
-            "lp_attach_nvls_count", "lp_recover_count"]
+            "lp_attach_nvls_count", "lp_recover_count", "lp_check_recover_ws"]
 
 
 def parse_cksum(spec) -> int:
@@ -109,6 +109,7 @@ def lib():
             "lp_stats": [P, pw, P, P, P],
             "lp_fn_study": [P, U32, ctypes.c_int32, I64, U64, I64, P, P, I64, P],
             "lp_check_recover": [P, pw, P, P, P, P],
+            "lp_check_recover_ws": [P, pw, P, P, P, P, P],
             "lp_attach_nvls_count": [P, P, P, ctypes.c_int32],
         }
         for name, args in sig.items():
@@ -297,10 +298,15 @@ class LP:
             _check(lib().lp_recover_count(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed),
                                           _ptr(d_n), _ptr(workspace), _ptr(d_n_recovered), _stream(stream)))
 
-    def check_recover(self, wl, out, ck, d_n_recovered, stream=None):
-        """Listing 7's same-grid check-and-recover (N2): validate + in-place re-execution in one kernel."""
-        _check(lib().lp_check_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(d_n_recovered),
-                                      _stream(stream)))
+    def check_recover(self, wl, out, ck, d_n_recovered, workspace=None, stream=None):
+        """Listing 7's same-grid check-and-recover (N2): validate + in-place re-execution in one kernel; with a
+        workspace the TMM form deals the failed tiles over all CTA pairs (lp_check_recover_ws)."""
+        if workspace is None:
+            _check(lib().lp_check_recover(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(d_n_recovered),
+                                          _stream(stream)))
+        else:
+            _check(lib().lp_check_recover_ws(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck),
+                                             _ptr(d_n_recovered), _ptr(workspace), _stream(stream)))
 
     def attach_nvls_count(self, mc_ptr, uc_ptr, world_size: int):
         """NVLS-fused all-rank failed count (lp_attach_nvls_count); pointers are ints or tensors (None, None: off)."""

@@ -14,14 +14,17 @@ for st in array quad_cas quad_lock cuckoo cuckoo_lock; do
 done
 D=$D python - <<'PY'
 import glob, json, os
-print("| store | reduction | t_prot ms | t_unprot ms | LP overhead | slowdown (x) | hash collisions |")
-print("|---|---|---|---|---|---|---|")
+print("| store | reduction | t_prot ms | t_unprot ms | LP overhead (median of pairs) | pair IQR | slowdown (x) | "
+      "hash collisions (quad: extra probes; cuckoo: evictions) |")
+print("|---|---|---|---|---|---|---|---|")
 for f in sorted(glob.glob(os.environ["D"] + "/*.json")):
     try:
         d = json.loads(open(f).read().strip().splitlines()[-1])
     except Exception:
         continue
     c = d["config"]
+    iqr = d.get("lp_overhead_detail", {}).get("iqr_pct", [None, None])
     print(f"| {c['store']} | {c['reduction']} | {d['t_protected_ms']:.3f} | {d['t_unprotected_ms']:.3f} | "
-          f"{d['lp_overhead_pct']:+.2f}% | {d['t_protected_ms'] / d['t_unprotected_ms']:.2f} | {d.get('hash_collisions')} |")
+          f"{d['lp_overhead_pct']:+.2f}% | [{iqr[0]:+.2f}, {iqr[1]:+.2f}]% | "
+          f"{d['t_protected_ms'] / d['t_unprotected_ms']:.2f} | {d.get('hash_collisions')} |")
 PY
