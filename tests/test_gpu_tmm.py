@@ -346,7 +346,8 @@ def test_cuckoo_full_r262144(store):
 @pytest.mark.parametrize("reg,out_dt,store", [(128, "bf16", "array"), (32, "bf16", "array"), (128, "f32", "array"),
                                               (32, "f32", "quad_cas"), (128, "bf16", "cuckoo")])
 @pytest.mark.parametrize("frac", [0.01, 0.10, 0.50])
-def test_tmm_same_grid_check_and_recover(reg, out_dt, store, frac):
+@pytest.mark.parametrize("balanced", [False, True])
+def test_tmm_same_grid_check_and_recover(reg, out_dt, store, frac, balanced):
     """Listing 7 (L565-578) on the tcgen05 CTA-pair TMM: one kernel validates every region of its tiles and
     recomputes in place only the tiles holding a failed region.  The count equals the oracle's failed set on
     the corrupted image, the recovered bytes equal the golden run, and a re-validate finds nothing."""
@@ -365,7 +366,8 @@ def test_tmm_same_grid_check_and_recover(reg, out_dt, store, frac):
     R = h.num_regions(wl)
     # clean image: nothing fails, nothing is recomputed
     d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
-    h.check_recover(wl, out, ck, d_rec)
+    wsb = ws if balanced else None
+    h.check_recover(wl, out, ck, d_rec, workspace=wsb)
     torch.cuda.synchronize()
     assert int(d_rec.item()) == 0
     inj = torch.from_numpy(lp.choose_regions(R, frac, 500 + reg)).cuda()
@@ -373,7 +375,7 @@ def test_tmm_same_grid_check_and_recover(reg, out_dt, store, frac):
     torch.cuda.synchronize()
     exp = oracle_validate(dev_to_host(out), dev_to_host(ck), store, reg, reg, h.mask)
     assert len(exp) > 0
-    h.check_recover(wl, out, ck, d_rec)
+    h.check_recover(wl, out, ck, d_rec, workspace=wsb)
     torch.cuda.synchronize()
     assert int(d_rec.item()) == len(exp)
     assert np.array_equal(dev_to_host(out).view(np.uint8), golden.view(np.uint8))
@@ -404,10 +406,12 @@ def test_tmm_check_and_recover_full_8192():
     torch.cuda.synchronize()
     exp = oracle_validate(dev_to_host(out), dev_to_host(ck), "array", 128, 128, h.mask)
     d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
-    h.check_recover(wl, out, ck, d_rec)
-    torch.cuda.synchronize()
-    assert int(d_rec.item()) == len(exp) > 0
-    assert torch.equal(out.view(torch.int16), golden.view(torch.int16))
+    for wsb in (None, ws):                     # static, then balanced (re-corrupted in between)
+        h.inject(wl, out, ck, stale, inj, mode="stale_words", seed=1001)
+        h.check_recover(wl, out, ck, d_rec, workspace=wsb)
+        torch.cuda.synchronize()
+        assert int(d_rec.item()) == len(exp) > 0
+        assert torch.equal(out.view(torch.int16), golden.view(torch.int16))
 
 
 @pytest.mark.parametrize("frac", [0.02, 0.3, 1.0])
