@@ -28,8 +28,6 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include <cstdlib>
-
 #include "lp_device.cuh"
 #include "lp_internal.h"
 
@@ -228,11 +226,9 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   const int sk = a.mask ? a.hash.store : 0;
   // full run: one region per CTA, barrier-free combine; list mode (recovery):
   // persistent CTAs over the failed list, barrier combine (accumulators reused)
-  static const int64_t per_sm = [] {  // list-mode CTAs per SM (LP_STENCIL_LIST_CTAS=<n> for A/B runs)
-    const char* e = getenv("LP_STENCIL_LIST_CTAS");
-    return e ? (int64_t)atoi(e) : (int64_t)2;
-  }();
-  int64_t grid = a.list ? (R < a.sm_count * per_sm ? R : a.sm_count * per_sm) : R;
+  // list mode: 2 persistent CTAs per SM (the occupancy limit); 8 / 32 / 64 per SM, and one region per CTA over
+  // R CTAs with the split-barrier combine, measured the same recovery phase
+  int64_t grid = a.list ? (R < a.sm_count * 2 ? R : a.sm_count * 2) : R;
   if (grid < 1) grid = 1;
   switch (a.mask * 5 + sk) {
 #define LP_LCASE(M, S)                                                                                          \
