@@ -950,9 +950,10 @@ def run_reference(args):
             "scaling": "weak" if W["weak"] else "strong", "vs_baseline": None, "dtype": W["in_dt"] + "->" + W["out_dt"],
             "data": "synthetic", "config": {"workload": args.workload, "region": [RM, RN], "cksum": W["cksum"]},
             "cpu_baseline": {"value": round(value, 4), "unit": "GB/s", "cores": T, "kind": "oracle",
-                             "sample": f"per step ~{per_step:.0f} s of oracle work on {T} host threads: records "
-                                       f"recomputed and compared on sampled {RM}x{RN} regions + fp64 re-execution "
-                                       f"of regions"},
+                             "sample": f"per step {sum(times) / len(times):.1f} s wall of oracle work on {T} host "
+                                       f"threads (budget {per_step:.0f} s): records recomputed and compared on the "
+                                       f"{R} {RM}x{RN} regions of a slab of the workload + fp64 re-execution of "
+                                       f"regions"},
             "e2e": {"value": round(value, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
