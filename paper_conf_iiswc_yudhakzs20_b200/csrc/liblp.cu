@@ -222,7 +222,7 @@ WsLayout ws_layout(const lp::RegionGeom& g) {
   w.part = w.d_ntasks + 256;
   w.cnt = w.part + al(npart * 32);
   w.gbits = w.cnt + al(npart * 4);                  // balanced check-and-recover: global failed-tile bitmask
-  w.gbar = w.gbits + al((size_t)(g.R + 31) / 32 * 4);  //   and its grid-barrier counter (cleared per call)
+  w.gbar = w.gbits + al((size_t)(g.R + 15) / 16 * 4);  //   (2 bits per tile) and its grid-barrier counter
   w.ticket = w.gbar + 256;                          // fused-compaction ticket (u32; zero-initialised, kept at 0)
   w.total = w.ticket + 256;
   return w;

@@ -332,8 +332,13 @@ constexpr int kSmem2Bytes = kStages2 * kStage2Bytes + 1024 + 1024;
 // (32x32 regions) or a whole 128-row half (128x128 regions) of a tile; the 6 warps take items
 // round robin, lane l reads 16-byte chunk l (+32) of every row (coalesced 512-B rows), each lane's
 // chunks stay inside one region column, so a segmented warp reduction yields the records.  A
-// failed region sets its tile's bit in this CTA's shared bitmask and bumps *d_rec.
-constexpr int kCheckUnroll = 8;
+// failed region sets its tile-half's bit (2 bits per tile) in this CTA's shared bitmask and bumps *d_rec;
+// a tile with one failed half is recomputed as a 256x128 tile (N = 128), else as the full 256x256.
+// rows of 16-B loads in flight per lane in the check phase (32 for bf16, 16 for fp32 rows of two chunks:
+// 128 registers of loads; the kernel has the register file to itself at 1 CTA per SM)
+#ifndef LP_CHECK_ROWS
+#define LP_CHECK_ROWS 32
+#endif
 
 __device__ __forceinline__ uint4 ld_u4_noalloc(const void* p) {
   uint4 r;
@@ -356,6 +361,7 @@ __device__ __forceinline__ void check_tiles(const OutT* __restrict__ C, int64_t 
   constexpr int LGL = CPRR >= 32 ? 5 : (CPRR == 16 ? 4 : (CPRR == 8 ? 3 : 2));
   constexpr int RB = REG == 32 ? 32 : 128;      // rows per work item
   constexpr int NB = 128 / RB;                  // items per tile half
+  constexpr int kCheckUnroll = (LP_CHECK_ROWS / U) < RB ? (LP_CHECK_ROWS / U) : RB;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t nloc = (ntiles - pair + npairs - 1) / npairs;
   for (int64_t it = warp; it < nloc * NB; it += kThreads / 32) {
@@ -402,7 +408,9 @@ __device__ __forceinline__ void check_tiles(const OutT* __restrict__ C, int64_t 
           for (int s2 = 0; s2 < S; ++s2) bad |= (!bad && stored[s2] != w[s2]);
         }
         if (bad) {
-          atomicOr(&s_fail[lt >> 5], 1u << (lt & 31));
+          // two bits per tile: which 128-column half holds the failed region
+          const int h = (int)((c / CPRR) * REG / 128);
+          atomicOr(&s_fail[lt >> 4], 1u << (2 * (lt & 15) + h));
           atomicAdd(reinterpret_cast<unsigned long long*>(d_rec), 1ull);
         }
       }
@@ -411,9 +419,10 @@ __device__ __forceinline__ void check_tiles(const OutT* __restrict__ C, int64_t 
 }
 
 // Tile walk of a CTA pair.  CHECK 0: the persistent schedule t = pair, pair + npairs, ...; 1 (Listing 7,
-// static): the same schedule, skipping tiles whose bit is clear in the pair's merged bitmask `todo`;
-// 2 (Listing 7, balanced): the j-th failed tile of the GLOBAL bitmask (ascending tile index) goes to pair
-// j % npairs -- every role of both CTAs derives the same sequence from the bitmask, no broadcast needed.
+// static): the same schedule, skipping tiles whose two half bits are clear in the pair's merged bitmask
+// `todo` (2 bits per local tile); 2 (Listing 7, balanced): the j-th failed tile of the GLOBAL bitmask (2 bits
+// per tile id, ascending tile index) goes to pair j % npairs -- every role of both CTAs derives the same
+// sequence from the bitmask, no broadcast needed.  half = which 128-column halves to compute (bit 0 / 1).
 template <int CHECK>
 struct TileWalk {
   int64_t t, lt, pair, npairs, ntiles;
@@ -424,20 +433,22 @@ struct TileWalk {
   __device__ __forceinline__ TileWalk(int64_t pair_, int64_t npairs_, int64_t ntiles_, const uint32_t* todo_,
                                       const uint32_t* gbits_)
       : t(pair_ - npairs_), lt(-1), pair(pair_), npairs(npairs_), ntiles(ntiles_), todo(todo_), gbits(gbits_), w(-1),
-        nwords((ntiles_ + 31) >> 5), j(0), cur(0u) {}
-  __device__ __forceinline__ bool next(int64_t& out) {
+        nwords((ntiles_ + 15) >> 4), j(0), cur(0u) {}
+  __device__ __forceinline__ bool next(int64_t& out, int& half) {
     if constexpr (CHECK == 2) {
       for (;;) {
         while (cur == 0u) {
           if (++w >= nwords) return false;
           cur = __ldcg(gbits + w);
         }
-        const int b = __ffs(cur) - 1;
-        cur &= cur - 1u;
+        const int b = (__ffs(cur) - 1) >> 1;  // tile slot in this word
+        const uint32_t m = (cur >> (2 * b)) & 3u;
+        cur &= ~(3u << (2 * b));
         const bool mine = (j % npairs) == pair;
         ++j;
         if (mine) {
-          out = w * 32 + b;
+          out = w * 16 + b;
+          half = (int)m;
           return true;
         }
       }
@@ -446,7 +457,11 @@ struct TileWalk {
         t += npairs;
         ++lt;
         if (t >= ntiles) return false;
-        if (CHECK == 1 && !((todo[lt >> 5] >> (lt & 31)) & 1u)) continue;
+        half = 3;
+        if (CHECK == 1) {
+          half = (int)((todo[lt >> 4] >> (2 * (lt & 15))) & 3u);
+          if (!half) continue;
+        }
         out = t;
         return true;
       }
@@ -504,7 +519,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   // Listing 7 form: failed-tile bitmask of this pair's local tile sequence (own half | peer half)
   uint32_t* s_fail = reinterpret_cast<uint32_t*>(srec + 16);
   const int64_t nloc = (ntiles - pair + npairs - 1) / npairs;
-  const int nwords = (int)((nloc + 31) >> 5);
+  const int nwords = (int)((nloc + 15) >> 4);  // 2 bits per local tile
   uint32_t* s_todo = s_fail + nwords;
   if constexpr (CHECK != 0) {
     for (int i = threadIdx.x; i < nwords; i += kThreads) s_fail[i] = 0u;
@@ -526,10 +541,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       for (int i = threadIdx.x; i < nwords; i += kThreads) {
         uint32_t m = s_fail[i];
         while (m) {
-          const int64_t lt = (int64_t)i * 32 + (__ffs(m) - 1);
+          const int bit = __ffs(m) - 1;
           m &= m - 1u;
+          const int64_t lt = (int64_t)i * 16 + (bit >> 1);
           const int64_t t = pair + lt * npairs;
-          atomicOr(gbits + (t >> 5), 1u << (t & 31));
+          atomicOr(gbits + (t >> 4), 1u << (2 * (t & 15) + (bit & 1)));
         }
       }
       __syncthreads();
@@ -552,20 +568,23 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       uint32_t phase = 0;
       TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
       int64_t t;
-      while (walk.next(t)) {
+      int half;
+      while (walk.next(t, half)) {
         int64_t mb, nb;
         tile_coords(t, num_m, num_n, mb, nb);
-        const int m0 = (int)(mb * 256 + rank * 128), n0 = (int)(nb * 256 + rank * 128);
+        // N = 256: each CTA stages 128 columns of B; one failed half (N = 128): 64 columns of that half
+        const int nw = half == 3 ? 256 : 128, hoff = half == 2 ? 128 : 0;
+        const int m0 = (int)(mb * 256 + rank * 128), n0 = (int)(nb * 256 + hoff + rank * (nw / 2));
         for (int kb = 0; kb < nkb; ++kb) {
           mbar_wait(&empty[stage], phase ^ 1);
           const uint32_t full0 = mapa_rank0(&full[stage]);
           if (rank == 0)
-            mbar_expect_tx(&full[stage], 2 * kStage2Bytes);
+            mbar_expect_tx(&full[stage], 2 * (kA2Bytes + (nw / 2) * kBK * 2));
           else
             mbar_arrive_remote(full0);
           tma_load_2d_pair(&tmap_a, full0, sA + stage * kA2Bytes, kb * kBK, m0);
           tma_load_2d_pair(&tmap_b, full0, sB + stage * kB2Bytes, n0, kb * kBK);
-          tma_load_2d_pair(&tmap_b, full0, sB + stage * kB2Bytes + kBK * 128, n0 + 64, kb * kBK);
+          if (nw == 256) tma_load_2d_pair(&tmap_b, full0, sB + stage * kB2Bytes + kBK * 128, n0 + 64, kb * kBK);
           if (++stage == kStages2) {
             stage = 0;
             phase ^= 1;
@@ -584,7 +603,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       uint32_t acc_phase = 0;
       TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
       int64_t t;
-      while (walk.next(t)) {
+      int half;
+      while (walk.next(t, half)) {
+        const uint32_t idesc_t = half == 3 ? idesc : ((idesc & ~(0x3Fu << 17)) | ((uint32_t)(128 >> 3) << 17));
         mbar_wait(&tempty[acc], acc_phase ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(acc * BN);
@@ -597,7 +618,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           for (int k = 0; k < kBK / kUmmaK; ++k) {
             const uint64_t ad = smem_desc(a_addr + k * kUmmaK * 2, 16, 1024);
             const uint64_t bd = smem_desc(b_addr + k * kUmmaK * 128, kBK * 128, 1024);
-            tc_mma_pair(d_tmem, ad, bd, idesc, (kb | k) ? 1u : 0u);
+            tc_mma_pair(d_tmem, ad, bd, idesc_t, (kb | k) ? 1u : 0u);
           }
           tc_commit_pair(&empty[stage]);
           if (++stage == kStages2) {
@@ -618,7 +639,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     uint32_t acc_phase = 0;
     TileWalk<CHECK> walk(pair, npairs, ntiles, s_todo, gbits);
     int64_t t;
-    while (walk.next(t)) {
+    int half;
+    while (walk.next(t, half)) {
       int64_t mb, nb;
       tile_coords(t, num_m, num_n, mb, nb);
       mbar_wait(&tfull[acc], acc_phase);
@@ -626,6 +648,26 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       const uint32_t t_row = tmem_base + ((uint32_t)(wq * 32) << 16) + (uint32_t)(acc * BN);
       CkRecord* srec_acc = srec + acc * 2 * 4;
       const int64_t m128 = mb * 2 + rank;
+      if (CHECK != 0 && half != 3) {
+        // one failed 128-column half recomputed as 256x128: accumulator columns [0, 128) -> C columns of that half
+        const int64_t n0h = nb * BN + (half == 2 ? 128 : 0);
+        epi_store<OutT, MASK, REG, 128, STORE>(t_row, C, ldc, m128, n0h, wq, lane, srec_acc, ck, Qr, rid_offset);
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (rank == 0)
+            mbar_arrive(&tempty[acc]);
+          else
+            mbar_arrive_remote(mapa_rank0(&tempty[acc]));
+        }
+        if constexpr (MASK != 0 && REG == 128)
+          epi_finish_halves<OutT, MASK, STORE>(warp, lane, srec_acc, ck, m128, n0h, n0h, false, Qr, rid_offset);
+        if (++acc == 2) {
+          acc = 0;
+          acc_phase ^= 1;
+        }
+        continue;
+      }
       epi_store<OutT, MASK, REG, BN, STORE>(t_row, C, ldc, m128, nb * BN, wq, lane, srec_acc, ck, Qr, rid_offset);
       tc_fence_before();
       __syncwarp();
@@ -1052,12 +1094,18 @@ cudaError_t launch_pair_check(const TmmArgs& a, int64_t* d_rec, uint32_t* gbits,
   cudaError_t e = cudaMemsetAsync(d_rec, 0, sizeof(int64_t), st);
   if (e != cudaSuccess) return e;
   const bool balanced = gbits != nullptr && gbar != nullptr;
-  if (balanced) {  // grid barrier counter + global failed-tile bitmask, cleared in stream order
-    e = cudaMemsetAsync(gbar, 0, sizeof(uint32_t), st);
-    if (e == cudaSuccess) e = cudaMemsetAsync(gbits, 0, (size_t)((num_m * num_n + 31) / 32) * 4, st);
+  if (balanced) {  // global failed-tile bitmask + grid barrier counter, cleared in stream order (one memset when
+                   // the counter directly follows the bitmask, as in liblp's workspace layout)
+    const size_t bits_bytes = (size_t)((num_m * num_n + 15) / 16) * 4;
+    if (gbar > gbits && (size_t)((uint8_t*)gbar - (uint8_t*)gbits) <= bits_bytes + 4096) {
+      e = cudaMemsetAsync(gbits, 0, (size_t)((uint8_t*)gbar - (uint8_t*)gbits) + sizeof(uint32_t), st);
+    } else {
+      e = cudaMemsetAsync(gbar, 0, sizeof(uint32_t), st);
+      if (e == cudaSuccess) e = cudaMemsetAsync(gbits, 0, bits_bytes, st);
+    }
     if (e != cudaSuccess) return e;
   }
-  auto smem_for = [&](int64_t g) { return kSmem2Bytes + (int)(2 * (((num_m * num_n + g / 2 - 1) / (g / 2)) + 31) / 32 * 4); };
+  auto smem_for = [&](int64_t g) { return kSmem2Bytes + (int)(2 * (((num_m * num_n + g / 2 - 1) / (g / 2)) + 15) / 16 * 4); };
   switch (a.mask * 5 + a.hash.store) {
 #define LP_TC2C_CASE(M, S)                                                                                  \
   case M * 5 + S: {                                                                                         \
