@@ -617,10 +617,15 @@ __global__ void hash_header_kernel(uint32_t* ck, uint32_t cap, uint32_t seed, ui
 constexpr int kRehashAttempts = 16;
 __global__ void __launch_bounds__(1024) cuckoo_rehash_kernel(uint32_t* ck) {
   HashHeader* hdr = reinterpret_cast<HashHeader*>(ck);
-  if (*reinterpret_cast<volatile uint32_t*>(&hdr->stash_n) == 0) return;
   __shared__ uint4 s_stash[kCuckooStash];
-  __shared__ uint32_t s_n, s_seed;
+  __shared__ uint32_t s_n, s_seed, s_more;
   __shared__ unsigned long long s_coll;
+  // loop control is decided by thread 0 (an atomic read of the stash count at gpu scope) and shared, so every
+  // thread takes the same number of attempts (a per-thread read could see a stale value and split the CTA
+  // across the __syncthreads below)
+  if (threadIdx.x == 0) s_more = atomicAdd(&hdr->stash_n, 0u);
+  __syncthreads();
+  if (s_more == 0) return;
   uint4* tab = reinterpret_cast<uint4*>(ck + sizeof(HashHeader) / 4);
   const uint32_t cap = hdr->cap;
   if (threadIdx.x == 0) s_coll = hdr->collisions;
@@ -654,7 +659,9 @@ __global__ void __launch_bounds__(1024) cuckoo_rehash_kernel(uint32_t* ck) {
     for (uint32_t i = threadIdx.x; i < s_n; i += blockDim.x) cuckoo_place(hdr, tab, cap, seed, s_stash[i], kCuckooMaxEvict, false);
     __threadfence();
     __syncthreads();
-    if (*reinterpret_cast<volatile uint32_t*>(&hdr->stash_n) == 0) break;
+    if (threadIdx.x == 0) s_more = atomicAdd(&hdr->stash_n, 0u);
+    __syncthreads();
+    if (s_more == 0) break;
   }
   __syncthreads();
   if (threadIdx.x == 0) {

@@ -709,7 +709,41 @@ constexpr int kB4Bytes = kBK * 128 * 2;   // 16 KiB: this CTA's 128 columns of B
 constexpr int kStage4Bytes = kA4Bytes + kB4Bytes;
 constexpr int kSmem4Bytes = kStages4 * kStage4Bytes + 1024 + 1024;
 
-template <typename OutT, uint32_t MASK, int REG, int STORE>
+// Work distribution of the 256-row kernel.  Static (CLC = false): persistent grid, pair p takes tiles p,
+// p + npairs, ...  Cluster launch control (CLC = true): one cluster per tile in the grid; a running pair
+// claims the next not-yet-launched cluster's tile with clusterlaunchcontrol.try_cancel (issued by the
+// leader's producer thread, multicast to both CTAs' smem, completing 16 bytes on each CTA's clc_full
+// barrier), so the tiles in flight stay a contiguous window of the raster (the order a non-persistent launch
+// would run them in) while each SM keeps its TMEM / barriers / pipeline across tiles.  Every role of both
+// CTAs reads each response and arrives on the leader's clc_empty for the slot (11 arrivals: 2 producers, the
+// MMA thread, 8 epilogue warps) before the slot is reused.
+constexpr int kClcSlots = 4;
+constexpr uint32_t kClcConsumers = 11;
+
+__device__ __forceinline__ void clc_try_cancel(uint4* resp, uint64_t* bar) {
+  asm volatile(
+      "clusterlaunchcontrol.try_cancel.async.shared::cta.mbarrier::complete_tx::bytes.multicast::cluster::all.b128 "
+      "[%0], [%1];" ::"r"(smem_u32(resp)),
+      "r"(smem_u32(bar))
+      : "memory");
+}
+// -1: no more work (no cluster was cancelled); else the tile of the cancelled cluster (first ctaid.x / 2)
+__device__ __forceinline__ int64_t clc_decode(const uint4* resp) {
+  uint32_t x, valid;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t.reg .b128 r;\n\t"
+      "ld.shared.b128 r, [%2];\n\t"
+      "clusterlaunchcontrol.query_cancel.is_canceled.pred.b128 p, r;\n\t"
+      "selp.u32 %1, 1, 0, p;\n\t"
+      "mov.u32 %0, 0;\n\t"
+      "@p clusterlaunchcontrol.query_cancel.get_first_ctaid.v4.b32.b128 {%0, _, _, _}, r;\n\t}"
+      : "=r"(x), "=r"(valid)
+      : "r"(smem_u32(resp))
+      : "memory");
+  return valid ? (int64_t)(x >> 1) : -1;
+}
+
+template <typename OutT, uint32_t MASK, int REG, int STORE, bool CLC = false>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     tmm_tc4_kernel(const __grid_constant__ CUtensorMap tmap_a, const __grid_constant__ CUtensorMap tmap_b,
                    OutT* __restrict__ C, int64_t ldc, int64_t K, int64_t num_m, int64_t num_n, int64_t group,
@@ -725,6 +759,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_holder = (uint32_t*)(tempty + 2);
   CkRecord* srec = (CkRecord*)(tmem_holder + 4);
+  uint4* clc_resp = (uint4*)(srec + 16);
+  uint64_t* clc_full = (uint64_t*)(clc_resp + kClcSlots);
+  uint64_t* clc_empty = clc_full + kClcSlots;
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
@@ -741,8 +778,38 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       mbar_init(&tfull[s], 1);
       mbar_init(&tempty[s], 8);  // 4 epilogue warps x 2 CTAs, used in rank 0
     }
+    if constexpr (CLC) {
+      for (int s = 0; s < kClcSlots; ++s) {
+        mbar_init(&clc_full[s], 1);                 // this CTA's producer: arrive.expect_tx(16)
+        mbar_init(&clc_empty[s], kClcConsumers);    // used in rank 0
+      }
+    }
     fence_barrier_init();
   }
+  // next tile of this role: the static stride, or the next CLC response (fetch index i)
+  int clc_i = 0;
+  auto clc_next = [&](bool expect_tx, bool arrive) -> int64_t {
+    const int slot = clc_i % kClcSlots;
+    const uint32_t par = (uint32_t)((clc_i / kClcSlots) & 1);
+    if (expect_tx) mbar_expect_tx(&clc_full[slot], 16);
+    mbar_wait(&clc_full[slot], par);
+    const int64_t t = clc_decode(&clc_resp[slot]);
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    if (arrive) {
+      if (rank == 0)
+        mbar_arrive(&clc_empty[slot]);
+      else
+        mbar_arrive_remote(mapa_rank0(&clc_empty[slot]));
+    }
+    ++clc_i;
+    return t;
+  };
+  // leader producer: claim the work for fetch j (slot j % S free once fetch j - S is consumed everywhere)
+  auto clc_issue = [&](int j) {
+    const int slot = j % kClcSlots;
+    mbar_wait(&clc_empty[slot], (uint32_t)(((j / kClcSlots) & 1) ^ 1));
+    clc_try_cancel(&clc_resp[slot], &clc_full[slot]);
+  };
   if (warp == 1) {
     asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_holder)),
                  "r"(512u)
@@ -760,7 +827,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int64_t t = pair; t < ntiles; t += npairs) {
+      if (CLC && rank == 0) clc_issue(0);
+      for (int64_t t = pair; CLC ? t >= 0 : t < ntiles;) {
         int64_t mb, nb;
         tile_coords_g(t, num_m, num_n, group, mb, nb);
         const int m0 = (int)(mb * 512 + rank * 256), n0 = (int)(nb * 256 + rank * 128);
@@ -779,6 +847,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
             phase ^= 1;
           }
         }
+        if constexpr (CLC) {
+          t = clc_next(true, true);
+          if (rank == 0 && t >= 0) clc_issue(clc_i);
+        } else {
+          t += npairs;
+        }
       }
     }
   } else if (warp == 1) {
@@ -788,7 +862,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       int stage = 0;
       uint32_t phase = 0;
       uint32_t acc_phase = 0;
-      for (int64_t t = pair; t < ntiles; t += npairs) {
+      for (int64_t t = pair; CLC ? t >= 0 : t < ntiles; t = CLC ? clc_next(false, true) : t + npairs) {
         mbar_wait(&tempty[0], acc_phase ^ 1);  // D0 drained by the previous tile's epilogue
         tc_fence_after();
         for (int kb = 0; kb < nkb; ++kb) {
@@ -818,10 +892,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
         acc_phase ^= 1;
       }
     }
-  } else {
+  } else if (warp >= kEpiWarp0) {
     const int wq = warp & 3;
     uint32_t acc_phase = 0;
-    for (int64_t t = pair; t < ntiles; t += npairs) {
+    for (int64_t t = pair; CLC ? t >= 0 : t < ntiles;) {
       int64_t mb, nb;
       tile_coords_g(t, num_m, num_n, group, mb, nb);
 #pragma unroll 1
@@ -844,6 +918,13 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
           epi_finish_128<OutT, MASK, BN, STORE>(warp, lane, srec_d, ck, m128, nb * BN, Qr, rid_offset);
       }
       acc_phase ^= 1;
+      if constexpr (CLC) {
+        // every lane reads the response; lane 0 arrives for the warp
+        t = clc_next(false, lane == 0);
+        __syncwarp();
+      } else {
+        t += npairs;
+      }
     }
   }
 
@@ -1007,12 +1088,21 @@ int tc4_mode() {
   }();
   return v;
 }
+// The 256-row kernel takes its tiles through cluster launch control (LP_TC_CLC=0: static persistent
+// schedule, A/B): at 32768^3 DRAM reads 158 -> 98 GB, C5 65536^3 485 -> 442 ms = cuBLAS (profiles/r02/ab_clc.txt)
+bool tc4_clc() {
+  static bool v = [] {
+    const char* e = getenv("LP_TC_CLC");
+    return !(e && atoi(e) == 0);
+  }();
+  return v;
+}
 int64_t tc4_group() {
   static int64_t v = [] {
     const char* e = getenv("LP_TC4_GROUP");
-    return e ? (int64_t)atoi(e) : (int64_t)2;
+    return e ? (int64_t)atoi(e) : (int64_t)0;  // 0: per launch, 4 with CLC, 2 static
   }();
-  return v < 1 ? 1 : v;
+  return v < 0 ? 0 : v;
 }
 
 template <typename OutT, int REG>
@@ -1024,18 +1114,27 @@ cudaError_t launch_pair4(const TmmArgs& a, cudaStream_t st, const char** why) {
     return cudaErrorInvalidValue;
   }
   const int64_t num_m = a.M / 512, num_n = a.N / 256;
-  int64_t grid = 2 * num_m * num_n;
+  // CLC only with the array store: with the hash-store ablations the CLC variant hung or stored wrong records
+  // from ~512 tiles up (8192^2+ outputs; smaller grids and the array store are exact) -- root cause not found
+  // (a standalone CLC loop with slow consumers is exactly-once, tools/probe/clc); hash stores keep the static
+  // persistent schedule
+  const bool clc = tc4_clc() && (a.mask == 0 || a.hash.store == 0);
+  int64_t grid = 2 * num_m * num_n;  // CLC: one cluster per tile
   const int64_t cap = a.sm_count & ~1;
-  if (grid > cap) grid = cap;
+  if (!clc && grid > cap) grid = cap;
   if (grid < 2) grid = 2;
+  if (grid > (int64_t)0x7FFFFFFF) {
+    *why = "grid too large";
+    return cudaErrorInvalidValue;
+  }
   const int64_t Qr = a.N / REG;
   const int sk = a.mask ? a.hash.store : 0;
-  const int64_t G = tc4_group();
+  const int64_t G = tc4_group() ? tc4_group() : (clc ? 4 : 2);
   cudaError_t e = cudaSuccess;
   switch (a.mask * 5 + sk) {
 #define LP_TC4_CASE(M, S)                                                                                   \
   case M * 5 + S: {                                                                                         \
-    auto kfn = tmm_tc4_kernel<OutT, M, REG, S>;                                                            \
+    auto kfn = clc ? tmm_tc4_kernel<OutT, M, REG, S, true> : tmm_tc4_kernel<OutT, M, REG, S, false>;        \
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem4Bytes);                \
     if (e != cudaSuccess) return e;                                                                         \
     kfn<<<(unsigned)grid, kThreads, kSmem4Bytes, st>>>(ma, mb, (OutT*)a.C, a.ldc, a.K, num_m, num_n, G, Qr, \
