@@ -788,13 +788,16 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
   }
   // next tile of this role: the static stride, or the next CLC response (fetch index i)
   int clc_i = 0;
-  auto clc_next = [&](bool expect_tx, bool arrive) -> int64_t {
+  // whole_warp: every lane reads the response; the warp converges BEFORE lane 0 releases the slot -- a lane
+  // still to read it would otherwise see the next response the leader may issue into the slot at once
+  auto clc_next = [&](bool expect_tx, bool arrive, bool whole_warp = false) -> int64_t {
     const int slot = clc_i % kClcSlots;
     const uint32_t par = (uint32_t)((clc_i / kClcSlots) & 1);
     if (expect_tx) mbar_expect_tx(&clc_full[slot], 16);
     mbar_wait(&clc_full[slot], par);
     const int64_t t = clc_decode(&clc_resp[slot]);
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    if (whole_warp) __syncwarp();
     if (arrive) {
       if (rank == 0)
         mbar_arrive(&clc_empty[slot]);
@@ -919,9 +922,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
       }
       acc_phase ^= 1;
       if constexpr (CLC) {
-        // every lane reads the response; lane 0 arrives for the warp
-        t = clc_next(false, lane == 0);
-        __syncwarp();
+        // every lane reads the response; lane 0 arrives for the warp once all have read it
+        t = clc_next(false, lane == 0, true);
       } else {
         t += npairs;
       }
@@ -1114,11 +1116,7 @@ cudaError_t launch_pair4(const TmmArgs& a, cudaStream_t st, const char** why) {
     return cudaErrorInvalidValue;
   }
   const int64_t num_m = a.M / 512, num_n = a.N / 256;
-  // CLC only with the array store: with the hash-store ablations the CLC variant hung or stored wrong records
-  // from ~512 tiles up (8192^2+ outputs; smaller grids and the array store are exact) -- root cause not found
-  // (a standalone CLC loop with slow consumers is exactly-once, tools/probe/clc); hash stores keep the static
-  // persistent schedule
-  const bool clc = tc4_clc() && (a.mask == 0 || a.hash.store == 0);
+  const bool clc = tc4_clc();
   int64_t grid = 2 * num_m * num_n;  // CLC: one cluster per tile
   const int64_t cap = a.sm_count & ~1;
   if (!clc && grid > cap) grid = cap;
