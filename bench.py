@@ -456,7 +456,7 @@ def run_ours(args):
         graphs = {}
         for name, fn in list(runners.items()):
             g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g):
+            with torch.cuda.graph(g, capture_error_mode="thread_local"):
                 fn()
             graphs[name] = g
         for name, g in graphs.items():
@@ -544,7 +544,7 @@ def run_ours(args):
         gs = []
         for with_val in (False, True):
             g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g):
+            with torch.cuda.graph(g, capture_error_mode="thread_local"):
                 for _ in range(nrep):
                     l2_flush()
                     if with_val:
