@@ -443,12 +443,14 @@ def run_ours(args):
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[2:3].copy_(nvls_buf[4:5] if nvls_buf is not None else d_n)
 
+    # One NCCL all-reduce per step: the recovery of every shard needs only its own (device) failed count, so
+    # the all-rank failed count travels with the summary {n_failed, n_recovered, n_failed_after} after the
+    # re-validation.  With the NVLS counter the failed count is already all-reduced inside lp_validate.
     def reduce_failed():
-        if nvls_buf is None:
-            shard.allreduce_counts(counts[0:1])
+        pass
 
     def reduce_summary():
-        shard.allreduce_counts(counts[1:2] if nvls_buf is not None else counts[1:3])
+        shard.allreduce_counts(counts[1:2] if nvls_buf is not None else counts[0:3])
 
     runners = {"body": seg_body, "inject": seg_inject, "validate": seg_validate, "recover": seg_recover}
 
@@ -772,8 +774,8 @@ def run_ours(args):
             "n_failed_per_step": n_failed,
             "n_recovered_per_step": n_recovered,
             "count_allreduce": (nvls_note if args.nvls_count else
-                                ("NCCL all_reduce(SUM) of int64 counts on the compute stream" if world > 1
-                                 else "none (N = 1)")),
+                                ("one NCCL all_reduce(SUM) of the int64 summary {n_failed, n_recovered, "
+                                 "n_failed_after} per step, on the compute stream" if world > 1 else "none (N = 1)")),
             "n_failed_after_recover": n_after,
             "per_rank": spread,
             "hash_collisions": hash_stats[0] if W["store"] != "array" else None,
