@@ -25,11 +25,15 @@
 // speeds the plain kernel up), so the LP overhead compares like with like.
 // (List-mode recovery, where a CTA handles several regions, uses the barrier
 // combine; measured A/Bs in DESIGN.md.)
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "lp_device.cuh"
 #include "lp_internal.h"
+#include "lp_ptx.cuh"
+#include "lp_tma.h"
 
 namespace lp {
 namespace {
@@ -216,6 +220,226 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
 }
 
 
+// ---- TMA-fed persistent form of the full run (one CTA per SM; A/B, LP_STENCIL_TMA=1, not the default) ----
+//
+// Per region, three cp.async.bulk.tensor boxes land in one stage of a 3-deep ring: the 130 x 128 centre
+// (region rows -1 .. 128, line-aligned) and the 4-column halo strips left and right.  The tensor maps
+// cover only this shard's readable rows [row_lo, row_lo + row_span) and the W domain columns, so TMA's
+// out-of-bounds zero fill IS the stencil's zero boundary (R19).  Warp NW (one lane) is the producer and
+// keeps two regions in flight ahead of the consumers, whatever the consumers' checksum epilogue costs;
+// it also combines the NW warp partials (Listing 3) and stores the record (L349) once a stage is
+// released.  Consumer warps read the stage from shared memory (one 16-B vector per row, conflict-free)
+// with the same lane -> column mapping and per-lane partials as the LDG form.
+// Measured (profiles/r02/ab_stencil_tma.txt): Adler costs only +1.6% over THIS form's twin, but the twin
+// itself takes 1.57-1.70 ms against the LDG form's 1.29 ms: with the output stores in the mix the halo
+// strips are re-read from DRAM (5.14 vs 4.35 GB read), and even without halos (diagnostic build) TMA +
+// stores ran 1.43 ms.  So the LDG form stays the default and Adler's +8% stands against it.
+constexpr int kTmaBoxR = kRM + 2;                                  // region rows -1 .. 128
+constexpr int kTmaHaloL = kTmaBoxR * kRN * 4;                          // 66 560: centre box [130][128]
+constexpr int kTmaHaloR = kTmaHaloL + ((kTmaBoxR * 16 + 127) / 128) * 128;  // left halo [130][4] (cols -4..-1)
+constexpr int kTmaStageBytes = ((kTmaHaloR + kTmaBoxR * 16 + 127) / 128) * 128;  // right halo [130][4] (128..131)
+constexpr uint32_t kTmaStageTx = kTmaBoxR * (kRN + 8) * 4;                // 70 720 B per region
+
+__host__ __device__ constexpr int stencil_tma_smem(int stages) {
+  return stages * kTmaStageBytes + stages * (2 * 8 + 16 * (int)sizeof(CkRecord)) + 128;
+}
+
+__device__ __forceinline__ float4 lds_v4(uint32_t a) {
+  float4 r;
+  asm volatile("ld.shared.v4.f32 {%0,%1,%2,%3}, [%4];" : "=f"(r.x), "=f"(r.y), "=f"(r.z), "=f"(r.w) : "r"(a));
+  return r;
+}
+__device__ __forceinline__ float lds_f(uint32_t a) {
+  float r;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(r) : "r"(a));
+  return r;
+}
+
+template <uint32_t MASK, int STORE, int NW>
+__global__ void __launch_bounds__((NW + 1) * 32, 1)
+    stencil5_tma_kernel(const __grid_constant__ CUtensorMap tctr, const __grid_constant__ CUtensorMap thalo,
+                        float* __restrict__ out, int64_t ldo, int row_lo, int64_t Q, int64_t R,
+                        uint32_t* __restrict__ ck, int64_t rid_offset, int stages) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + stages * kTmaStageBytes);
+  uint64_t* empty = full + stages;
+  CkRecord* srec = reinterpret_cast<CkRecord*>(empty + stages);  // [stages][NW]
+  constexpr int RW = kRM / NW;  // region rows per consumer warp
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int64_t first = blockIdx.x, stride = gridDim.x;
+  const int64_t niter = first < R ? (R - 1 - first) / stride + 1 : 0;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < stages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], NW);
+    }
+    fence_barrier_init();
+  }
+  __syncthreads();
+
+  if (wid == NW) {  // producer (+ record store)
+    if (lane != 0) return;
+    prefetch_tmap(&tctr);
+    prefetch_tmap(&thalo);
+    auto finish = [&](int64_t it, int s) {
+      if constexpr (MASK != 0) {
+        const int64_t rid = first + it * stride;
+        CkRecord rr = srec[s * NW];
+#pragma unroll
+        for (int w = 1; w < NW; ++w) rr = combine(rr, srec[s * NW + w]);
+        uint32_t words[3];
+        record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
+        store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
+      }
+    };
+    for (int64_t it = 0; it < niter; ++it) {
+      const int s = (int)(it % stages);
+      const uint32_t k = (uint32_t)(it / stages);
+      if (it >= stages) {
+        mbar_wait(&empty[s], (k & 1u) ^ 1u);  // the stage's previous region (it - stages) is consumed
+        finish(it - stages, s);
+      }
+      const int64_t rid = first + it * stride, p = rid / Q, q = rid - p * Q;
+      mbar_expect_tx(&full[s], kTmaStageTx);
+      const int c0 = (int)(q * kRN), r0 = (int)(p * kRM) - 1 - row_lo;
+      uint8_t* dst = smem_raw + s * kTmaStageBytes;
+      // the 128 region columns as one line-aligned box, the 4-column halo strips left and right apart
+      tma_load_2d(&tctr, &full[s], dst, c0, r0);
+      tma_load_2d(&thalo, &full[s], dst + kTmaHaloL, c0 - 4, r0);
+      tma_load_2d(&thalo, &full[s], dst + kTmaHaloR, c0 + kRN, r0);
+    }
+    for (int64_t it = niter > stages ? niter - stages : 0; it < niter; ++it) {
+      const int s = (int)(it % stages);
+      mbar_wait(&empty[s], (uint32_t)(it / stages) & 1u);
+      finish(it, s);
+    }
+    return;
+  }
+
+  // consumers: warp wid owns region rows wid*RW .. wid*RW+RW-1 (box rows +1), lane owns columns lane*4 .. +3
+  const uint32_t sbase = smem_u32(smem_raw);
+  const uint32_t lane_off = (uint32_t)((wid * RW) * kRN * 4 + lane * 16);
+  const uint32_t edge_off = (uint32_t)((lane < 16 ? kTmaHaloL + 12 : kTmaHaloR) + (wid * RW + 1) * 16);
+  for (int64_t it = 0; it < niter; ++it) {
+    const int s = (int)(it % stages);
+    const int64_t rid = first + it * stride, p = rid / Q, q = rid - p * Q;
+    mbar_wait(&full[s], (uint32_t)(it / stages) & 1u);
+    const uint32_t st0 = sbase + (uint32_t)s * kTmaStageBytes;
+    float* orow = out + (p * kRM + wid * RW) * ldo + q * kRN + lane * 4;
+    float4 u = lds_v4(st0 + lane_off), c = lds_v4(st0 + lane_off + kRN * 4);
+    CkPartial<MASK> part;
+    AdlerRows ad;
+#pragma unroll
+    for (int r = 0; r < RW; ++r) {
+      const float4 d = lds_v4(st0 + lane_off + (r + 2) * kRN * 4);
+      const float e = lds_f(st0 + edge_off + r * 16);
+      float left = __shfl_up_sync(0xFFFFFFFFu, c.w, 1);
+      float right = __shfl_down_sync(0xFFFFFFFFu, c.x, 1);
+      if (lane == 0) left = e;
+      if (lane == 31) right = e;
+      float4 o;
+      o.x = st5(c.x, u.x, d.x, left, c.y);
+      o.y = st5(c.y, u.y, d.y, c.x, c.z);
+      o.z = st5(c.z, u.z, d.z, c.y, c.w);
+      o.w = st5(c.w, u.w, d.w, c.z, right);
+      __stcs(reinterpret_cast<float4*>(orow + (int64_t)r * ldo), o);
+      if constexpr (MASK != 0) {
+        add4_modxor(part, __float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
+        if constexpr ((MASK & kAdler) != 0)
+          ad.add_row(__float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
+      }
+      u = c;
+      c = d;
+    }
+    if constexpr (MASK != 0) {
+      if constexpr ((MASK & kAdler) != 0) ad.fold(part, (uint32_t)(wid * RW * kRN * 4 + lane * 16 + 1), RW, kRN * 4);
+      const CkRecord wr = warp_reduce<MASK>(part);
+      if (lane == 0) srec[s * NW + wid] = wr;
+    }
+    __syncwarp();
+    if (lane == 0) mbar_arrive(&empty[s]);
+  }
+}
+
+int stencil_tma_stages() {
+  static int v = [] {
+    const char* e = getenv("LP_STENCIL_STAGES");
+    const int s = e ? atoi(e) : 3;
+    return s < 2 ? 2 : (s > 3 ? 3 : s);
+  }();
+  return v;
+}
+CUtensorMapL2promotion stencil_tma_promo() {
+  static CUtensorMapL2promotion v = [] {
+    const char* e = getenv("LP_STENCIL_PROMO");
+    const int b = e ? atoi(e) : 0;
+    return b == 256 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B
+                    : (b == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
+                                : (b == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B : CU_TENSOR_MAP_L2_PROMOTION_NONE));
+  }();
+  return v;
+}
+int stencil_tma_warps() {
+  static int v = [] {
+    const char* e = getenv("LP_STENCIL_NW");
+    return (e && atoi(e) == 8) ? 8 : 16;
+  }();
+  return v;
+}
+bool stencil_use_tma() {
+  static bool v = [] {
+    const char* e = getenv("LP_STENCIL_TMA");
+    return e ? atoi(e) != 0 : false;
+  }();
+  return v;
+}
+
+cudaError_t launch_stencil_tma(const StencilArgs& a, int64_t Q, int64_t R, cudaStream_t st) {
+  CUtensorMap tm, tt;
+  const int nw = stencil_tma_warps();
+  // rows [row_lo, row_lo + row_span) of the shard, columns [0, W): everything else reads as zero
+  const float* base = a.in + (int64_t)a.row_lo * a.ldi;
+  const CUtensorMapL2promotion promo = stencil_tma_promo();
+  if (!tma_map_2d(&tm, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, base, (uint64_t)a.W, (uint64_t)a.row_span,
+                  (uint64_t)a.ldi, kRN, kTmaBoxR, CU_TENSOR_MAP_SWIZZLE_NONE, promo) ||
+      !tma_map_2d(&tt, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, base, (uint64_t)a.W, (uint64_t)a.row_span,
+                  (uint64_t)a.ldi, 4, kTmaBoxR, CU_TENSOR_MAP_SWIZZLE_NONE, promo))
+    return cudaErrorInvalidValue;
+  const int stages = stencil_tma_stages();
+  const int smem = stencil_tma_smem(stages);
+  int64_t grid = R < a.sm_count ? R : a.sm_count;
+  if (grid < 1) grid = 1;
+  const int sk = a.mask ? a.hash.store : 0;
+  cudaError_t e = cudaSuccess;
+  switch (a.mask * 5 + sk) {
+#define LP_TCASE(M, S)                                                                                       \
+  case M * 5 + S: {                                                                                          \
+    auto kfn = nw == 16 ? stencil5_tma_kernel<M, S, 16> : stencil5_tma_kernel<M, S, 8>;                      \
+    e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                        \
+    if (e != cudaSuccess) return e;                                                                          \
+    kfn<<<(unsigned)grid, (nw + 1) * 32, smem, st>>>(tm, tt, a.out, a.ldo, a.row_lo, Q, R, a.ck, a.rid_offset, \
+                                                     stages);                                                \
+    break;                                                                                                   \
+  }
+#define LP_TCASE3(M) LP_TCASE(M, 0)
+#define LP_TCASE5(M) LP_TCASE(M, 0) LP_TCASE(M, 1) LP_TCASE(M, 2) LP_TCASE(M, 3) LP_TCASE(M, 4)
+    LP_TCASE(0, 0)
+    LP_TCASE5(1)
+    LP_TCASE3(2)
+    LP_TCASE5(3)
+    LP_TCASE3(4)
+    LP_TCASE3(5)
+    LP_TCASE3(6)
+    LP_TCASE3(7)
+#undef LP_TCASE3
+#undef LP_TCASE5
+#undef LP_TCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
 }  // namespace
 
 bool stencil_supported(int RM, int RN) { return RM == kRM && RN == kRN; }
@@ -223,6 +447,7 @@ bool stencil_supported(int RM, int RN) { return RM == kRM && RN == kRN; }
 cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   const int64_t Q = a.W / kRN, R = (a.H / kRM) * Q;
   if (a.H > (int64_t)INT32_MAX / 2 || a.W > (int64_t)INT32_MAX / 2) return cudaErrorInvalidValue;
+  if (!a.list && stencil_use_tma()) return launch_stencil_tma(a, Q, R, st);
   const int sk = a.mask ? a.hash.store : 0;
   // full run: one region per CTA, barrier-free combine; list mode (recovery):
   // persistent CTAs over the failed list, barrier combine (accumulators reused)
