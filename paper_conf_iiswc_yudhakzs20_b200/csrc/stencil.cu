@@ -11,10 +11,15 @@
 // outside the domain.
 //
 // Structure: CTA = one 128x128 region, 8 warps x 16 rows, lane = 4 adjacent
-// columns (one 16-B vector).  Every lane issues all 18 row loads and its 16
-// edge loads up front (non-allocating 16-B loads through volatile PTX), then
+// columns (one 16-B vector).  Every lane issues all 18 row loads and its edge
+// loads up front (non-allocating 16-B loads through volatile PTX), then
 // computes; left/right neighbours come from the adjacent lanes by shuffle;
 // results leave with streaming 16-B stores.  2 CTAs (16 warps) per SM.
+// Protected full runs use the two-phase epilogue: the 16 edge values of a warp
+// are loaded one per lane (lanes 0-15 left, 16-31 right) and broadcast by
+// shuffle, every row is stored first, and the checksum pass runs over the
+// stored vectors afterwards (four Adler accumulator sets); the plain twin keeps
+// per-row edge loads, its fastest form (A/B in profiles/r02/ab_stencil_epilogue.txt).
 //
 // LP epilogue: each lane folds the exact stored words into its checksum
 // partials (L192) and the warp reduces them with redux.sync (Listing 4).  The
@@ -88,15 +93,15 @@ __device__ __forceinline__ float ldg_nc_f(const float* p) {
   return r;
 }
 
-template <uint32_t MASK, int STORE, int COMBINE>
-__global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __restrict__ in, int64_t ldi,
+template <uint32_t MASK, int STORE, int COMBINE, int RWS = 16, int EL = 0>
+__global__ void __launch_bounds__(kRM / RWS * 32, 2) stencil5_ldg_kernel(const float* __restrict__ in, int64_t ldi,
                                                               float* __restrict__ out, int64_t ldo, int row_lo,
                                                               int row_span, int W,
                                                               int64_t Q, int64_t R, uint32_t* __restrict__ ck,
                                                               int64_t rid_offset, const int64_t* __restrict__ list,
                                                               const int64_t* __restrict__ d_n) {
-  constexpr int kRowsW = 16;
-  __shared__ CkRecord warp_rec[8];
+  constexpr int kRowsW = RWS, kNW = kRM / RWS, kNT = kNW * 32;  // rows per warp, warps, threads
+  __shared__ CkRecord warp_rec[kNW];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   __shared__ int s_bad;
   const int64_t ntiles = (list && COMBINE != 2) ? *d_n : R;
@@ -124,7 +129,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       if (threadIdx.x == 0) {
         CkRecord rr = warp_rec[0];
 #pragma unroll
-        for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
+        for (int w = 1; w < kNW; ++w) rr = combine(rr, warp_rec[w]);
         uint32_t words[3];
         record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
         constexpr int S = selem_of(MASK);
@@ -147,14 +152,24 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
     const int je = lane == 0 ? j - 1 : j + 4;
     const bool eok = (lane == 0 || lane == 31) && je >= 0 && je < W;
     float4 v[kRowsW + 2];
-    float edge[kRowsW];
+    constexpr bool kEdgeLanes = (EL & 1) != 0, kTwoPhase = (EL & 2) != 0;
+    float edge[kEdgeLanes ? 1 : kRowsW];
 #pragma unroll
     for (int r = 0; r < kRowsW + 2; ++r) {
       const int i = i0 - 1 + r;
       v[r] = ((unsigned)(i - row_lo) < (unsigned)row_span) ? ldg_nc_v4(in + (int64_t)i * ldi + j) : make_float4(0.f, 0.f, 0.f, 0.f);
     }
 #pragma unroll
-    for (int r = 0; r < kRowsW; ++r) edge[r] = eok ? ldg_nc_f(in + (int64_t)(i0 + r) * ldi + je) : 0.f;
+    if constexpr (kEdgeLanes) {
+      // edge columns by lane: lanes 0..RWS-1 hold the left edge (column q*128-1) of rows 0..RWS-1, lanes
+      // RWS..2*RWS-1 the right edge (column q*128+128); broadcast to lanes 0 / 31 by shuffle per row
+      const int jq = (int)(q * kRN), er = lane % kRowsW;
+      const int jc = lane < kRowsW ? jq - 1 : jq + kRN;
+      edge[0] = (lane < 2 * kRowsW && jc >= 0 && jc < W) ? ldg_nc_f(in + (int64_t)(i0 + er) * ldi + jc) : 0.f;
+    } else {
+#pragma unroll
+      for (int r = 0; r < kRowsW; ++r) edge[r] = eok ? ldg_nc_f(in + (int64_t)(i0 + r) * ldi + je) : 0.f;
+    }
     CkPartial<MASK> part;
     AdlerRows ad;
 #pragma unroll
@@ -162,21 +177,59 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       const float4 u = v[r], c = v[r + 1], d = v[r + 2];
       float left = __shfl_up_sync(0xFFFFFFFFu, c.w, 1);
       float right = __shfl_down_sync(0xFFFFFFFFu, c.x, 1);
-      if (lane == 0) left = edge[r];
-      if (lane == 31) right = edge[r];
+      if constexpr (kEdgeLanes) {
+        const float el = __shfl_sync(0xFFFFFFFFu, edge[0], r), er = __shfl_sync(0xFFFFFFFFu, edge[0], kRowsW + r);
+        if (lane == 0) left = el;
+        if (lane == 31) right = er;
+      } else {
+        if (lane == 0) left = edge[r];
+        if (lane == 31) right = edge[r];
+      }
       float4 o;
       o.x = st5(c.x, u.x, d.x, left, c.y);
       o.y = st5(c.y, u.y, d.y, c.x, c.z);
       o.z = st5(c.z, u.z, d.z, c.y, c.w);
       o.w = st5(c.w, u.w, d.w, c.z, right);
       __stcs(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
-      if constexpr (MASK != 0) {
+      if constexpr (kTwoPhase) {
+        v[r] = o;  // row r's input is dead: keep the stored vector for the checksum pass below
+      } else if constexpr (MASK != 0) {
         add4_modxor(part, __float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
         if constexpr ((MASK & kAdler) != 0)
           ad.add_row(__float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
       }
     }
-    if constexpr ((MASK & kAdler) != 0) ad.fold(part, (uint32_t)(wid * kRowsW * kRN * 4 + lane * 16 + 1), kRowsW, kRN * 4);
+    if constexpr (kTwoPhase && MASK != 0) {
+      // two-phase form: every row's store is issued before the checksum arithmetic starts (the warp
+      // barrier keeps ptxas from hoisting the dp4a chains above the stores)
+      __syncwarp();
+      // Adler with four independent accumulator sets (rows r mod 4) so the dp4a chains overlap; the row
+      // moment is summed directly (R = sum_r r * bs_r = n * S - T of AdlerRows): the same integer sums
+      uint32_t aS[4] = {0, 0, 0, 0}, aR[4] = {0, 0, 0, 0}, aW[4] = {0, 0, 0, 0};
+#pragma unroll
+      for (int r = 0; r < kRowsW; ++r) {
+        const float4 o = v[r];
+        const uint32_t x = __float_as_uint(o.x), y = __float_as_uint(o.y), z = __float_as_uint(o.z),
+                       w = __float_as_uint(o.w);
+        add4_modxor(part, x, y, z, w);
+        if constexpr ((MASK & kAdler) != 0) {
+          const uint32_t bs = (uint32_t)__dp4a(x, 0x01010101u, __dp4a(y, 0x01010101u, 0u)) +
+                              (uint32_t)__dp4a(z, 0x01010101u, __dp4a(w, 0x01010101u, 0u));
+          aS[r & 3] += bs;
+          aR[r & 3] += (uint32_t)r * bs;
+          aW[r & 3] = (uint32_t)__dp4a(x, 0x03020100u, __dp4a(y, 0x07060504u,
+                                       __dp4a(z, 0x0B0A0908u, __dp4a(w, 0x0F0E0D0Cu, aW[r & 3]))));
+        }
+      }
+      if constexpr ((MASK & kAdler) != 0) {
+        const uint32_t S = (aS[0] + aS[1]) + (aS[2] + aS[3]), Rm = (aR[0] + aR[1]) + (aR[2] + aR[3]),
+                       Wl = (aW[0] + aW[1]) + (aW[2] + aW[3]);
+        part.s += S;
+        part.w += (uint64_t)(uint32_t)(wid * kRowsW * kRN * 4 + lane * 16 + 1) * S + (uint64_t)(kRN * 4) * Rm + Wl;
+      }
+    }
+    if constexpr ((MASK & kAdler) != 0 && !kTwoPhase)
+      ad.fold(part, (uint32_t)(wid * kRowsW * kRN * 4 + lane * 16 + 1), kRowsW, kRN * 4);
     if constexpr (MASK != 0 && COMBINE == 1) {
       // split-barrier combine (one region per CTA): every warp parks its partial in shared memory and
       // ARRIVES on named barrier 2 without waiting; only warp 0 waits (bar.sync) and then combines the
@@ -185,13 +238,13 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       const CkRecord wr = warp_reduce<MASK>(part);
       if (lane == 0) warp_rec[wid] = wr;
       if (wid != 0) {
-        asm volatile("bar.arrive 2, 256;" ::: "memory");
+        asm volatile("bar.arrive 2, %0;" ::"n"(kNT) : "memory");
       } else {
-        asm volatile("bar.sync 2, 256;" ::: "memory");
+        asm volatile("bar.sync 2, %0;" ::"n"(kNT) : "memory");
         if (lane == 0) {
           CkRecord rr = warp_rec[0];
 #pragma unroll
-          for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
+          for (int w = 1; w < kNW; ++w) rr = combine(rr, warp_rec[w]);
           uint32_t words[3];
           record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
           store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
@@ -199,8 +252,8 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       }
     } else if constexpr (MASK == 0 && COMBINE == 1 && LP_STENCIL_TWIN_BAR) {
       // the unprotected twin keeps the same split barrier, so the LP overhead compares like with like
-      if (wid != 0) asm volatile("bar.arrive 2, 256;" ::: "memory");
-      else asm volatile("bar.sync 2, 256;" ::: "memory");
+      if (wid != 0) asm volatile("bar.arrive 2, %0;" ::"n"(kNT) : "memory");
+      else asm volatile("bar.sync 2, %0;" ::"n"(kNT) : "memory");
     } else if constexpr (MASK != 0) {
       const CkRecord wr = warp_reduce<MASK>(part);
       __syncthreads();  // warp_rec may still be read by the check phase (COMBINE == 2)
@@ -209,7 +262,7 @@ __global__ void __launch_bounds__(256, 2) stencil5_ldg_kernel(const float* __res
       if (threadIdx.x == 0) {
         CkRecord rr = warp_rec[0];
 #pragma unroll
-        for (int w = 1; w < 8; ++w) rr = combine(rr, warp_rec[w]);
+        for (int w = 1; w < kNW; ++w) rr = combine(rr, warp_rec[w]);
         uint32_t words[3];
         record_words<MASK>(rr, (uint64_t)kRM * kRN * 4, words);
         store_record<MASK, STORE>(ck, rid, (uint32_t)(rid + rid_offset), words);
@@ -386,6 +439,18 @@ int stencil_tma_warps() {
   }();
   return v;
 }
+// full run, LDG form, bit 0: edge columns loaded by lanes and broadcast by shuffle (one register instead
+// of 16), bit 1: two-phase epilogue (every row stored before the checksum pass).  Default: both for the
+// protected kernels (frees the registers the Adler accumulators need and keeps ptxas from scheduling the
+// dp4a chains ahead of the stores: Adler +7% -> +1%, profiles/r02/ab_stencil_epilogue.txt), neither for
+// the unprotected twin (its fastest form, so the LP overhead is measured against the fastest plain kernel).
+int stencil_edge_lanes(uint32_t mask) {
+  static int v = [] {
+    const char* e = getenv("LP_STENCIL_EL");
+    return e ? (atoi(e) == 3 ? 3 : 0) : -1;  // A/B override: 0 or 3 for every kernel
+  }();
+  return v >= 0 ? v : (mask ? 3 : 0);
+}
 bool stencil_use_tma() {
   static bool v = [] {
     const char* e = getenv("LP_STENCIL_TMA");
@@ -460,6 +525,10 @@ cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   case M * 5 + S:                                                                                               \
     if (a.list)                                                                                                 \
       stencil5_ldg_kernel<M, S, 0><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo,          \
+                                                                   a.row_span, (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
+                                                                   a.d_n);                                      \
+    else if (stencil_edge_lanes(a.mask) == 3)                                                                   \
+      stencil5_ldg_kernel<M, S, 1, 16, 3><<<(unsigned)grid, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo,   \
                                                                    a.row_span, (int)a.W, Q, R, a.ck, a.rid_offset, a.list,   \
                                                                    a.d_n);                                      \
     else                                                                                                        \
