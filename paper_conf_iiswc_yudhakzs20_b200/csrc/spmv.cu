@@ -48,6 +48,9 @@ constexpr int kSpWarps = kSpThreads / 32;
 #ifndef LP_SPMV_MINB
 #define LP_SPMV_MINB 5
 #endif
+#ifndef LP_SPMV_EARLY
+#define LP_SPMV_EARLY 0
+#endif
 constexpr int kPerThread = LP_SPMV_PT;               // nnz per thread per chunk (kPerThread / 4 uint4)
 constexpr int kVec = kPerThread / 4;
 constexpr int kChunk = kSpThreads * kPerThread;      // nnz per chunk
@@ -123,6 +126,12 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
     for (int ch = 0; ch < nch; ++ch) {
       const int64_t kc = kbase + (int64_t)ch * kChunk;
       float* pb = prod + (ch & 1) * kChunk;
+#if LP_SPMV_EARLY
+      // the next chunk's (value, column) loads are issued before this chunk's x gathers, so HBM latency
+      // overlaps the gathers, the products and the row phase
+      uint4 vn[kVec], cn[kVec];
+      if (ch + 1 < nch) load_chunk(val, col, kc + kChunk, K0, K1, nnz, vn, cn);
+#endif
       // products of this thread's kPerThread elements (the x gathers are independent of each other);
       // masked lanes (value 0, column 0) read x[0] and store 0, never summed
       float xv[kPerThread];
@@ -141,8 +150,18 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
         p.w = __fmul_rn(__uint_as_float(v[h].w), xv[4 * h + 3]);
         *reinterpret_cast<float4*>(pb + (h * kSpThreads + tid) * 4) = p;
       }
+#if !LP_SPMV_EARLY
       // the next chunk's loads fly while this one is reduced
       if (ch + 1 < nch) load_chunk(val, col, kc + kChunk, K0, K1, nnz, v, c);
+#else
+      if (ch + 1 < nch) {
+#pragma unroll
+        for (int h = 0; h < kVec; ++h) {
+          v[h] = vn[h];
+          c[h] = cn[h];
+        }
+      }
+#endif
       __syncthreads();
       // row phase: rows overlapping [lo, hi) (offsets relative to K0).  A row's products in this
       // chunk are summed in CSR order by its thread when there are <= kLong of them; longer
