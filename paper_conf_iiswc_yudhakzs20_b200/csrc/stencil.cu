@@ -87,9 +87,20 @@ __device__ __forceinline__ float4 ldg_nc_v4(const float* p) {
                : "l"(p));
   return r;
 }
+#ifndef LP_STENCIL_EDGE_LD
+#define LP_STENCIL_EDGE_LD 0
+#endif
 __device__ __forceinline__ float ldg_nc_f(const float* p) {
   float r;
+#if LP_STENCIL_EDGE_LD == 1
+  asm volatile("ld.global.nc.L2::64B.f32 %0, [%1];" : "=f"(r) : "l"(p));
+#elif LP_STENCIL_EDGE_LD == 2
+  asm volatile("ld.global.f32 %0, [%1];" : "=f"(r) : "l"(p));
+#elif LP_STENCIL_EDGE_LD == 3
+  asm volatile("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(r) : "l"(p));
+#else
   asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(r) : "l"(p));
+#endif
   return r;
 }
 
@@ -294,7 +305,7 @@ constexpr int kTmaStageBytes = ((kTmaHaloR + kTmaBoxR * 16 + 127) / 128) * 128; 
 constexpr uint32_t kTmaStageTx = kTmaBoxR * (kRN + 8) * 4;                // 70 720 B per region
 
 __host__ __device__ constexpr int stencil_tma_smem(int stages) {
-  return stages * kTmaStageBytes + stages * (2 * 8 + 16 * (int)sizeof(CkRecord)) + 128;
+  return stages * kTmaStageBytes + stages * (2 * 8 + 16 * (int)sizeof(CkRecord) + 8) + 128;
 }
 
 __device__ __forceinline__ float4 lds_v4(uint32_t a) {
@@ -312,7 +323,8 @@ template <uint32_t MASK, int STORE, int NW>
 __global__ void __launch_bounds__((NW + 1) * 32, 1)
     stencil5_tma_kernel(const __grid_constant__ CUtensorMap tctr, const __grid_constant__ CUtensorMap thalo,
                         float* __restrict__ out, int64_t ldo, int row_lo, int64_t Q, int64_t R,
-                        uint32_t* __restrict__ ck, int64_t rid_offset, int stages) {
+                        uint32_t* __restrict__ ck, int64_t rid_offset, int stages,
+                        const int64_t* __restrict__ list, const int64_t* __restrict__ d_n) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem_raw + stages * kTmaStageBytes);
   uint64_t* empty = full + stages;
@@ -320,7 +332,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1)
   constexpr int RW = kRM / NW;  // region rows per consumer warp
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int64_t first = blockIdx.x, stride = gridDim.x;
-  const int64_t niter = first < R ? (R - 1 - first) / stride + 1 : 0;
+  const int64_t nwork = list ? *d_n : R;  // list mode (recovery): the failed list's entries
+  const int64_t niter = first < nwork ? (nwork - 1 - first) / stride + 1 : 0;
+  int64_t* s_rid = reinterpret_cast<int64_t*>(smem_raw + stencil_tma_smem(stages) - 128 - stages * 8);
   if (threadIdx.x == 0) {
     for (int s = 0; s < stages; ++s) {
       mbar_init(&full[s], 1);
@@ -336,7 +350,7 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1)
     prefetch_tmap(&thalo);
     auto finish = [&](int64_t it, int s) {
       if constexpr (MASK != 0) {
-        const int64_t rid = first + it * stride;
+        const int64_t rid = s_rid[s];
         CkRecord rr = srec[s * NW];
 #pragma unroll
         for (int w = 1; w < NW; ++w) rr = combine(rr, srec[s * NW + w]);
@@ -352,7 +366,9 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1)
         mbar_wait(&empty[s], (k & 1u) ^ 1u);  // the stage's previous region (it - stages) is consumed
         finish(it - stages, s);
       }
-      const int64_t rid = first + it * stride, p = rid / Q, q = rid - p * Q;
+      const int64_t rid = list ? list[first + it * stride] - rid_offset : first + it * stride;
+      const int64_t p = rid / Q, q = rid - p * Q;
+      s_rid[s] = rid;  // published to the consumers by the full barrier's completion
       mbar_expect_tx(&full[s], kTmaStageTx);
       const int c0 = (int)(q * kRN), r0 = (int)(p * kRM) - 1 - row_lo;
       uint8_t* dst = smem_raw + s * kTmaStageBytes;
@@ -375,8 +391,8 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1)
   const uint32_t edge_off = (uint32_t)((lane < 16 ? kTmaHaloL + 12 : kTmaHaloR) + (wid * RW + 1) * 16);
   for (int64_t it = 0; it < niter; ++it) {
     const int s = (int)(it % stages);
-    const int64_t rid = first + it * stride, p = rid / Q, q = rid - p * Q;
     mbar_wait(&full[s], (uint32_t)(it / stages) & 1u);
+    const int64_t rid = s_rid[s], p = rid / Q, q = rid - p * Q;
     const uint32_t st0 = sbase + (uint32_t)s * kTmaStageBytes;
     float* orow = out + (p * kRM + wid * RW) * ldo + q * kRN + lane * 4;
     float4 u = lds_v4(st0 + lane_off), c = lds_v4(st0 + lane_off + kRN * 4);
@@ -425,7 +441,7 @@ int stencil_tma_stages() {
 CUtensorMapL2promotion stencil_tma_promo() {
   static CUtensorMapL2promotion v = [] {
     const char* e = getenv("LP_STENCIL_PROMO");
-    const int b = e ? atoi(e) : 0;
+    const int b = e ? atoi(e) : 64;
     return b == 256 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B
                     : (b == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B
                                 : (b == 64 ? CU_TENSOR_MAP_L2_PROMOTION_L2_64B : CU_TENSOR_MAP_L2_PROMOTION_NONE));
@@ -451,6 +467,16 @@ int stencil_edge_lanes(uint32_t mask) {
   }();
   return v >= 0 ? v : (mask ? 3 : 0);
 }
+// list-mode recovery through the TMA-fed form (default): the producer reads the failed list ahead and keeps
+// two scattered regions in flight per SM; the LDG form re-executes them one region per CTA at a time
+// (232 -> 185 us for 10% of C4, profiles/r02/ab_stencil_tma.txt)
+bool stencil_tma_list() {
+  static bool v = [] {
+    const char* e = getenv("LP_STENCIL_TMA_LIST");
+    return e ? atoi(e) != 0 : true;
+  }();
+  return v;
+}
 bool stencil_use_tma() {
   static bool v = [] {
     const char* e = getenv("LP_STENCIL_TMA");
@@ -472,7 +498,7 @@ cudaError_t launch_stencil_tma(const StencilArgs& a, int64_t Q, int64_t R, cudaS
     return cudaErrorInvalidValue;
   const int stages = stencil_tma_stages();
   const int smem = stencil_tma_smem(stages);
-  int64_t grid = R < a.sm_count ? R : a.sm_count;
+  int64_t grid = (a.list || R >= a.sm_count) ? a.sm_count : R;
   if (grid < 1) grid = 1;
   const int sk = a.mask ? a.hash.store : 0;
   cudaError_t e = cudaSuccess;
@@ -483,7 +509,7 @@ cudaError_t launch_stencil_tma(const StencilArgs& a, int64_t Q, int64_t R, cudaS
     e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);                        \
     if (e != cudaSuccess) return e;                                                                          \
     kfn<<<(unsigned)grid, (nw + 1) * 32, smem, st>>>(tm, tt, a.out, a.ldo, a.row_lo, Q, R, a.ck, a.rid_offset, \
-                                                     stages);                                                \
+                                                     stages, a.list, a.d_n);                                 \
     break;                                                                                                   \
   }
 #define LP_TCASE3(M) LP_TCASE(M, 0)
@@ -512,7 +538,7 @@ bool stencil_supported(int RM, int RN) { return RM == kRM && RN == kRN; }
 cudaError_t launch_stencil(const StencilArgs& a, cudaStream_t st) {
   const int64_t Q = a.W / kRN, R = (a.H / kRM) * Q;
   if (a.H > (int64_t)INT32_MAX / 2 || a.W > (int64_t)INT32_MAX / 2) return cudaErrorInvalidValue;
-  if (!a.list && stencil_use_tma()) return launch_stencil_tma(a, Q, R, st);
+  if (a.list ? stencil_tma_list() : stencil_use_tma()) return launch_stencil_tma(a, Q, R, st);
   const int sk = a.mask ? a.hash.store : 0;
   // full run: one region per CTA, barrier-free combine; list mode (recovery):
   // persistent CTAs over the failed list, barrier combine (accumulators reused)
