@@ -15,6 +15,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "lp_device.cuh"
 #include "lp_internal.h"
@@ -73,7 +74,13 @@ __device__ __forceinline__ uint32_t word_of<int32_t>(int32_t v) { return (uint32
 // SEQ = the paper's "no shuffle" ablation (L343, Table IV "+no"): partials go to
 // shared memory and ONE thread folds all 256 of them sequentially, O(N) instead of
 // the O(log N) warp reduction (L220).
-template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE, bool SEQ = false>
+// RMR x RNR = the LP region.  RMR == BM, RNR == BN: the CTA tile is the region (the paper's TB = region,
+// L181).  Smaller regions (the paper's 32x32, Table V TMM) may tile a 128x128 CTA tile (Reading c10): every
+// thread's UM x UN micro-tile lies inside one region, the region's partials are combined by a segmented xor
+// butterfly inside the warp and a two-warp combine through shared memory, and one record per region is
+// stored -- 16 records per CTA, with the 8x8 register micro-tiles of the 128x128 tile instead of 2x2.
+template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE, bool SEQ = false,
+          int RMR = BM, int RNR = BN>
 __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
                                                             const TIn* __restrict__ B, int64_t ldb,
                                                             TOut* __restrict__ C, int64_t ldc, int64_t K,
@@ -92,7 +99,8 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
 
   __shared__ __align__(16) TA As[2][kBK][BM + 4];
   __shared__ __align__(16) TA Bs[2][kBK][BN + 4];
-  __shared__ CkRecord warp_rec[kThreads / 32];
+  constexpr bool kMulti = RMR != BM || RNR != BN;
+  __shared__ CkRecord warp_rec[kMulti ? (kThreads / 32) * (BN / RNR) : kThreads / 32];
   __shared__ uint32_t seq_part[SEQ ? 4 : 1][SEQ ? kThreads : 1];
 
   const int tid = threadIdx.x;
@@ -180,13 +188,39 @@ __global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restric
           *reinterpret_cast<__nv_bfloat162*>(crow + j) = h;
         }
         if constexpr (MASK != 0) {
-          const uint32_t pos = (uint32_t)(lr * BN * ES + (tx * UN + j) * ES + 1);
+          const uint32_t pos = (uint32_t)((lr % RMR) * RNR * ES + ((tx * UN + j) % RNR) * ES + 1);
           part.add(w0, pos);
           if constexpr (ES == 4) part.add(w1, pos + 4);
         }
       }
     }
-    if constexpr (MASK != 0 && SEQ) {
+    if constexpr (MASK != 0 && kMulti) {
+      // 128x128 tile, 8x8 micro-tiles, 32x32 regions: a warp = 2 rows of threads (ty) x 16 columns (tx); the
+      // 4 x 4 threads of a region are lanes {4a..4a+3} x {+0, +16} of two consecutive warps
+      static_assert(BM == 128 && BN == 128 && UM == 8 && UN == 8 && RMR == 32 && RNR == 32, "one multi-region shape");
+      CkRecord r{part.mod, part.xr, part.s, 0u};
+      if constexpr ((MASK & kAdler) != 0) r.wmod = (uint32_t)(part.w % kAdlerBase);
+#pragma unroll
+      for (int o : {1, 2, 16}) {
+        if constexpr ((MASK & kMod) != 0) r.mod += __shfl_xor_sync(0xFFFFFFFFu, r.mod, o);
+        if constexpr ((MASK & kXor) != 0) r.xr ^= __shfl_xor_sync(0xFFFFFFFFu, r.xr, o);
+        if constexpr ((MASK & kAdler) != 0) {
+          r.s += __shfl_xor_sync(0xFFFFFFFFu, r.s, o);
+          r.wmod += __shfl_xor_sync(0xFFFFFFFFu, r.wmod, o);
+        }
+      }
+      const int lane = tid & 31, warp = tid >> 5;
+      if ((lane & 19) == 0) warp_rec[warp * 4 + (lane >> 2)] = r;  // lanes 0, 4, 8, 12: region column lane / 4
+      __syncthreads();
+      if (tid < 16) {
+        const int ry = tid >> 2, rx = tid & 3;
+        const CkRecord rr = combine(warp_rec[(2 * ry) * 4 + rx], warp_rec[(2 * ry + 1) * 4 + rx]);
+        uint32_t words[3];
+        record_words<MASK>(rr, (uint64_t)RMR * RNR * ES, words);
+        const int64_t rrid = (p * 4 + ry) * (Q * 4) + q * 4 + rx;  // region id in the 32x32 grid
+        store_record<MASK, STORE>(ck, rrid, (uint32_t)(rrid + rid_offset), words);
+      }
+    } else if constexpr (MASK != 0 && SEQ) {
       seq_part[0][tid] = part.mod;
       seq_part[1][tid] = part.xr;
       seq_part[2][tid] = part.s;
@@ -274,8 +308,52 @@ cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// full runs of 32x32 regions on 128x128 CTA tiles (16 regions per tile); list-mode recovery, the no-shuffle
+// ablation and shapes not divisible by 128 keep one CTA per 32x32 region
+template <typename TIn, typename TOut>
+cudaError_t launch_multi32(const TmmArgs& a, cudaStream_t st) {
+  const int64_t Q = a.N / 128, R = (a.M / 128) * Q;
+  const TIn* A = (const TIn*)a.A;
+  const TIn* B = (const TIn*)a.B;
+  TOut* C = (TOut*)a.C;
+  const int sk = a.mask ? a.hash.store : 0;
+  switch (a.mask * 5 + sk) {
+#define LP_MCASE(M, S)                                                                                         \
+  case M * 5 + S:                                                                                              \
+    tmm_simt_kernel<TIn, TOut, 128, 128, 8, 8, M, S, false, 32, 32><<<(unsigned)R, kThreads, 0, st>>>(          \
+        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.rid_offset, nullptr, nullptr);                         \
+    break;
+#define LP_MCASE3(M) LP_MCASE(M, 0)
+#define LP_MCASE5(M) LP_MCASE(M, 0) LP_MCASE(M, 1) LP_MCASE(M, 2) LP_MCASE(M, 3) LP_MCASE(M, 4)
+    LP_MCASE(0, 0)
+    LP_MCASE5(1)
+    LP_MCASE3(2)
+    LP_MCASE5(3)
+    LP_MCASE3(4)
+    LP_MCASE3(5)
+    LP_MCASE3(6)
+    LP_MCASE3(7)
+#undef LP_MCASE3
+#undef LP_MCASE5
+#undef LP_MCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
+}
+
+bool simt_multi32() {
+  static bool v = [] {
+    const char* e = getenv("LP_SIMT_MULTI");
+    return e ? atoi(e) != 0 : true;
+  }();
+  return v;
+}
+
 template <typename TIn, typename TOut>
 cudaError_t launch_shape(const TmmArgs& a, cudaStream_t st) {
+  if (a.RM == 32 && a.RN == 32 && !a.list && !a.no_shuffle && a.M % 128 == 0 && a.N % 128 == 0 && simt_multi32())
+    return launch_multi32<TIn, TOut>(a, st);
   if (a.RM == 32 && a.RN == 32) return launch_mask<TIn, TOut, 32, 32, 2, 2>(a, st);
   if (a.RM == 64 && a.RN == 64) return launch_mask<TIn, TOut, 64, 64, 4, 4>(a, st);
   if (a.RM == 128 && a.RN == 128) return launch_mask<TIn, TOut, 128, 128, 8, 8>(a, st);

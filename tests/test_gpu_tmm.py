@@ -294,6 +294,44 @@ def test_int32_tmm_paper_shape(mask, mode):
     run_cycle(256, 320, 192, 32, 32, "i32", "i32", "int17", mask, "simt", mode=mode, frac=0.1)
 
 
+@pytest.mark.parametrize("in_dt,out_dt,kind", [("i32", "i32", "int17"), ("f32", "f32", "uniform"),
+                                                ("bf16", "bf16", "uniform"), ("bf16", "f32", "int5")])
+@pytest.mark.parametrize("mask", ["mod", "mod|xor", "xor|adler", "mod|xor|adler"])
+def test_simt_multi_region_tile(in_dt, out_dt, kind, mask):
+    """32x32 regions on the SIMT body with M, N % 128 == 0: 16 regions per 128x128 CTA tile (8x8 micro-tiles,
+    segmented butterfly + two-warp combine, Reading c10); recovery re-executes single regions with the
+    one-CTA-per-region kernel, which must reproduce the same bytes and records."""
+    run_cycle(256, 384, 96, 32, 32, in_dt, out_dt, kind, mask, "simt", frac=0.15)
+
+
+@pytest.mark.parametrize("store", ["quad_cas", "quad_lock", "cuckoo"])
+def test_simt_multi_region_tile_hash_stores(store):
+    run_cycle(384, 256, 64, 32, 32, "i32", "i32", "int17", "mod|xor", "simt", store=store, frac=0.1)
+
+
+def test_int32_tmm_paper_4096_tile_forms_agree():
+    """The paper's 4096^2 int TMM: the 128x128-tile body and the one-CTA-per-region body (LP_SIMT_MULTI=0 in a
+    subprocess) store the same bytes and records."""
+    import subprocess, sys, os
+    code = (
+        "import sys, hashlib; sys.path.insert(0, %r)\n"
+        "import torch; from tests.gpu_util import *\n"
+        "from paper_conf_iiswc_yudhakzs20_b200 import lp\n"
+        "A, B = make_inputs(3, 4096, 4096, 4096, 'int17', 'i32')\n"
+        "h = lp.LP(32, 32, cksum='mod|xor|adler', body='simt')\n"
+        "wl = lp.Workload.tmm(host_to_dev(A, 'i32'), host_to_dev(B, 'i32'), out_dtype='i32')\n"
+        "out, ck, *_ = h.alloc(wl); h.cksum_init(wl, ck); h.run_protected(wl, out, ck); torch.cuda.synchronize()\n"
+        "print(hashlib.sha256(dev_to_host(out).tobytes() + dev_to_host(ck).tobytes()).hexdigest())\n"
+    ) % os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    digests = []
+    for multi in ("1", "0"):
+        env = dict(os.environ, LP_SIMT_MULTI=multi)
+        r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=600)
+        assert r.returncode == 0, r.stderr[-2000:]
+        digests.append(r.stdout.strip().splitlines()[-1])
+    assert digests[0] == digests[1]
+
+
 @pytest.mark.parametrize("store", ["quad_cas", "cuckoo", "cuckoo_lock"])
 def test_tf32x3_hash_stores(store):
     run_cycle(512, 512, 128, 128, 128, "f32", "f32", "int5", "mod|xor", "tcgen05", store=store, frac=0.2)
