@@ -38,18 +38,19 @@ def tmm(M, N, K, reg, in_dt, out_dt, body, store="array", shuffle=True, **flags)
     return h, wl, out, ck, stale
 
 
-def stencil(store="array"):
+def stencil(store="array", cksum="mod|xor", shard=False):
     x = torch.empty((512, 384), dtype=torch.float32, device="cuda")
     lpsynth.device_fill(x, 1, "uniform", "f32")
-    h = lp.LP(128, 128, cksum="mod|xor", store=store)
-    wl = lp.Workload.stencil(x)
+    h = lp.LP(128, 128, cksum=cksum, store=store)
+    # shard: rows 128..383 of the 512-row domain (halo rows above and below read, not written)
+    wl = lp.Workload.stencil(x[128:384], row_offset=128, global_m=512) if shard else lp.Workload.stencil(x)
     out, ck, failed, d_n, ws = h.alloc(wl)
     stale = torch.zeros_like(out)
     cycle(h, wl, out, ck, failed, d_n, ws, stale)
     d_rec = torch.zeros(1, dtype=torch.int64, device="cuda")
     h.check_recover(wl, out, ck, d_rec)
     torch.cuda.synchronize()
-    print("ok stencil", store, flush=True)
+    print("ok stencil", store, cksum, shard, flush=True)
 
 
 def spmv():
@@ -111,3 +112,12 @@ _, _, failed2, d_n2, ws2 = h2.alloc(wl2)
 h2.validate(wl2, out2, ck2, failed2, d_n2, ws2)
 torch.cuda.synchronize()
 print("ok nvls emulation", int(cnt[3].item()), flush=True)
+
+
+# round 2 (late): two-phase stencil epilogue with Adler, TMA-fed stencil recovery on a row shard (halo rows
+# through the tensor map's OOB fill), SIMT 32x32 regions on 128x128 CTA tiles with a hash store
+stencil(cksum="mod|xor|adler")
+stencil(shard=True)
+stencil("cuckoo", cksum="mod|xor|adler", shard=True)
+tmm(256, 384, 64, 32, "i32", "i32", "simt", store="quad_cas")
+tmm(256, 384, 64, 32, "bf16", "f32", "simt")
