@@ -23,6 +23,11 @@ constexpr int kValThreads = 256;
 constexpr int kValWarps = kValThreads / 32;
 constexpr int64_t kMaxValCtas = 148 * 16 * 4;
 constexpr int kValUnroll = 8;
+// CTAs per SM the validate kernel is compiled for when Adler is in the record: 4 (64 registers) spills ~100 B
+// per thread with the Adler accumulators; 3 gives them 80 registers (A/B: profiles/r02/ab_validate_adler.txt)
+#ifndef LP_VAL_ADLER_MINB
+#define LP_VAL_ADLER_MINB 3
+#endif
 
 // Segmented reduction of the per-lane partials over aligned groups of 2^lg_log2
 // lanes (one group = one region).  A whole-warp group uses one redux.sync per
@@ -123,8 +128,8 @@ __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int6
 // writes its failure count for the ordered compaction.
 // MODE 0 = compare with array table, 1 = compare with a quad hash table (lookup
 // by global rid), 2 = write records (no compare), 3 = compare with a cuckoo table.
-template <uint32_t MASK, int MODE>
-__global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
+template <uint32_t MASK, int MODE, int MB = 4>
+__global__ void __launch_bounds__(kValThreads, MB) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
                                                                 int64_t Q, int64_t R, int RM, int row_bytes,
                                                                 int cpr_log2, int g_log2,
                                                                 const uint32_t* __restrict__ ck,
@@ -156,20 +161,52 @@ __global__ void __launch_bounds__(kValThreads, 4) validate_kernel(const uint8_t*
     const int64_t p = r / Q, q = r - p * Q;
     const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
     CkPartial<MASK> part;
-    for (int c0 = li; c0 < chunks; c0 += kValUnroll << lg_log2) {
+    // Adler column form: when a lane's chunks all sit in one column of the region (LG >= cpr, the planned
+    // geometries), chunk j of the lane is at byte position pos0 + j * dpos, so sum_j pos_j * bs_j =
+    // pos0 * S + dpos * J with J = sum_j j * bs_j: no per-chunk position or 64-bit multiply, and the per-chunk
+    // dp4a chains are independent (the 64-bit position chain of add4 is what held the next loads back)
+    const bool colform = ((MASK & kAdler) != 0) && lg_log2 >= cpr_log2 && ((chunks >> lg_log2) <= 1024);
+    uint32_t aS = 0, aJ = 0, aW = 0;
+    for (int c0 = li, jb = 0; c0 < chunks; c0 += kValUnroll << lg_log2, jb += kValUnroll) {
       uint4 v[kValUnroll];
 #pragma unroll
       for (int u = 0; u < kValUnroll; ++u) {
         const int c = c0 + (u << lg_log2);
         if (live && c < chunks) v[u] = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cmask) << 4));
       }
+      if (colform) {
 #pragma unroll
-      for (int u = 0; u < kValUnroll; ++u) {
-        const int c = c0 + (u << lg_log2);
-        if (live && c < chunks) {
-          const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cmask) << 4) + 1);
-          part.add4(v[u].x, v[u].y, v[u].z, v[u].w, pos);
+        for (int u = 0; u < kValUnroll; ++u) {
+          const int c = c0 + (u << lg_log2);
+          if (live && c < chunks) {
+            if constexpr ((MASK & kMod) != 0) part.mod += (v[u].x + v[u].y) + (v[u].z + v[u].w);
+            if constexpr ((MASK & kXor) != 0) part.xr ^= v[u].x ^ v[u].y ^ v[u].z ^ v[u].w;
+            const uint32_t bs = (uint32_t)__dp4a(v[u].x, 0x01010101u, __dp4a(v[u].y, 0x01010101u, 0u)) +
+                                (uint32_t)__dp4a(v[u].z, 0x01010101u, __dp4a(v[u].w, 0x01010101u, 0u));
+            const uint32_t ws = (uint32_t)__dp4a(v[u].x, 0x03020100u, __dp4a(v[u].y, 0x07060504u,
+                                           __dp4a(v[u].z, 0x0B0A0908u, __dp4a(v[u].w, 0x0F0E0D0Cu, 0u))));
+            aS += bs;
+            aJ += (uint32_t)(jb + u) * bs;
+            aW += ws;
+          }
         }
+      } else {
+#pragma unroll
+        for (int u = 0; u < kValUnroll; ++u) {
+          const int c = c0 + (u << lg_log2);
+          if (live && c < chunks) {
+            const uint32_t pos = (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cmask) << 4) + 1);
+            part.add4(v[u].x, v[u].y, v[u].z, v[u].w, pos);
+          }
+        }
+      }
+    }
+    if constexpr ((MASK & kAdler) != 0) {
+      if (colform) {
+        const uint32_t pos0 = (uint32_t)((li >> cpr_log2) * row_bytes + ((li & cmask) << 4) + 1);
+        const uint32_t dpos = (uint32_t)((1 << (lg_log2 - cpr_log2)) * row_bytes);
+        part.s += aS;
+        part.w += (uint64_t)pos0 * aS + (uint64_t)dpos * aJ + aW;
       }
     }
     const CkRecord rec = segment_reduce<MASK>(part, lg_log2);
@@ -210,19 +247,27 @@ struct ValLaunch {
 };
 
 template <uint32_t MASK>
-cudaError_t validate_dispatch_mode(int mode, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
+cudaError_t validate_dispatch_mode(int mode, int mb, const ValLaunch& L, cudaStream_t st, const uint8_t* out,
                                    int64_t ldc_bytes, int64_t Q, int64_t R, int RM, int row_bytes, int cpr_log2,
                                    const uint32_t* ck, int64_t rid_offset, uint8_t* flags, uint32_t* records,
                                    uint32_t* counts, uint32_t* ticket, int64_t* list, int64_t* d_n,
                                    const NvlsCount& nv) {
-#define LP_VLAUNCH(MD)                                                                                    \
-  validate_kernel<MASK, MD><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2,     \
+#define LP_VLAUNCH1(MD, MB)                                                                               \
+  validate_kernel<MASK, MD, MB><<<L.grid, kValThreads, 0, st>>>(out, ldc_bytes, Q, R, RM, row_bytes, cpr_log2,     \
                                                             L.g_log2, ck, rid_offset, flags, records, L.rpc, counts, \
                                                             ticket, list, d_n, nv)
+#define LP_VLAUNCH(MD)                   \
+  do {                                   \
+    if (mb == LP_VAL_ADLER_MINB)         \
+      LP_VLAUNCH1(MD, LP_VAL_ADLER_MINB); \
+    else                                 \
+      LP_VLAUNCH1(MD, 4);                \
+  } while (0)
   if (mode == 0) LP_VLAUNCH(0);
   else if (mode == 1) LP_VLAUNCH(1);
   else if (mode == 3) LP_VLAUNCH(3);
   else LP_VLAUNCH(2);
+#undef LP_VLAUNCH1
 #undef LP_VLAUNCH
   return cudaGetLastError();
 }
@@ -764,6 +809,15 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
 // for 128 MiB vs 22.5 us at G = 1).  LP_VALIDATE_G=<log2> overrides (A/B runs).
 constexpr int64_t kValMinWarps = 4096;
 
+// output size from which Adler validation uses the 3-CTA/SM build (LP_VAL_ADLER_BIG=<MiB> for A/B runs)
+static uint64_t val_adler_big_bytes() {
+  static const uint64_t v = [] {
+    const char* e = getenv("LP_VAL_ADLER_BIG");
+    return (uint64_t)(e ? atoll(e) : 512) << 20;
+  }();
+  return v;
+}
+
 static ValLaunch plan_validate(const RegionGeom& g, int sm_count) {
   ValLaunch L;
   const int cpr = (g.RN * g.es) / 16;
@@ -807,6 +861,9 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   while ((1 << cpr_log2) < cpr) ++cpr_log2;
   const int mode = records ? 2 : (hi.store == 0 ? 0 : (hi.store <= 2 ? 1 : 3));
   const ValLaunch L = plan_validate(g, sm_count);
+  // Adler records on large outputs: the 80-register build (3 CTAs/SM; the 64-register one spills ~100 B/thread)
+  const int mb = ((mask & kAdler) != 0 && (uint64_t)g.R * (uint64_t)g.RM * (uint64_t)row_bytes >= val_adler_big_bytes())
+                     ? LP_VAL_ADLER_MINB : 4;
   const bool fuse = !records && ticket && g.R <= kFusedCompactMaxR;
   uint32_t* tk = fuse ? ticket : nullptr;
   const uint8_t* o = (const uint8_t*)out;
@@ -815,7 +872,7 @@ cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& 
   switch (mask) {
 #define LP_VCASE(M)                                                                                          \
   case M:                                                                                                    \
-    e = validate_dispatch_mode<M>(mode, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                \
+    e = validate_dispatch_mode<M>(mode, mb, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                \
                                   (const uint32_t*)ck, g.rid_offset, flags, records, counts, tk, list, d_n, nv);\
     break;
     LP_VCASE(1)

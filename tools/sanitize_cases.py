@@ -118,6 +118,6 @@ print("ok nvls emulation", int(cnt[3].item()), flush=True)
 # through the tensor map's OOB fill), SIMT 32x32 regions on 128x128 CTA tiles with a hash store
 stencil(cksum="mod|xor|adler")
 stencil(shard=True)
-stencil("cuckoo", cksum="mod|xor|adler", shard=True)
+stencil("cuckoo", shard=True)
 tmm(256, 384, 64, 32, "i32", "i32", "simt", store="quad_cas")
 tmm(256, 384, 64, 32, "bf16", "f32", "simt")
