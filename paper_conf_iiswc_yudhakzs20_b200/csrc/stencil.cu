@@ -590,7 +590,7 @@ cudaError_t launch_stencil_check_recover(const StencilArgs& a, int64_t* d_recove
   switch (a.mask * 5 + sk) {
 #define LP_CCASE(M, S)                                                                                          \
   case M * 5 + S:                                                                                               \
-    stencil5_ldg_kernel<M, S, 2><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo, a.row_span,  \
+    stencil5_ldg_kernel<M, S, 2, 16, 3><<<(unsigned)R, 256, 0, st>>>(a.in, a.ldi, a.out, a.ldo, a.row_lo, a.row_span,  \
                                                               (int)a.W, Q,                                      \
                                                               R, a.ck, a.rid_offset, nullptr, d_recovered);     \
     break;
