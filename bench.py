@@ -335,19 +335,32 @@ def run_ours(args):
         wl = lp.Workload.tmm(a, b, out_dtype=W["out_dt"], row_offset=sh.row_offset, global_m=gM)
         body_flops = 2.0 * M * N * K
     elif W["kind"] == "spmv":
+        # weak scaling: a (M * world)-row square banded matrix, rank g owns rows [g * M, (g + 1) * M) in whole
+        # regions (row band, like the TMM / stencil shards), x (all columns) generated on every rank from the
+        # counter formula; the rank's CSR slice keeps the global 4-element alignment (shard.csr_band)
         from lpsynth import csr
-        gM = W["M"]
-        if world > 1:
-            raise SystemExit("spmv workload is single-GPU in this round")
-        sh = shard.plan(gM // RN, RN, 1, RN, 1, 0)   # y viewed as [M / RN][RN]
-        M, N, K = W["M"], W["N"], 0
-        rp_d, cols_d, vals_d = lpsynth.device_csr(31, 32, 33, M, N, "uniform")
+        gM = W["M"] * (world if W["weak"] else 1)
+        N, K = gM, 0
+        sh0 = shard.plan(gM // RN, RN, 1, RN, world, rank)          # y viewed as [gM / RN][RN]
+        sh = shard.Shard(rank, world, sh0.row_offset * RN, sh0.rows * RN, sh0.rid_offset, sh0.regions)
+        M = sh.rows
+        rp_g = csr.row_ptr(31, sh.row_offset + M)
+        g0, rp_host, nnz_l, pad = shard.csr_band(rp_g, sh.row_offset, M)
+        rp_d = torch.from_numpy(rp_host).to(dev)
+        cols_d = torch.zeros(nnz_l, dtype=torch.int32, device=dev)
+        vals_d = torch.zeros((nnz_l, 1), dtype=torch.float32, device=dev)
+        rp_abs = torch.from_numpy(rp_g[sh.row_offset:sh.row_offset + M + 1]).to(dev)
+        rc = lpsynth.lib().synth_csr_cols(rp_abs.data_ptr(), M, sh.row_offset, N, 32, cols_d.data_ptr() + 4 * pad,
+                                          torch.cuda.current_stream().cuda_stream)
+        if rc != 0:
+            raise RuntimeError(f"synth_csr_cols rc={rc}")
+        lpsynth.device_fill(vals_d, 33, "uniform", "f32", row0=g0, ncols_global=1)   # counter = global nnz index
+        vals_d = vals_d.view(-1)
         x_d = torch.empty((1, N), dtype=torch.float32, device=dev)
         lpsynth.device_fill(x_d, 34, "uniform", "f32")
-        rp_host = csr.row_ptr(31, M)
         a, b = vals_d, x_d.view(-1)
-        wl = lp.Workload.spmv(vals_d, x_d.view(-1), rp_d, cols_d)
-        body_flops = 2.0 * float(rp_host[-1])
+        wl = lp.Workload.spmv(vals_d, x_d.view(-1), rp_d, cols_d, row_offset=sh.row_offset, global_m=gM)
+        body_flops = 2.0 * float(rp_host[-1] - rp_host[0])
     else:
         # row band of a (M * world) x N domain; the band's input keeps its halo rows (the neighbouring ranks'
         # boundary rows of the read-only input, generated here from the same counter formula: no exchange)
@@ -676,7 +689,7 @@ def run_ours(args):
     if rank == 0:
         launches = args.steps * kernels_per_step(W, W["store"], R)
         if W["kind"] == "spmv":
-            nnz = float(rp_host[-1])
+            nnz = float(rp_host[-1] - rp_host[0])
             sb = nnz * 8 + (M + 1) * 8 + N * 4 + M * 4
             achieved = sb / (t_prot * 1e-3) / 1e9
             roof = {"bound": "hbm", "kernel": f"spmv_kernel (protected, {W['cksum']})", "achieved": round(achieved, 1),
@@ -977,7 +990,8 @@ def run_reference(args):
 
 def recovery_desc(args, RM, W):
     if W["kind"] == "stencil":
-        return "failed 128x128 regions re-executed in list mode by persistent CTAs (one region per CTA pass)"
+        return ("failed 128x128 regions re-executed in list mode by one persistent TMA-fed CTA per SM (producer warp "
+                "reads the failed list ahead, 3-stage ring of halo tiles)")
     if W["kind"] == "spmv" or W.get("body") == "simt":
         return "failed regions re-executed in list mode (one region per CTA pass)"
     if args.no_pairing:

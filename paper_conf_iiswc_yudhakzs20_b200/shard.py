@@ -37,6 +37,23 @@ def plan(global_m: int, n: int, region_m: int, region_n: int, world: int, rank: 
     return Shard(rank, world, lo * region_m, (hi - lo) * region_m, lo * Q, (hi - lo) * Q)
 
 
+def csr_band(rp_global, row0: int, rows: int):
+    """A rank's slice of a CSR matrix for SpMV row-band shards: rows [row0, row0 + rows) with global row_ptr
+    rp_global (int64, at least row0 + rows + 1 entries).  The rank's value / column arrays start at global nnz
+    index g0 = rp_global[row0] rounded down to a multiple of 4 (up to 3 leading elements of the previous row,
+    never summed), so every region's 16-B vector and 2048-nnz chunk grid (Reading R25) sit exactly where they
+    sit in the unsharded matrix: the sharded product is bit-identical to the single-GPU one.
+    Returns (g0, local row_ptr = rp_global[row0 : row0 + rows + 1] - g0, local nnz = rp[-1] - g0, pad)."""
+    import numpy as np
+
+    sl = np.asarray(rp_global[row0:row0 + rows + 1], dtype=np.int64)
+    if len(sl) != rows + 1:
+        raise ValueError("row_ptr too short for the band")
+    g0 = int(sl[0]) & ~3
+    local = sl - g0
+    return g0, local, int(local[-1]), int(sl[0]) - g0
+
+
 def allreduce_counts(counts, group=None):
     """SUM all-reduce of the device int64 count vector (the one collective of the path)."""
     import torch.distributed as dist

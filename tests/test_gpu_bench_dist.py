@@ -76,3 +76,19 @@ def test_inject_skips_rids_of_other_shards():
     h.validate(wl, out, ck, failed, d_n, ws)
     torch.cuda.synchronize()
     assert int(d_n.item()) == 1 and int(failed[0].item()) == 9
+
+
+def test_two_rank_spmv_bench_same_device():
+    """SpMV row-band shards (strong scaling of the 4 Mi-row matrix over 2 ranks, 4-aligned CSR slices)."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", "29543", "bench.py", "--gpus", "2", "--steps", "2",
+           "--warmup", "3", "--overhead-reps", "2", "--no-cpu-baseline", "--dist-backend", "gloo", "--same-device",
+           "--workload", "spmv4m"]
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["n_failed_after_recover"] == 0
+    assert d["config"]["regions_per_rank"] == 4194304 // 1024 // 2
+    assert d["n_failed_per_step"] == 2 * round(0.10 * 2048)

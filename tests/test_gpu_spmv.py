@@ -159,3 +159,39 @@ def test_spmv_invalid_region_shape(RM, RN):
     wl = lp.Workload.spmv(None, x, None, None, m=RN * 8)
     with pytest.raises(lp.LPError):
         h.num_regions(wl)
+
+
+@pytest.mark.parametrize("row0_regions", [1, 3])
+def test_spmv_row_band_shard_bit_identical(row0_regions):
+    """SpMV row-band shard (bench --gpus N): the rank's value / column arrays start at the 4-aligned global nnz
+    index below its first row (shard.csr_band), so the shard's y words and records are bit-identical to the
+    same rows of the unsharded run (the 2048-nnz chunk grid and 16-B vectors sit where they sit globally)."""
+    from paper_conf_iiswc_yudhakzs20_b200 import shard
+
+    RN, rows_all = 256, 256 * 6
+    rp, cols, vals, x = synth(rows_all, rows_all)
+    h = lp.LP(1, RN, cksum="mod|xor|adler")
+    # full matrix
+    wl = lp.Workload.spmv(torch.from_numpy(vals).cuda(), torch.from_numpy(x).cuda(), torch.from_numpy(rp).cuda(),
+                          torch.from_numpy(cols).cuda())
+    y_full, ck_full, *_ = h.alloc(wl)
+    h.cksum_init(wl, ck_full)
+    h.run_protected(wl, y_full, ck_full)
+    # the band of rows [row0, row0 + 2 regions) with rebased, 4-aligned arrays
+    row0, rows = RN * row0_regions, 2 * RN
+    g0, rp_l, nnz_l, pad = shard.csr_band(rp, row0, rows)
+    assert g0 % 4 == 0 and 0 <= pad < 4 and rp_l[0] == pad
+    wls = lp.Workload.spmv(torch.from_numpy(vals[g0:g0 + nnz_l].copy()).cuda(), torch.from_numpy(x).cuda(),
+                           torch.from_numpy(rp_l).cuda(), torch.from_numpy(cols[g0:g0 + nnz_l].copy()).cuda(),
+                           row_offset=row0, global_m=rows_all)
+    y_s, ck_s, *_ = h.alloc(wls)
+    h.cksum_init(wls, ck_s)
+    h.run_protected(wls, y_s, ck_s)
+    torch.cuda.synchronize()
+    yf = dev_to_host(y_full).reshape(-1).view(np.uint32)
+    ys = dev_to_host(y_s).reshape(-1).view(np.uint32)
+    assert np.array_equal(ys, yf[row0:row0 + rows])
+    sel = oracle.selem(h.mask)
+    cf = dev_to_host(ck_full)[:(rows_all // RN) * sel].reshape(-1, sel)
+    cs = dev_to_host(ck_s)[:(rows // RN) * sel].reshape(-1, sel)
+    assert np.array_equal(cs, cf[row0 // RN:(row0 + rows) // RN])

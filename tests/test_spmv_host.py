@@ -87,3 +87,17 @@ def test_csr_deterministic(seed):
     rp1, c1, v1, x1 = _matrix(700, 900, seed=seed)
     rp2, c2, v2, x2 = _matrix(700, 900, seed=seed)
     assert np.array_equal(rp1, rp2) and np.array_equal(c1, c2) and np.array_equal(v1, v2) and np.array_equal(x1, x2)
+
+
+def test_csr_band_alignment_and_rebase():
+    """shard.csr_band: 4-aligned global start, rebased row_ptr with the same row lengths, pad < 4."""
+    from paper_conf_iiswc_yudhakzs20_b200 import shard
+
+    rp = csr.row_ptr(31, 5000)
+    for row0, rows in [(0, 5000), (1024, 2048), (1, 7), (4999, 1)]:
+        g0, local, nnz, pad = shard.csr_band(rp, row0, rows)
+        assert g0 % 4 == 0 and 0 <= pad < 4 and g0 + pad == rp[row0]
+        assert np.array_equal(np.diff(local), np.diff(rp[row0:row0 + rows + 1]))
+        assert local[0] == pad and nnz == rp[row0 + rows] - g0
+        # the chunk grid of every row's region start: (K0 & ~3) relative to the array is the same globally
+        assert all(((int(rp[r]) & ~3) - g0) == (int(local[r - row0]) & ~3) for r in range(row0, row0 + rows))
