@@ -40,8 +40,16 @@ constexpr int kFBK = 32;                          // 32 fp32 = 128 B = one swizz
 constexpr int kFUmmaK = 8;                        // K per tcgen05.mma kind::tf32
 constexpr int kFRawStages = 3;                    // TMA ring
 constexpr int kFCvStages = 2;                     // converted ring
-constexpr int kFThreads = 320;                    // TMA, MMA, 4 epilogue, 4 converter warps
+#ifndef LP_TF32_CONV_WARPS
+#define LP_TF32_CONV_WARPS 8
+#endif
+#ifndef LP_TF32_BLOOP
+#define LP_TF32_BLOOP 0
+#endif
+constexpr int kFConvWarps = LP_TF32_CONV_WARPS;   // converter warps per CTA (4: one column of B per thread)
+constexpr int kFConvThreads = kFConvWarps * 32;
 constexpr int kFConvWarp0 = 6;
+constexpr int kFThreads = (kFConvWarp0 + kFConvWarps) * 32;  // TMA, MMA, 4 epilogue, converter warps
 constexpr int kFTile = 16384;                     // one 128 x 32 fp32 operand tile
 constexpr int kFRawBytes = 2 * kFTile;            // raw stage: [A (K-major)][B (MN-major, 4 x 32-col chunks)]
 constexpr int kFCvBytes = 4 * kFTile;             // converted stage: [A_hi][A_lo][B_hi][B_lo], all K-major SW128
@@ -119,10 +127,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
     prefetch_tmap(&tmap_b);
     for (int s = 0; s < kFRawStages; ++s) {
       mbar_init(&raw_full[s], 1);   // this CTA's TMA bytes
-      mbar_init(&raw_empty[s], 4);  // this CTA's 4 converter warps
+      mbar_init(&raw_empty[s], kFConvWarps);  // this CTA's converter warps
     }
     for (int s = 0; s < kFCvStages; ++s) {
-      mbar_init(&cv_full[s], 8);    // 4 converter warps x 2 CTAs (used in rank 0)
+      mbar_init(&cv_full[s], 2 * kFConvWarps);  // converter warps x 2 CTAs (used in rank 0)
       mbar_init(&cv_empty[s], 1);   // leader's MMA commit (multicast)
     }
     for (int s = 0; s < 2; ++s) {
@@ -169,7 +177,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
     }
   } else if (warp >= kFConvWarp0) {
     // ===================== converters: raw -> [A_hi|A_lo|B_hi|B_lo] =====================
-    const int ct = threadIdx.x - kFConvWarp0 * 32;  // 0..127
+    const int ct = threadIdx.x - kFConvWarp0 * 32;  // 0 .. kFConvThreads - 1
     int rs = 0, cs = 0;
     uint32_t rphase = 0, cphase = 0;
     for (int64_t t = pair; t < ntiles; t += npairs) {
@@ -180,7 +188,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
         uint8_t* cv = cvs(cs);
         // A: K-major SW128 in and out -> element-wise over 1024 16-B units
 #pragma unroll 4
-        for (int i = ct; i < kFTile / 16; i += 128) {
+        for (int i = ct; i < kFTile / 16; i += kFConvThreads) {
           const float4 x = *reinterpret_cast<const float4*>(r + i * 16);
           float4 hi, lo;
           hi.x = __uint_as_float(__float_as_uint(x.x) & 0xFFFFE000u);
@@ -196,15 +204,25 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
         }
         // B: raw MN-major (chunk c = n/32 holds 32 K-rows x 32 columns, 16-B unit u of
         // row k stored at u ^ (k & 7)) -> K-major SW128 rows n (K quad j at j ^ (n & 7)).
-        // Thread ct owns column n = ct; lanes of a warp read 32 consecutive columns of
-        // one K row (conflict-free) and write 16-B units (optimal wavefronts).
+        // Unit u = (column n = u % 128, K quad j = u / 128): the lanes of a warp read 32 consecutive columns
+        // of one K row (conflict-free) and write 16-B units (optimal wavefronts).
         {
-          const int n = ct, c = n >> 5, l = n & 31;
-          const uint8_t* rb = r + kFTile + c * (kFBK * 128) + (l & 3) * 4;
-          uint8_t* bhi = cv + 2 * kFTile + n * 128;
-          uint8_t* blo = cv + 3 * kFTile + n * 128;
+          // units (column n, K quad j): 128 x 8 per stage, strided over the converter threads
+          // (LP_TF32_BLOOP=0: each thread takes consecutive K quads of one column, for 128 | 256 | 512 threads)
+#if LP_TF32_BLOOP == 0
+          constexpr int kJPer = (kFBK / 4) * 128 / kFConvThreads;
+          static_assert(kJPer * kFConvThreads == (kFBK / 4) * 128, "column form needs 128, 256 or 512 threads");
 #pragma unroll
-          for (int j = 0; j < kFBK / 4; ++j) {
+          for (int jj = 0; jj < kJPer; ++jj) {
+            const int n = ct & 127, j = (ct >> 7) * kJPer + jj, c = n >> 5, l = n & 31;
+#else
+#pragma unroll 2
+          for (int u = ct; u < 128 * (kFBK / 4); u += kFConvThreads) {
+            const int n = u & 127, j = u >> 7, c = n >> 5, l = n & 31;
+#endif
+            const uint8_t* rb = r + kFTile + c * (kFBK * 128) + (l & 3) * 4;
+            uint8_t* bhi = cv + 2 * kFTile + n * 128;
+            uint8_t* blo = cv + 3 * kFTile + n * 128;
             float xv[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
