@@ -24,6 +24,10 @@ namespace lp {
 namespace {
 
 constexpr int kThreads = 256;
+// CTAs per SM the 128x128-tile builds are compiled for (1: ptxas takes ~240 registers; 2: <= 128)
+#ifndef LP_SIMT_MINB
+#define LP_SIMT_MINB 2
+#endif
 constexpr int kBK = 16;
 
 // compute type: fp32 for float / bf16 operands (FFMA), int32 for the paper's int TMM (IMAD, wrapping)
@@ -81,7 +85,7 @@ __device__ __forceinline__ uint32_t word_of<int32_t>(int32_t v) { return (uint32
 // stored -- 16 records per CTA, with the 8x8 register micro-tiles of the 128x128 tile instead of 2x2.
 template <typename TIn, typename TOut, int BM, int BN, int UM, int UN, uint32_t MASK, int STORE, bool SEQ = false,
           int RMR = BM, int RNR = BN>
-__global__ void __launch_bounds__(kThreads) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
+__global__ void __launch_bounds__(kThreads, (BM * BN >= 128 * 128) ? LP_SIMT_MINB : 1) tmm_simt_kernel(const TIn* __restrict__ A, int64_t lda,
                                                             const TIn* __restrict__ B, int64_t ldb,
                                                             TOut* __restrict__ C, int64_t ldc, int64_t K,
                                                             int64_t Q, int64_t R, uint32_t* __restrict__ ck,
