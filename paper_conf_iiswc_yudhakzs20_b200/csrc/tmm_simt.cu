@@ -198,7 +198,32 @@ __global__ void __launch_bounds__(kThreads, (BM * BN >= 128 * 128) ? LP_SIMT_MIN
         }
       }
     }
-    if constexpr (MASK != 0 && kMulti) {
+    if constexpr (MASK != 0 && kMulti && SEQ) {
+      // the no-shuffle ablation (L343) on the multi-region tile: every thread parks its partials in shared
+      // memory and ONE thread per region folds its region's 16 threads' partials sequentially
+      static_assert(BM == 128 && BN == 128 && UM == 8 && UN == 8 && RMR == 32 && RNR == 32, "one multi-region shape");
+      seq_part[0][tid] = part.mod;
+      seq_part[1][tid] = part.xr;
+      seq_part[2][tid] = part.s;
+      seq_part[3][tid] = (uint32_t)(part.w % kAdlerBase);
+      __syncthreads();
+      if (tid < 16) {
+        const int ry = tid >> 2, rx = tid & 3;
+        CkRecord rr{0u, 0u, 0u, 0u};
+        for (int ty2 = 4 * ry; ty2 < 4 * ry + 4; ++ty2)
+          for (int tx2 = 4 * rx; tx2 < 4 * rx + 4; ++tx2) {
+            const int j = ty2 * 16 + tx2;
+            rr.mod += seq_part[0][j];
+            rr.xr ^= seq_part[1][j];
+            rr.s += seq_part[2][j];
+            rr.wmod = (rr.wmod + seq_part[3][j]) % kAdlerBase;
+          }
+        uint32_t words[3];
+        record_words<MASK>(rr, (uint64_t)RMR * RNR * ES, words);
+        const int64_t rrid = (p * 4 + ry) * (Q * 4) + q * 4 + rx;
+        store_record<MASK, STORE>(ck, rrid, (uint32_t)(rrid + rid_offset), words);
+      }
+    } else if constexpr (MASK != 0 && kMulti) {
       // 128x128 tile, 8x8 micro-tiles, 32x32 regions: a warp = 2 rows of threads (ty) x 16 columns (tx); the
       // 4 x 4 threads of a region are lanes {4a..4a+3} x {+0, +16} of two consecutive warps
       static_assert(BM == 128 && BN == 128 && UM == 8 && UN == 8 && RMR == 32 && RNR == 32, "one multi-region shape");
@@ -312,8 +337,8 @@ cudaError_t launch_mask(const TmmArgs& a, cudaStream_t st) {
   return cudaGetLastError();
 }
 
-// full runs of 32x32 regions on 128x128 CTA tiles (16 regions per tile); list-mode recovery, the no-shuffle
-// ablation and shapes not divisible by 128 keep one CTA per 32x32 region
+// full runs of 32x32 regions on 128x128 CTA tiles (16 regions per tile; the no-shuffle ablation too);
+// list-mode recovery and shapes not divisible by 128 keep one CTA per 32x32 region
 template <typename TIn, typename TOut>
 cudaError_t launch_multi32(const TmmArgs& a, cudaStream_t st) {
   const int64_t Q = a.N / 128, R = (a.M / 128) * Q;
@@ -321,6 +346,25 @@ cudaError_t launch_multi32(const TmmArgs& a, cudaStream_t st) {
   const TIn* B = (const TIn*)a.B;
   TOut* C = (TOut*)a.C;
   const int sk = a.mask ? a.hash.store : 0;
+  if (a.no_shuffle) {
+    if (a.mask != 3) return cudaErrorInvalidValue;  // the ablation is built for MOD|XOR (Table IV)
+    switch (sk) {
+#define LP_MQCASE(S)                                                                                           \
+  case S:                                                                                                      \
+    tmm_simt_kernel<TIn, TOut, 128, 128, 8, 8, 3, S, true, 32, 32><<<(unsigned)R, kThreads, 0, st>>>(           \
+        A, a.lda, B, a.ldb, C, a.ldc, a.K, Q, R, a.ck, a.rid_offset, nullptr, nullptr);                         \
+    break;
+      LP_MQCASE(0)
+      LP_MQCASE(1)
+      LP_MQCASE(2)
+      LP_MQCASE(3)
+      LP_MQCASE(4)
+#undef LP_MQCASE
+      default:
+        return cudaErrorInvalidValue;
+    }
+    return cudaGetLastError();
+  }
   switch (a.mask * 5 + sk) {
 #define LP_MCASE(M, S)                                                                                         \
   case M * 5 + S:                                                                                              \
@@ -356,7 +400,7 @@ bool simt_multi32() {
 
 template <typename TIn, typename TOut>
 cudaError_t launch_shape(const TmmArgs& a, cudaStream_t st) {
-  if (a.RM == 32 && a.RN == 32 && !a.list && !a.no_shuffle && a.M % 128 == 0 && a.N % 128 == 0 && simt_multi32())
+  if (a.RM == 32 && a.RN == 32 && !a.list && a.M % 128 == 0 && a.N % 128 == 0 && simt_multi32())
     return launch_multi32<TIn, TOut>(a, st);
   if (a.RM == 32 && a.RN == 32) return launch_mask<TIn, TOut, 32, 32, 2, 2>(a, st);
   if (a.RM == 64 && a.RN == 64) return launch_mask<TIn, TOut, 64, 64, 4, 4>(a, st);
