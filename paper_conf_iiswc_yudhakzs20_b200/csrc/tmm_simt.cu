@@ -19,6 +19,7 @@
 
 #include "lp_device.cuh"
 #include "lp_internal.h"
+#include "lp_ptx.cuh"
 
 namespace lp {
 namespace {
@@ -27,6 +28,9 @@ constexpr int kThreads = 256;
 // CTAs per SM the 128x128-tile builds are compiled for (1: ptxas takes ~240 registers; 2: <= 128)
 #ifndef LP_SIMT_MINB
 #define LP_SIMT_MINB 2
+#endif
+#ifndef LP_SIMT_ASYNC
+#define LP_SIMT_ASYNC 1
 #endif
 constexpr int kBK = 16;
 
@@ -122,7 +126,27 @@ __global__ void __launch_bounds__(kThreads, (BM * BN >= 128 * 128) ? LP_SIMT_MIN
 #pragma unroll
       for (int j = 0; j < UN; ++j) acc[i][j] = TA(0);
 
-    TA ra[A_PER], rb[B_PER];
+    // 4-byte operands that need no conversion (fp32, int32) go global -> shared with cp.async (no register
+    // staging: the 128x128 builds then fit 2 CTAs/SM without spills); bf16 is converted through registers
+    constexpr bool kAsync = sizeof(TIn) == 4 && LP_SIMT_ASYNC;
+    auto aload = [&](int64_t k0, int buf) {
+#pragma unroll
+      for (int i = 0; i < A_PER; ++i) {
+        const int e = tid + i * kThreads;
+        const int m = e / kBK, k = e % kBK;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(&As[buf][k][m])),
+                     "l"(A + (row0 + m) * lda + k0 + k) : "memory");
+      }
+#pragma unroll
+      for (int i = 0; i < B_PER; ++i) {
+        const int e = tid + i * kThreads;
+        const int k = e / BN, n = e % BN;
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(&Bs[buf][k][n])),
+                     "l"(B + (k0 + k) * ldb + col0 + n) : "memory");
+      }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    TA ra[kAsync ? 1 : A_PER], rb[kAsync ? 1 : B_PER];
     auto gload = [&](int64_t k0) {
 #pragma unroll
       for (int i = 0; i < A_PER; ++i) {
@@ -151,13 +175,22 @@ __global__ void __launch_bounds__(kThreads, (BM * BN >= 128 * 128) ? LP_SIMT_MIN
     };
 
     __syncthreads();  // previous tile's smem readers are done
-    gload(0);
-    sstore(0);
+    if constexpr (kAsync) {
+      aload(0, 0);
+      asm volatile("cp.async.wait_all;" ::: "memory");
+    } else {
+      gload(0);
+      sstore(0);
+    }
     __syncthreads();
     const int64_t nk = K / kBK;
     for (int64_t kt = 0; kt < nk; ++kt) {
       const int buf = (int)(kt & 1);
-      if (kt + 1 < nk) gload((kt + 1) * kBK);
+      if constexpr (kAsync) {
+        if (kt + 1 < nk) aload((kt + 1) * kBK, buf ^ 1);  // buf ^ 1 was released by the previous barrier
+      } else {
+        if (kt + 1 < nk) gload((kt + 1) * kBK);
+      }
 #pragma unroll
       for (int k = 0; k < kBK; ++k) {
         TA a[UM], b[UN];
@@ -168,7 +201,11 @@ __global__ void __launch_bounds__(kThreads, (BM * BN >= 128 * 128) ? LP_SIMT_MIN
 #pragma unroll
           for (int j = 0; j < UN; ++j) acc[i][j] = mac(a[i], b[j], acc[i][j]);
       }
-      if (kt + 1 < nk) sstore(buf ^ 1);
+      if constexpr (kAsync) {
+        asm volatile("cp.async.wait_all;" ::: "memory");
+      } else {
+        if (kt + 1 < nk) sstore(buf ^ 1);
+      }
       __syncthreads();
     }
 
