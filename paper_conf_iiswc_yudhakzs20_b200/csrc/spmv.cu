@@ -51,6 +51,12 @@ constexpr int kSpWarps = kSpThreads / 32;
 #ifndef LP_SPMV_EARLY
 #define LP_SPMV_EARLY 0
 #endif
+// element -> thread mapping of the product phase: 0 = each thread owns 4 consecutive elements per 16-B vector
+// (lanes 4 elements apart: a warp's x gather touches ~32 lines of the banded x); 1 = element s*256 + tid
+// (lanes on consecutive elements: ~8 lines per gather).  The shared product chunk, hence every sum, is the same.
+#ifndef LP_SPMV_SCALAR
+#define LP_SPMV_SCALAR 1
+#endif
 constexpr int kPerThread = LP_SPMV_PT;               // nnz per thread per chunk (kPerThread / 4 uint4)
 constexpr int kVec = kPerThread / 4;
 constexpr int kChunk = kSpThreads * kPerThread;      // nnz per chunk
@@ -92,6 +98,24 @@ __device__ __forceinline__ void load_chunk(const float* __restrict__ val, const 
   }
 }
 
+__device__ __forceinline__ uint32_t ld_nc_u32(const void* p) {
+  uint32_t r;
+  asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+
+// Element kc + s * kSpThreads + tid of the chunk into slot s (0 outside [K0, K1)).
+__device__ __forceinline__ void load_chunk_s(const float* __restrict__ val, const int32_t* __restrict__ col, int64_t kc,
+                                             int64_t K0, int64_t K1, uint32_t* va, uint32_t* ca) {
+#pragma unroll
+  for (int s = 0; s < kPerThread; ++s) {
+    const int64_t k = kc + (int64_t)s * kSpThreads + threadIdx.x;
+    const bool in = k >= K0 && k < K1;
+    va[s] = in ? ld_nc_u32(val + k) : 0u;
+    ca[s] = in ? ld_nc_u32(col + k) : 0u;
+  }
+}
+
 template <uint32_t MASK, int STORE, bool SEQ>
 __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const int64_t* __restrict__ row_ptr,
                                                           const int32_t* __restrict__ col,
@@ -120,8 +144,13 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
     if (tid == 0) s_ra = 0;
     const int64_t kbase = K0 & ~(int64_t)3;
     const int nch = (int)((K1 - kbase + kChunk - 1) / kChunk);
+#if LP_SPMV_SCALAR
+    uint32_t va[kPerThread], ca[kPerThread];
+    if (nch > 0) load_chunk_s(val, col, kbase, K0, K1, va, ca);
+#else
     uint4 v[kVec], c[kVec];
     if (nch > 0) load_chunk(val, col, kbase, K0, K1, nnz, v, c);
+#endif
     __syncthreads();
     for (int ch = 0; ch < nch; ++ch) {
       const int64_t kc = kbase + (int64_t)ch * kChunk;
@@ -135,6 +164,13 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
       // products of this thread's kPerThread elements (the x gathers are independent of each other);
       // masked lanes (value 0, column 0) read x[0] and store 0, never summed
       float xv[kPerThread];
+#if LP_SPMV_SCALAR
+#pragma unroll
+      for (int e = 0; e < kPerThread; ++e) xv[e] = __ldg(x + (ca[e] < (uint64_t)n ? ca[e] : 0u));
+#pragma unroll
+      for (int e = 0; e < kPerThread; ++e) pb[e * kSpThreads + tid] = __fmul_rn(__uint_as_float(va[e]), xv[e]);
+      if (ch + 1 < nch) load_chunk_s(val, col, kc + kChunk, K0, K1, va, ca);
+#else
 #pragma unroll
       for (int h = 0; h < kVec; ++h) {
         const uint32_t c4[4] = {c[h].x, c[h].y, c[h].z, c[h].w};
@@ -153,7 +189,8 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
 #if !LP_SPMV_EARLY
       // the next chunk's loads fly while this one is reduced
       if (ch + 1 < nch) load_chunk(val, col, kc + kChunk, K0, K1, nnz, v, c);
-#else
+#endif
+#if LP_SPMV_EARLY && !LP_SPMV_SCALAR
       if (ch + 1 < nch) {
 #pragma unroll
         for (int h = 0; h < kVec; ++h) {
@@ -162,6 +199,7 @@ __global__ void __launch_bounds__(kSpThreads, LP_SPMV_MINB) spmv_kernel(const in
         }
       }
 #endif
+#endif  // LP_SPMV_SCALAR
       __syncthreads();
       // row phase: rows overlapping [lo, hi) (offsets relative to K0).  A row's products in this
       // chunk are summed in CSR order by its thread when there are <= kLong of them; longer
