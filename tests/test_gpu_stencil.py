@@ -142,3 +142,18 @@ def test_stencil_row_shard(shard):
     torch.cuda.synchronize()
     assert int(d_n.item()) == 0
     assert np.array_equal(dev_to_host(out).view(np.uint32), golden.view(np.uint32))
+
+
+@pytest.mark.parametrize("frac", [0.0, 1.0])
+def test_stencil_recover_none_and_all(frac):
+    """Degenerate crash sets for the TMA-fed list-mode recovery: no failed region (an empty list: every
+    persistent CTA exits at once) and every region failed (the list is the whole table)."""
+    nf = stencil_cycle(640, 512, "uniform", "mod|xor", "stale_region", frac)
+    assert nf == round(frac * (640 // 128) * (512 // 128))
+
+
+def test_stencil_tma_list_more_regions_than_ctas_per_sm_ring():
+    """More failed regions than 3 ring stages x #SM, with a region count not a multiple of the grid: every CTA
+    wraps its stage ring several times and the last CTAs take one region fewer."""
+    nf = stencil_cycle(128 * 30, 128 * 23, "int17", "mod|xor|adler", "stale_region", 0.9)
+    assert nf == round(0.9 * 30 * 23)
