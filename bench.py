@@ -152,6 +152,9 @@ def parse():
     ap.add_argument("--nvls-count", action="store_true",
                     help="N>1 over NCCL: all-reduce the failed count inside lp_validate through an NVSwitch multicast "
                          "counter (multimem.red, lp_attach_nvls_count) instead of an NCCL all-reduce")
+    ap.add_argument("--split-revalidate", action="store_true",
+                    help="re-validate the regions the first validate did not flag beside the recovery (side stream) "
+                         "and the failed list after it, instead of a full validate after the recovery -- A/B switch")
     ap.add_argument("--no-graph", dest="graph", action="store_false",
                     help="launch the step eagerly instead of replaying captured CUDA graphs")
     return ap.parse_args()
@@ -451,7 +454,15 @@ def run_ours(args):
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[0:1].copy_(nvls_buf[4:5] if nvls_buf is not None else d_n)
 
+    # recovery, then the re-validation of the whole output (lp_recover + lp_validate).  --split-revalidate: the
+    # regions the first validate did not flag are re-validated on liblp's side stream beside the recovery and the
+    # failed list after it (lp_recover_revalidate; array store) -- measured slower, an A/B switch
+    split_reval = (W["store"] == "array" and h.mask != 0 and nvls_buf is None and args.split_revalidate)
+
     def seg_recover():
+        if split_reval:
+            h.recover_revalidate(wl, out, ck, failed, d_n, ws, counts[2:3], d_n_recovered=counts[1:2])
+            return
         h.recover(wl, out, ck, failed, d_n, ws, d_n_recovered=counts[1:2])
         h.validate(wl, out, ck, failed, d_n, ws)
         counts[2:3].copy_(nvls_buf[4:5] if nvls_buf is not None else d_n)
@@ -778,6 +789,9 @@ def run_ours(args):
                        "cksum": W["cksum"], "store": W["store"], "inject_frac": W["frac"],
                        "reduction": "sequential smem (no shuffle)" if args.no_shuffle else "redux.sync + block combine",
                        "recovery": recovery_desc(args, RM, W),
+                       "revalidate": ("whole output: unflagged regions on a side stream beside the recovery, the failed "
+                                      "list after it (lp_recover_revalidate)" if split_reval else
+                                      "whole output after the recovery (lp_validate)"),
                        "inject_mode": "stale_words", "regions_per_rank": R, "parallelism": f"region-row dp{world}",
                        "l2": "flushed (2x L2 write, then 2x L2 read of another buffer: clean lines) before every recovery phase and every isolated kernel rep",
                        "launch": "CUDA graph replay per step segment" if args.graph else "eager"},

@@ -140,9 +140,11 @@ typedef enum {
                                        instead of 128, so entries reach the stash and the rehash (L270) runs */
   LP_FLAG_NVLS_COUNT = 64u, /* allow lp_attach_nvls_count: lp_validate all-reduces the failed count through an
                               NVSwitch multicast counter (multimem.red) from the CTA that finalises it */
-  LP_FLAG_RECOVER_SLICES128 = 128u /* tcgen05 bf16 recovery of 128x128 regions: two 128x64 slices per failed region,
+  LP_FLAG_RECOVER_SLICES128 = 128u, /* tcgen05 bf16 recovery of 128x128 regions: two 128x64 slices per failed region,
                                       grouped 1-4 per task (finer load balance; the two slice partial records are
                                       combined across tasks) instead of same-row pairs of 128x128 tiles (A/B switch) */
+  LP_FLAG_TEST_SKIP_REEXEC = 256u /* test hook: lp_recover_revalidate skips the re-execution, so the re-validation
+                                     of the failed list must count every listed region */
 } lp_config_flags;
 
 typedef struct {
@@ -242,6 +244,25 @@ LP_API lp_status lp_recover(lp_handle h, const lp_workload_t* wl, void* out, voi
 LP_API lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
                                   const int64_t* failed_list, const int64_t* d_n_failed, void* workspace,
                                   int64_t* d_n_recovered, lp_stream_t stream);
+
+/* Recovery followed by the re-validation of the whole output (steps a10 + a11), with the re-validation split
+ * so that most of it overlaps the recovery: the regions the PREVIOUS lp_validate on this workspace did not
+ * flag (its per-region flags are read from `workspace`, which must be that call's, untouched since) are
+ * re-validated on a liblp-owned side stream while `stream` re-executes the flagged ones (lp_recover_count);
+ * after both, the regions of failed_list are re-validated.  Recovery writes only the listed regions' data
+ * and array-table records, so the unflagged regions' bytes and records are not written while they are read.
+ * *d_n_after (device int64, zeroed by the call) = regions whose record still mismatches (0 after a
+ * successful recovery); no failed list is produced (call lp_validate for one if it is not 0).
+ * *d_n_recovered as in lp_recover_count (may be NULL).  Work and result equal lp_recover_count +
+ * lp_validate; stream-ordered on `stream` (the side stream is forked from and joined back into it with
+ * events, so the call may be captured into a CUDA graph).  Array store with cfg.cksum != 0 only
+ * (hash-store inserts can move other keys): LP_ERR_UNSUPPORTED otherwise.
+ * Measured on B200 (bench --split-revalidate): not faster than lp_recover_count + lp_validate for the
+ * C2 TMM (0.136 vs 0.128 ms) or the C4 stencil (1.57 vs 1.43 ms) -- the concurrent re-validation contends
+ * with the recovery for the L2->SM fabric / DRAM -- so the bench's default path stays sequential. */
+LP_API lp_status lp_recover_revalidate(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
+                                       const int64_t* failed_list, const int64_t* d_n_failed, void* workspace,
+                                       int64_t* d_n_after, int64_t* d_n_recovered, lp_stream_t stream);
 
 /* The paper's own recovery form (Listing 7; NEXT row N2): ONE kernel
  * with the grid of the original kernel, in which every CTA validates its regions

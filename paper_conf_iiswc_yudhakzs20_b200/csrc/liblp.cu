@@ -26,6 +26,10 @@ struct lp_ctx {
   int dev_checked;  // 0 = not yet, 1 = ok
   int sm_count;
   lp::NvlsCount nvls;  // NVLS-fused failed count (lp_attach_nvls_count); mc == nullptr: off
+  // lp_recover_revalidate: a side stream for the re-validation of the unflagged regions + fork / join events
+  // (created on first use on cfg.device, destroyed by lp_destroy)
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
 };
 
 namespace {
@@ -442,7 +446,7 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
   if (cfg->device < 0) return fail(LP_ERR_INVALID_ARG, "negative device");
   if (cfg->flags & ~(uint32_t)(LP_FLAG_TC_1CTA | LP_FLAG_NO_SHUFFLE | LP_FLAG_NO_PAIRING | LP_FLAG_NO_FUSED_COMPACT |
                                  LP_FLAG_RECOVER_TILE128 | LP_FLAG_CUCKOO_SHORT_CHAINS | LP_FLAG_NVLS_COUNT |
-                                 LP_FLAG_RECOVER_SLICES128))
+                                 LP_FLAG_RECOVER_SLICES128 | LP_FLAG_TEST_SKIP_REEXEC))
     return fail(LP_ERR_INVALID_ARG, "unknown flags 0x%x", cfg->flags);
   if ((cfg->flags & LP_FLAG_NO_SHUFFLE) && (cfg->body == LP_BODY_TCGEN05 || cfg->cksum != (LP_CK_MOD | LP_CK_XOR)))
     return fail(LP_ERR_UNSUPPORTED, "the no-shuffle ablation is built for the SIMT TMM and SPMV bodies with MOD|XOR");
@@ -460,6 +464,15 @@ lp_status lp_config(const lp_config_t* cfg, lp_handle* out) {
 }
 
 lp_status lp_destroy(lp_handle h) {
+  if (h && h->side) {
+    int prev = 0;
+    cudaGetDevice(&prev);
+    cudaSetDevice(h->cfg.device);
+    cudaEventDestroy(h->ev_fork);
+    cudaEventDestroy(h->ev_join);
+    cudaStreamDestroy(h->side);
+    cudaSetDevice(prev);
+  }
   delete h;
   return ok();
 }
@@ -568,6 +581,51 @@ lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void
   if ((s = run_body(h, wl, g, out, cksum, failed_list, d_n_failed, (cudaStream_t)stream, workspace, d_n_recovered)))
     return s;
   return cuckoo_rehash(h, cksum, (cudaStream_t)stream);
+}
+
+lp_status lp_recover_revalidate(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
+                                const int64_t* failed_list, const int64_t* d_n_failed, void* workspace,
+                                int64_t* d_n_after, int64_t* d_n_recovered, lp_stream_t stream) {
+  lp::RegionGeom g;
+  lp_status s = check_wl(h, wl, &g);
+  if (s) return s;
+  if (!out || !cksum || !failed_list || !d_n_failed || !workspace || !d_n_after)
+    return fail(LP_ERR_INVALID_ARG, "null argument");
+  if (h->mask == 0 || h->cfg.store != LP_STORE_ARRAY)
+    return fail(LP_ERR_UNSUPPORTED, "recover + split re-validation needs checksums in the array store (hash-store "
+                                    "inserts move other entries: use lp_recover then lp_validate)");
+  if (!aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
+  if ((s = check_device(h))) return s;
+  DeviceGuard dg(h->cfg.device);
+  cudaError_t e = cudaSuccess;
+  if (!h->side) {
+    // the side stream gets the LOWEST priority: the recovery's CTAs (a persistent grid that needs whole SMs)
+    // are dispatched first, the re-validation fills the SMs and cycles they leave
+    int lo_prio = 0, hi_prio = 0;
+    cudaDeviceGetStreamPriorityRange(&lo_prio, &hi_prio);
+    if ((e = cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, lo_prio)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&h->ev_fork, cudaEventDisableTiming)) != cudaSuccess ||
+        (e = cudaEventCreateWithFlags(&h->ev_join, cudaEventDisableTiming)) != cudaSuccess)
+      return cuda_fail(e, "side stream / events");
+  }
+  cudaStream_t st = (cudaStream_t)stream;
+  const WsLayout w = ws_layout(g);
+  const uint8_t* flags = (const uint8_t*)workspace + w.flags;   // the previous lp_validate's per-region flags
+  unsigned long long* cnt = reinterpret_cast<unsigned long long*>(d_n_after);
+  if ((e = cudaMemsetAsync(d_n_after, 0, sizeof(int64_t), st)) != cudaSuccess) return cuda_fail(e, "memset");
+  // fork: the unflagged regions are re-validated on the side stream while the main stream recovers the flagged
+  // ones (the recovery is submitted first; the side stream depends only on the work before the fork)
+  if ((e = cudaEventRecord(h->ev_fork, st)) != cudaSuccess || (e = cudaStreamWaitEvent(h->side, h->ev_fork, 0)) != cudaSuccess)
+    return cuda_fail(e, "fork");
+  if (!(h->cfg.flags & LP_FLAG_TEST_SKIP_REEXEC) &&
+      (s = run_body(h, wl, g, out, cksum, failed_list, d_n_failed, st, workspace, d_n_recovered)))
+    return s;
+  if ((e = lp::launch_validate_skip_count(g, h->mask, out, cksum, flags, cnt, h->sm_count, h->side)) != cudaSuccess)
+    return cuda_fail(e, "re-validate (unflagged regions)");
+  if ((e = cudaEventRecord(h->ev_join, h->side)) != cudaSuccess) return cuda_fail(e, "join record");
+  if ((e = cudaStreamWaitEvent(st, h->ev_join, 0)) != cudaSuccess) return cuda_fail(e, "join");
+  e = lp::launch_validate_list_count(g, h->mask, out, cksum, failed_list, d_n_failed, cnt, h->sm_count, st);
+  return e == cudaSuccess ? ok() : cuda_fail(e, "re-validate (recovered regions)");
 }
 
 lp_status lp_check_recover(lp_handle h, const lp_workload_t* wl, void* out, void* cksum, int64_t* d_n_recovered,

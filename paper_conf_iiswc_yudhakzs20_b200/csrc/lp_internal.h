@@ -34,6 +34,14 @@ cudaError_t launch_cksum_init(void* ck, size_t bytes, const HashInfo& hi, cudaSt
 // itself (1 launch); otherwise a PDL scatter launch follows (2 launches).
 // records != null => records mode (no compare, no compaction).
 constexpr int64_t kFusedCompactMaxR = 16384;
+// re-validation split around a recovery (array table): regions not flagged by the previous validate (beside the
+// recovery) and the failed list (after it); mismatches are added to *d_count
+cudaError_t launch_validate_skip_count(const RegionGeom& g, uint32_t mask, const void* out, const void* ck,
+                                       const uint8_t* flags, unsigned long long* d_count, int sm_count,
+                                       cudaStream_t st);
+cudaError_t launch_validate_list_count(const RegionGeom& g, uint32_t mask, const void* out, const void* ck,
+                                       const int64_t* list, const int64_t* d_n, unsigned long long* d_count,
+                                       int sm_count, cudaStream_t st);
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,
                             uint8_t* flags, uint32_t* records, int sm_count, cudaStream_t st, uint32_t* counts,
                             int64_t* list, int64_t* d_n, uint32_t* ticket = nullptr,

@@ -127,7 +127,10 @@ __device__ __forceinline__ void fused_compact_if_last(const uint8_t* flags, int6
 // 256-512 B contiguous segments.  Each CTA owns a contiguous range of regions and
 // writes its failure count for the ordered compaction.
 // MODE 0 = compare with array table, 1 = compare with a quad hash table (lookup
-// by global rid), 2 = write records (no compare), 3 = compare with a cuckoo table.
+// by global rid), 2 = write records (no compare), 3 = compare with a cuckoo table,
+// 4 = count-only re-validation of the regions NOT flagged by the previous validate
+// (flags read as the skip mask, mismatches added to *(u64*)d_n; array table) --
+// runs beside the recovery of the flagged ones (lp_recover_revalidate).
 template <uint32_t MASK, int MODE, int MB = 4>
 __global__ void __launch_bounds__(kValThreads, MB) validate_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
                                                                 int64_t Q, int64_t R, int RM, int row_bytes,
@@ -157,7 +160,7 @@ __global__ void __launch_bounds__(kValThreads, MB) validate_kernel(const uint8_t
   const int64_t r1 = r0 + rpc < R ? r0 + rpc : R;
   for (int64_t t0 = r0 + (int64_t)warp * G; t0 < r1; t0 += (int64_t)kValWarps * G) {
     const int64_t r = t0 + gi;
-    const bool live = r < r1;
+    const bool live = r < r1 && (MODE != 4 || !flags[r]);
     const int64_t p = r / Q, q = r - p * Q;
     const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
     CkPartial<MASK> part;
@@ -218,7 +221,7 @@ __global__ void __launch_bounds__(kValThreads, MB) validate_kernel(const uint8_t
         for (int s = 0; s < S; ++s) records[r * S + s] = w[s];
       } else {
         bool bad = false;
-        if constexpr (MODE == 0) {
+        if constexpr (MODE == 0 || MODE == 4) {
 #pragma unroll
           for (int s = 0; s < S; ++s) bad |= (ck[r * S + s] != w[s]);
         } else {
@@ -228,12 +231,16 @@ __global__ void __launch_bounds__(kValThreads, MB) validate_kernel(const uint8_t
 #pragma unroll
           for (int s = 0; s < S; ++s) bad |= (!bad && stored[s] != w[s]);
         }
-        flags[r] = bad ? 1 : 0;
-        if (bad) atomicAdd(&s_fail, 1u);
+        if constexpr (MODE == 4) {
+          if (bad) atomicAdd(reinterpret_cast<unsigned long long*>(d_n), 1ull);
+        } else {
+          flags[r] = bad ? 1 : 0;
+          if (bad) atomicAdd(&s_fail, 1u);
+        }
       }
     }
   }
-  if constexpr (MODE != 2) {
+  if constexpr (MODE != 2 && MODE != 4) {
     __syncthreads();
     if (threadIdx.x == 0) cta_counts[blockIdx.x] = s_fail;
     if (ticket) fused_compact_if_last(flags, R, rid_offset, ticket, list, d_n, nv);
@@ -264,6 +271,7 @@ cudaError_t validate_dispatch_mode(int mode, int mb, const ValLaunch& L, cudaStr
       LP_VLAUNCH1(MD, 4);                \
   } while (0)
   if (mode == 0) LP_VLAUNCH(0);
+  else if (mode == 4) LP_VLAUNCH(4);
   else if (mode == 1) LP_VLAUNCH(1);
   else if (mode == 3) LP_VLAUNCH(3);
   else LP_VLAUNCH(2);
@@ -848,6 +856,110 @@ static ValLaunch plan_validate(const RegionGeom& g, int sm_count) {
 size_t validate_counts_bytes(const RegionGeom& g, int sm_count) {
   (void)g;
   return (size_t)sm_count * 16 * sizeof(uint32_t) + 256;
+}
+
+// Re-validation split around a recovery (lp_recover_revalidate; array table): the regions the previous validate
+// did NOT flag are re-validated beside the recovery (MODE 4: flags = skip mask, mismatches counted), the flagged
+// ones -- the failed list -- after it, one warp per region.  Together: every region of the final state checked.
+cudaError_t launch_validate_skip_count(const RegionGeom& g, uint32_t mask, const void* out, const void* ck,
+                                       const uint8_t* flags, unsigned long long* d_count, int sm_count,
+                                       cudaStream_t st) {
+  const int row_bytes = g.RN * g.es;
+  const int cpr = row_bytes / 16;
+  int cpr_log2 = 0;
+  while ((1 << cpr_log2) < cpr) ++cpr_log2;
+  const ValLaunch L = plan_validate(g, sm_count);
+  const int mb = ((mask & kAdler) != 0 && (uint64_t)g.R * (uint64_t)g.RM * (uint64_t)row_bytes >= val_adler_big_bytes())
+                     ? LP_VAL_ADLER_MINB : 4;
+  const NvlsCount nv{nullptr, nullptr, 1};
+  const uint8_t* o = (const uint8_t*)out;
+  const int64_t ldcb = g.ldc * g.es;
+  cudaError_t e;
+  switch (mask) {
+#define LP_VCASE(M)                                                                                          \
+  case M:                                                                                                    \
+    e = validate_dispatch_mode<M>(4, mb, L, st, o, ldcb, g.Q, g.R, g.RM, row_bytes, cpr_log2,                   \
+                                  (const uint32_t*)ck, g.rid_offset, const_cast<uint8_t*>(flags), nullptr,      \
+                                  nullptr, nullptr, nullptr, reinterpret_cast<int64_t*>(d_count), nv);          \
+    break;
+    LP_VCASE(1)
+    LP_VCASE(2)
+    LP_VCASE(3)
+    LP_VCASE(4)
+    LP_VCASE(5)
+    LP_VCASE(6)
+    LP_VCASE(7)
+#undef LP_VCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return e;
+}
+
+namespace {
+// One warp per listed region (global rid list[i]): record of the stored words vs the array table entry;
+// mismatches added to *d_count.
+template <uint32_t MASK>
+__global__ void __launch_bounds__(256) validate_list_count_kernel(const uint8_t* __restrict__ out, int64_t ldc_bytes,
+                                                                  int64_t Q, int RM, int row_bytes, int cpr_log2,
+                                                                  const uint32_t* __restrict__ ck, int64_t rid_offset,
+                                                                  const int64_t* __restrict__ list,
+                                                                  const int64_t* __restrict__ d_n,
+                                                                  unsigned long long* __restrict__ d_count) {
+  constexpr int S = selem_of(MASK);
+  const int lane = threadIdx.x & 31;
+  const int64_t n = *d_n;
+  const int chunks = RM << cpr_log2, cmask = (1 << cpr_log2) - 1;
+  const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+  for (int64_t i = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < n; i += warps) {
+    const int64_t r = list[i] - rid_offset, p = r / Q, q = r - p * Q;
+    const uint8_t* base = out + p * (int64_t)RM * ldc_bytes + q * (int64_t)row_bytes;
+    CkPartial<MASK> part;
+    for (int c = lane; c < chunks; c += 32) {
+      const uint4 v = ld_stream_u4(base + (int64_t)(c >> cpr_log2) * ldc_bytes + ((c & cmask) << 4));
+      part.add4(v.x, v.y, v.z, v.w, (uint32_t)((c >> cpr_log2) * row_bytes + ((c & cmask) << 4) + 1));
+    }
+    const CkRecord rec = warp_reduce<MASK>(part);
+    if (lane == 0) {
+      uint32_t w[3];
+      record_words<MASK>(rec, (uint64_t)RM * (uint64_t)row_bytes, w);
+      bool bad = false;
+#pragma unroll
+      for (int s2 = 0; s2 < S; ++s2) bad |= (ck[r * S + s2] != w[s2]);
+      if (bad) atomicAdd(d_count, 1ull);
+    }
+  }
+}
+}  // namespace
+
+cudaError_t launch_validate_list_count(const RegionGeom& g, uint32_t mask, const void* out, const void* ck,
+                                       const int64_t* list, const int64_t* d_n, unsigned long long* d_count,
+                                       int sm_count, cudaStream_t st) {
+  const int row_bytes = g.RN * g.es;
+  const int cpr = row_bytes / 16;
+  int cpr_log2 = 0;
+  while ((1 << cpr_log2) < cpr) ++cpr_log2;
+  const unsigned grid = (unsigned)(sm_count * 8);
+  const uint8_t* o = (const uint8_t*)out;
+  const int64_t ldcb = g.ldc * g.es;
+  switch (mask) {
+#define LP_LVCASE(M)                                                                                            \
+  case M:                                                                                                       \
+    validate_list_count_kernel<M><<<grid, 256, 0, st>>>(o, ldcb, g.Q, g.RM, row_bytes, cpr_log2,                 \
+                                                        (const uint32_t*)ck, g.rid_offset, list, d_n, d_count); \
+    break;
+    LP_LVCASE(1)
+    LP_LVCASE(2)
+    LP_LVCASE(3)
+    LP_LVCASE(4)
+    LP_LVCASE(5)
+    LP_LVCASE(6)
+    LP_LVCASE(7)
+#undef LP_LVCASE
+    default:
+      return cudaErrorInvalidValue;
+  }
+  return cudaGetLastError();
 }
 
 cudaError_t launch_validate(const RegionGeom& g, uint32_t mask, const HashInfo& hi, const void* out, const void* ck,

@@ -34,6 +34,7 @@ FLAG_RECOVER_TILE128 = 16
 FLAG_CUCKOO_SHORT_CHAINS = 32
 FLAG_NVLS_COUNT = 64
 FLAG_RECOVER_SLICES128 = 128
+FLAG_TEST_SKIP_REEXEC = 256
 INJ_STALE_WORDS, INJ_STALE_REGION, INJ_BITFLIP, INJ_STALE_RECORD = 0, 1, 2, 3
 
 CK_NAMES = {"none": 0, "mod": 1, "xor": 2, "adler": 4, "adler32": 4}
@@ -43,7 +44,8 @@ INJ_NAMES = {"stale_words": 0, "stale_region": 1, "bitflip": 2, "stale_record": 
 EXPORTED = ["lp_config", "lp_destroy", "lp_num_regions", "lp_cksum_bytes", "lp_workspace_bytes", "lp_cksum_init",
             "lp_run_protected", "lp_validate", "lp_recover", "lp_region_checksums", "lp_inject", "lp_stats",
             "lp_device_sm_count", "lp_last_error", "lp_abi_version", "lp_fn_study", "lp_check_recover",
-            "lp_attach_nvls_count", "lp_recover_count", "lp_check_recover_ws"]
+            "lp_attach_nvls_count", "lp_recover_count", "lp_check_recover_ws",
+            "lp_recover_revalidate"]
 
 
 def parse_cksum(spec) -> int:
@@ -104,6 +106,7 @@ def lib():
             "lp_validate": [P, pw, P, P, P, I64, P, P, P],
             "lp_recover": [P, pw, P, P, P, P, P, P],
             "lp_recover_count": [P, pw, P, P, P, P, P, P, P],
+            "lp_recover_revalidate": [P, pw, P, P, P, P, P, P, P, P],
             "lp_region_checksums": [P, pw, P, P, P],
             "lp_inject": [P, pw, P, P, P, P, I64, U32, U64, P],
             "lp_stats": [P, pw, P, P, P],
@@ -232,7 +235,7 @@ class LP:
                  body="auto", hash_seed: int = 0x9747B28C,
                  tc_pair: bool = True, shuffle: bool = True, pairing: bool = True, fused_compact: bool = True,
                  recover_slices: bool = True, cuckoo_short_chains: bool = False, nvls_count: bool = False,
-                 recover_slices128: bool = False):
+                 recover_slices128: bool = False, test_skip_reexec: bool = False):
         self.mask = parse_cksum(cksum)
         self.store = STORE_NAMES[store] if isinstance(store, str) else int(store)
         self.body = BODY_NAMES[body] if isinstance(body, str) else int(body)
@@ -244,7 +247,8 @@ class LP:
                           (0 if recover_slices else FLAG_RECOVER_TILE128) |
                           (FLAG_CUCKOO_SHORT_CHAINS if cuckoo_short_chains else 0) |
                           (FLAG_NVLS_COUNT if nvls_count else 0) |
-                          (FLAG_RECOVER_SLICES128 if recover_slices128 else 0))
+                          (FLAG_RECOVER_SLICES128 if recover_slices128 else 0) |
+                          (FLAG_TEST_SKIP_REEXEC if test_skip_reexec else 0))
         h = ctypes.c_void_p()
         _check(lib().lp_config(ctypes.byref(self.cfg), ctypes.byref(h)))
         self._h = h
@@ -297,6 +301,12 @@ class LP:
         else:
             _check(lib().lp_recover_count(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed),
                                           _ptr(d_n), _ptr(workspace), _ptr(d_n_recovered), _stream(stream)))
+
+    def recover_revalidate(self, wl, out, ck, failed, d_n, workspace, d_n_after, d_n_recovered=None, stream=None):
+        """lp_recover_revalidate: recover the failed list and re-validate the whole output, the unflagged regions
+        on a side stream beside the recovery; *d_n_after (device int64[1]) = regions still mismatching."""
+        _check(lib().lp_recover_revalidate(self._h, ctypes.byref(wl.c()), _ptr(out), _ptr(ck), _ptr(failed), _ptr(d_n),
+                                           _ptr(workspace), _ptr(d_n_after), _ptr(d_n_recovered), _stream(stream)))
 
     def check_recover(self, wl, out, ck, d_n_recovered, workspace=None, stream=None):
         """Listing 7's same-grid check-and-recover (N2): validate + in-place re-execution in one kernel; with a
