@@ -256,7 +256,9 @@ LP_API lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* ou
  * *d_n_recovered as in lp_recover_count (may be NULL).  Work and result equal lp_recover_count +
  * lp_validate; stream-ordered on `stream` (the side stream is forked from and joined back into it with
  * events, so the call may be captured into a CUDA graph).  Array store with cfg.cksum != 0 only
- * (hash-store inserts can move other keys): LP_ERR_UNSUPPORTED otherwise.
+ * (hash-store inserts can move other keys), and only where the recovery writes exactly the listed regions:
+ * the stencil, SpMV, the SIMT TMM and the tcgen05 bf16 TMM with 128x128 regions (the tensor-core bodies
+ * with smaller regions rewrite whole recovery tiles); LP_ERR_UNSUPPORTED otherwise.
  * Measured on B200 (bench --split-revalidate): not faster than lp_recover_count + lp_validate for the
  * C2 TMM (0.136 vs 0.128 ms) or the C4 stencil (1.57 vs 1.43 ms) -- the concurrent re-validation contends
  * with the recovery for the L2->SM fabric / DRAM -- so the bench's default path stays sequential. */

@@ -583,6 +583,24 @@ lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* out, void
   return cuckoo_rehash(h, cksum, (cudaStream_t)stream);
 }
 
+// True when the list-mode recovery writes exactly the listed regions (and their records): stencil, SpMV, the SIMT
+// TMM, and the tcgen05 bf16 TMM with 128x128 regions (tile = region).  The tcgen05 bodies with regions smaller
+// than their recovery tile (bf16 32x32 in 128x64 slices, fp32 3xTF32 in 256x256 tiles) also rewrite the clean
+// regions sharing a tile (identical bits), which a re-validation running beside the recovery would race.
+bool recovery_writes_only_listed(const lp_ctx* h, const lp_workload_t* wl, const lp::RegionGeom& g, const void* out) {
+  if (wl->kind != LP_WL_TMM) return true;
+  const bool i32 = wl->in_dtype == LP_I32, in_bf16 = wl->in_dtype == LP_BF16, out_bf16 = wl->out_dtype == LP_BF16;
+  const bool tc_ok = lp::tmm_tc_supported(wl->m, wl->n, wl->k, g.RM, g.RN, in_bf16, wl->lda, wl->ldb, wl->ldc, wl->a,
+                                          wl->b, out);
+  const bool tf_ok = !i32 && lp::tmm_tf32_supported(wl->m, wl->n, wl->k, g.RM, g.RN, in_bf16, out_bf16, wl->lda,
+                                                     wl->ldb, wl->ldc, wl->a, wl->b, out);
+  const bool no_shuffle = (h->cfg.flags & LP_FLAG_NO_SHUFFLE) != 0;
+  int body = h->cfg.body;
+  if (body == LP_BODY_AUTO) body = (tc_ok || tf_ok) && !no_shuffle ? LP_BODY_TCGEN05 : LP_BODY_SIMT;
+  if (body != LP_BODY_TCGEN05) return true;
+  return tc_ok && g.RM == 128 && g.RN == 128;
+}
+
 lp_status lp_recover_revalidate(lp_handle h, const lp_workload_t* wl, void* out, void* cksum,
                                 const int64_t* failed_list, const int64_t* d_n_failed, void* workspace,
                                 int64_t* d_n_after, int64_t* d_n_recovered, lp_stream_t stream) {
@@ -595,6 +613,9 @@ lp_status lp_recover_revalidate(lp_handle h, const lp_workload_t* wl, void* out,
     return fail(LP_ERR_UNSUPPORTED, "recover + split re-validation needs checksums in the array store (hash-store "
                                     "inserts move other entries: use lp_recover then lp_validate)");
   if (!aligned16(workspace)) return fail(LP_ERR_INVALID_ARG, "workspace must be 16-B aligned");
+  if (!recovery_writes_only_listed(h, wl, g, out))
+    return fail(LP_ERR_UNSUPPORTED, "this body's recovery rewrites whole tensor-core tiles (regions smaller than the "
+                                    "tile): use lp_recover then lp_validate");
   if ((s = check_device(h))) return s;
   DeviceGuard dg(h->cfg.device);
   cudaError_t e = cudaSuccess;
