@@ -255,7 +255,8 @@ LP_API lp_status lp_recover_count(lp_handle h, const lp_workload_t* wl, void* ou
  * successful recovery); no failed list is produced (call lp_validate for one if it is not 0).
  * *d_n_recovered as in lp_recover_count (may be NULL).  Work and result equal lp_recover_count +
  * lp_validate; stream-ordered on `stream` (the side stream is forked from and joined back into it with
- * events, so the call may be captured into a CUDA graph).  Array store with cfg.cksum != 0 only
+ * events, so the call may be captured into a CUDA graph; the side stream and events belong to the handle, so
+ * concurrent lp_recover_revalidate calls on ONE handle from several host threads are not supported).  Array store with cfg.cksum != 0 only
  * (hash-store inserts can move other keys), and only where the recovery writes exactly the listed regions:
  * the stencil, SpMV, the SIMT TMM and the tcgen05 bf16 TMM with 128x128 regions (the tensor-core bodies
  * with smaller regions rewrite whole recovery tiles); LP_ERR_UNSUPPORTED otherwise.
