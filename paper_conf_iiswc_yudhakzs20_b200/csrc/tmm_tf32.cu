@@ -38,7 +38,13 @@ namespace {
 
 constexpr int kFBK = 32;                          // 32 fp32 = 128 B = one swizzle-atom row
 constexpr int kFUmmaK = 8;                        // K per tcgen05.mma kind::tf32
-constexpr int kFRawStages = 3;                    // TMA ring
+#ifndef LP_TF32_RAW_HI  // the MMA reads A's hi part straight from the raw TMA stage (see below)
+#define LP_TF32_RAW_HI 1
+#endif
+// kind::tf32 ignores the low 13 mantissa bits of its 32-bit operands (measured: raw fp32 words as the hi operand
+// give bit-identical products to x & 0xFFFFE000 -- tools/probe/tf32_raw_hi.sh), so with LP_TF32_RAW_HI the
+// converters write only A_lo, B_hi, B_lo and the MMA takes A_hi from the raw ring, which it then releases too.
+constexpr int kFRawStages = LP_TF32_RAW_HI ? 4 : 3;   // TMA ring
 constexpr int kFCvStages = 2;                     // converted ring
 #ifndef LP_TF32_CONV_WARPS
 #define LP_TF32_CONV_WARPS 8
@@ -46,13 +52,18 @@ constexpr int kFCvStages = 2;                     // converted ring
 #ifndef LP_TF32_BLOOP
 #define LP_TF32_BLOOP 0
 #endif
+#ifndef LP_TF32_RAW_HI_PROBE  // probe build: does kind::tf32 ignore the low 13 mantissa bits of its operands?
+#define LP_TF32_RAW_HI_PROBE 0
+#endif
 constexpr int kFConvWarps = LP_TF32_CONV_WARPS;   // converter warps per CTA (4: one column of B per thread)
 constexpr int kFConvThreads = kFConvWarps * 32;
 constexpr int kFConvWarp0 = 6;
 constexpr int kFThreads = (kFConvWarp0 + kFConvWarps) * 32;  // TMA, MMA, 4 epilogue, converter warps
 constexpr int kFTile = 16384;                     // one 128 x 32 fp32 operand tile
 constexpr int kFRawBytes = 2 * kFTile;            // raw stage: [A (K-major)][B (MN-major, 4 x 32-col chunks)]
-constexpr int kFCvBytes = 4 * kFTile;             // converted stage: [A_hi][A_lo][B_hi][B_lo], all K-major SW128
+// converted stage: [A_hi][A_lo][B_hi][B_lo] (or [A_lo][B_hi][B_lo] with LP_TF32_RAW_HI), all K-major SW128
+constexpr int kFCvBytes = (LP_TF32_RAW_HI ? 3 : 4) * kFTile;
+constexpr int kFCvALo = LP_TF32_RAW_HI ? 0 : kFTile, kFCvBHi = kFCvALo + kFTile, kFCvBLo = kFCvBHi + kFTile;
 constexpr int kFSmemBytes = kFRawStages * kFRawBytes + kFCvStages * kFCvBytes + 512 + 1024;
 // K is accumulated in chunks of kFChunkKB x 32 = 512 in one TMEM accumulator (columns
 // 0..255); after each chunk the epilogue warps fold it into a TMEM-resident running
@@ -127,7 +138,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
     prefetch_tmap(&tmap_b);
     for (int s = 0; s < kFRawStages; ++s) {
       mbar_init(&raw_full[s], 1);   // this CTA's TMA bytes
-      mbar_init(&raw_empty[s], kFConvWarps);  // this CTA's converter warps
+      mbar_init(&raw_empty[s], kFConvWarps + (LP_TF32_RAW_HI ? 1 : 0));  // converter warps (+ the MMA commit)
     }
     for (int s = 0; s < kFCvStages; ++s) {
       mbar_init(&cv_full[s], 2 * kFConvWarps);  // converter warps x 2 CTAs (used in rank 0)
@@ -199,8 +210,12 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
           lo.y = __fsub_rn(x.y, hi.y);
           lo.z = __fsub_rn(x.z, hi.z);
           lo.w = __fsub_rn(x.w, hi.w);
+#if LP_TF32_RAW_HI_PROBE
+          *reinterpret_cast<float4*>(cv + i * 16) = x;  // probe: the MMA reads the raw fp32 word as its tf32 hi
+#elif !LP_TF32_RAW_HI
           *reinterpret_cast<float4*>(cv + i * 16) = hi;
-          *reinterpret_cast<float4*>(cv + kFTile + i * 16) = lo;
+#endif
+          *reinterpret_cast<float4*>(cv + kFCvALo + i * 16) = lo;
         }
         // B: raw MN-major (chunk c = n/32 holds 32 K-rows x 32 columns, 16-B unit u of
         // row k stored at u ^ (k & 7)) -> K-major SW128 rows n (K quad j at j ^ (n & 7)).
@@ -221,8 +236,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
             const int n = u & 127, j = u >> 7, c = n >> 5, l = n & 31;
 #endif
             const uint8_t* rb = r + kFTile + c * (kFBK * 128) + (l & 3) * 4;
-            uint8_t* bhi = cv + 2 * kFTile + n * 128;
-            uint8_t* blo = cv + 3 * kFTile + n * 128;
+            uint8_t* bhi = cv + kFCvBHi + n * 128;
+            uint8_t* blo = cv + kFCvBLo + n * 128;
             float xv[4];
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
@@ -239,7 +254,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
             lo.z = __fsub_rn(xv[2], hi.z);
             lo.w = __fsub_rn(xv[3], hi.w);
             const int off = ((j ^ (n & 7)) << 4);
+#if LP_TF32_RAW_HI_PROBE
+            *reinterpret_cast<float4*>(bhi + off) = make_float4(xv[0], xv[1], xv[2], xv[3]);
+#else
             *reinterpret_cast<float4*>(bhi + off) = hi;
+#endif
             *reinterpret_cast<float4*>(blo + off) = lo;
           }
         }
@@ -268,7 +287,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
       // kind::tf32, D fp32, A and B both K-major, M = 256 (cta_group::2), N = 256
       constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | (0u << 15) | (0u << 16) |
                                  ((uint32_t)(256 >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
-      int stage = 0;
+      int stage = 0, rstage = 0;
       uint32_t phase = 0;
       uint32_t acc_phase = 0;
       for (int64_t t = pair; t < ntiles; t += npairs) {
@@ -280,7 +299,9 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
           for (int kb = kb0; kb < kb1; ++kb) {
             mbar_wait(&cv_full[stage], phase);
             tc_fence_after();
-            const uint32_t ah = smem_u32(cvs(stage)), al = ah + kFTile, bh = ah + 2 * kFTile, bl = ah + 3 * kFTile;
+            const uint32_t cvb = smem_u32(cvs(stage));
+            const uint32_t ah = LP_TF32_RAW_HI ? smem_u32(raw(rstage)) : cvb;  // raw A tile: K-major SW128 too
+            const uint32_t al = cvb + kFCvALo, bh = cvb + kFCvBHi, bl = cvb + kFCvBLo;
 #pragma unroll
             for (int k = 0; k < kFBK / kFUmmaK; ++k) {
               const uint64_t dah = smem_desc(ah + k * kFUmmaK * 4, 16, 1024);
@@ -292,6 +313,8 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kFThreads, 1)
               tc_mma_pair_tf32(d_tmem, dal, dbh, idesc, 1u);
             }
             tc_commit_pair(&cv_empty[stage]);
+            if (LP_TF32_RAW_HI) tc_commit_pair(&raw_empty[rstage]);   // the raw A tile is free once these MMAs ran
+            if (++rstage == kFRawStages) rstage = 0;
             if (++stage == kFCvStages) {
               stage = 0;
               phase ^= 1;
