@@ -80,6 +80,32 @@ __device__ __forceinline__ void add4_modxor(CkPartial<MASK>& p, uint32_t x, uint
   if constexpr ((MASK & kXor) != 0) p.xr ^= x ^ y ^ z ^ v;
 }
 
+// output stores of the LDG form: the two-phase protected kernels store with .cg (cache at L2), the plain twin
+// with evict-first .cs -- each its faster flavour (profiles/r02/ab_stencil_st.txt: Adler 1.330 -> 1.314 ms with
+// .cg, the twin 1.300 with .cs vs 1.304-1.308); LP_STENCIL_ST=1..3 force one flavour everywhere (A/B runs)
+#ifndef LP_STENCIL_ST
+#define LP_STENCIL_ST 0
+#endif
+template <bool CG>
+__device__ __forceinline__ void st_out(float4* p, float4 o) {
+#if LP_STENCIL_ST == 0
+  if constexpr (CG) {
+    asm volatile("st.global.cg.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w) : "memory");
+  } else {
+    __stcs(p, o);
+  }
+#elif LP_STENCIL_ST == 1
+  *p = o;  // plain (write-back)
+#elif LP_STENCIL_ST == 2
+  asm volatile("st.global.cg.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w) : "memory");
+#elif LP_STENCIL_ST == 3
+  asm volatile("st.global.L1::no_allocate.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "f"(o.x), "f"(o.y), "f"(o.z), "f"(o.w)
+               : "memory");
+#else
+  __stcs(p, o);
+#endif
+}
+
 __device__ __forceinline__ float4 ldg_nc_v4(const float* p) {
   float4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
@@ -201,7 +227,7 @@ __global__ void __launch_bounds__(kRM / RWS * 32, 2) stencil5_ldg_kernel(const f
       o.y = st5(c.y, u.y, d.y, c.x, c.z);
       o.z = st5(c.z, u.z, d.z, c.y, c.w);
       o.w = st5(c.w, u.w, d.w, c.z, right);
-      __stcs(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
+      st_out<kTwoPhase>(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
       if constexpr (kTwoPhase) {
         v[r] = o;  // row r's input is dead: keep the stored vector for the checksum pass below
       } else if constexpr (MASK != 0) {
