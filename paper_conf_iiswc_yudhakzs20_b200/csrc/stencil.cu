@@ -86,6 +86,9 @@ __device__ __forceinline__ void add4_modxor(CkPartial<MASK>& p, uint32_t x, uint
 #ifndef LP_STENCIL_ST
 #define LP_STENCIL_ST 0
 #endif
+#ifndef LP_STENCIL_TMA_ST_CG  // TMA-fed form (list-mode recovery): .cg instead of .cs output stores
+#define LP_STENCIL_TMA_ST_CG 0
+#endif
 template <bool CG>
 __device__ __forceinline__ void st_out(float4* p, float4 o) {
 #if LP_STENCIL_ST == 0
@@ -437,7 +440,11 @@ __global__ void __launch_bounds__((NW + 1) * 32, 1)
       o.y = st5(c.y, u.y, d.y, c.x, c.z);
       o.z = st5(c.z, u.z, d.z, c.y, c.w);
       o.w = st5(c.w, u.w, d.w, c.z, right);
+#if LP_STENCIL_TMA_ST_CG
+      st_out<true>(reinterpret_cast<float4*>(orow + (int64_t)r * ldo), o);
+#else
       __stcs(reinterpret_cast<float4*>(orow + (int64_t)r * ldo), o);
+#endif
       if constexpr (MASK != 0) {
         add4_modxor(part, __float_as_uint(o.x), __float_as_uint(o.y), __float_as_uint(o.z), __float_as_uint(o.w));
         if constexpr ((MASK & kAdler) != 0)
