@@ -80,9 +80,10 @@ __device__ __forceinline__ void add4_modxor(CkPartial<MASK>& p, uint32_t x, uint
   if constexpr ((MASK & kXor) != 0) p.xr ^= x ^ y ^ z ^ v;
 }
 
-// output stores of the LDG form: the two-phase protected kernels store with .cg (cache at L2), the plain twin
-// with evict-first .cs -- each its faster flavour (profiles/r02/ab_stencil_st.txt: Adler 1.330 -> 1.314 ms with
-// .cg, the twin 1.300 with .cs vs 1.304-1.308); LP_STENCIL_ST=1..3 force one flavour everywhere (A/B runs)
+// output stores of the LDG form: the two-phase protected kernels with Adler in the record store with .cg (cache
+// at L2), the others (MOD / XOR, and the plain twin) with evict-first .cs -- each its faster flavour
+// (profiles/r02/ab_stencil_st.txt: Adler 1.330 -> 1.314 ms with .cg; the twin 1.300 with .cs vs 1.304-1.308;
+// MOD|XOR equal); LP_STENCIL_ST=1..3 force one flavour everywhere (A/B runs)
 #ifndef LP_STENCIL_ST
 #define LP_STENCIL_ST 0
 #endif
@@ -230,7 +231,7 @@ __global__ void __launch_bounds__(kRM / RWS * 32, 2) stencil5_ldg_kernel(const f
       o.y = st5(c.y, u.y, d.y, c.x, c.z);
       o.z = st5(c.z, u.z, d.z, c.y, c.w);
       o.w = st5(c.w, u.w, d.w, c.z, right);
-      st_out<kTwoPhase>(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
+      st_out<kTwoPhase && (MASK & kAdler) != 0>(reinterpret_cast<float4*>(out + (int64_t)(i0 + r) * ldo + j), o);
       if constexpr (kTwoPhase) {
         v[r] = o;  // row r's input is dead: keep the stored vector for the checksum pass below
       } else if constexpr (MASK != 0) {
