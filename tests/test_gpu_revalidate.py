@@ -115,3 +115,34 @@ def test_hash_store_is_refused():
     after = torch.zeros(1, dtype=torch.int64, device="cuda")
     with pytest.raises(lp.LPError):
         h.recover_revalidate(wl, out, ck, failed, d_n, ws, after)
+
+
+def test_recover_revalidate_in_a_cuda_graph():
+    """The side stream is forked from and joined into the caller's stream with events, so the call can be captured
+    into a CUDA graph (bench.py replays its step segments as graphs): replay on a freshly crashed state."""
+    h, wl, out, ck, failed, d_n, ws, stale = _setup("stencil", "mod|xor", 128)
+    golden = dev_to_host(out)
+    R = h.num_regions(wl)
+    inj = torch.from_numpy(lp.choose_regions(R, 0.25, 15)).cuda()
+    after = torch.full((1,), -1, dtype=torch.int64, device="cuda")
+    h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=15)
+    h.validate(wl, out, ck, failed, d_n, ws)
+    h.recover_revalidate(wl, out, ck, failed, d_n, ws, after)        # eager warm-up (creates the side stream)
+    torch.cuda.synchronize()
+    assert int(after.item()) == 0
+    g = torch.cuda.CUDAGraph()
+    s = torch.cuda.Stream()
+    s.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(s):
+        with torch.cuda.graph(g, stream=s, capture_error_mode="thread_local"):
+            h.validate(wl, out, ck, failed, d_n, ws)
+            h.recover_revalidate(wl, out, ck, failed, d_n, ws, after)
+    torch.cuda.synchronize()
+    for _ in range(2):
+        after.fill_(-1)
+        h.inject(wl, out, ck, stale, inj, mode="stale_region", seed=15)
+        torch.cuda.synchronize()
+        g.replay()
+        torch.cuda.synchronize()
+        assert int(d_n.item()) == inj.numel() and int(after.item()) == 0
+        assert np.array_equal(dev_to_host(out).view(np.uint32), golden.view(np.uint32))
