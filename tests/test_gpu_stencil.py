@@ -157,3 +157,17 @@ def test_stencil_tma_list_more_regions_than_ctas_per_sm_ring():
     wraps its stage ring several times and the last CTAs take one region fewer."""
     nf = stencil_cycle(128 * 30, 128 * 23, "int17", "mod|xor|adler", "stale_region", 0.9)
     assert nf == round(0.9 * 30 * 23)
+
+
+@pytest.mark.parametrize("case", range(12))
+def test_stencil_fuzz_shapes(case):
+    """Seeded random shapes (1..9 region rows, 1..7 region columns, incl. single-region domains), checksum sets,
+    stores, crash modes and fractions through the full-run body and the TMA-fed list recovery."""
+    rng = np.random.default_rng(1000 + case)
+    H, W = 128 * int(rng.integers(1, 10)), 128 * int(rng.integers(1, 8))
+    store = str(rng.choice(["array", "array", "quad_cas", "cuckoo"]))
+    mask = str(rng.choice(["mod", "xor", "mod|xor", "adler", "mod|xor|adler"])) if store == "array" else "mod|xor"
+    mode = str(rng.choice(["stale_words", "stale_region", "bitflip"]))
+    frac = float(rng.choice([0.0, 0.3, 1.0]))
+    kind = str(rng.choice(["uniform", "int17"]))
+    stencil_cycle(H, W, kind, mask, mode, frac, seed=3 + case, store=store)

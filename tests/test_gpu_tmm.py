@@ -497,3 +497,19 @@ def test_tc4_matches_tc2_bits():
         outs.append(out)
     torch.cuda.synchronize()
     assert torch.equal(outs[0].view(torch.int32), torch.cat([outs[1], outs[2]]).view(torch.int32))
+
+
+@pytest.mark.parametrize("case", range(8))
+def test_simt_fuzz_shapes(case):
+    """Seeded random SIMT shapes with 32x32 regions: M, N multiples of 128 (16-region tiles) or of 32 only (one CTA
+    per region), int32 / fp32 / bf16, checksum sets and stores, through body, validate and per-region recovery."""
+    rng = np.random.default_rng(2000 + case)
+    tile = bool(rng.integers(0, 2))
+    M = int(rng.integers(1, 4)) * (128 if tile else 96)
+    N = int(rng.integers(1, 4)) * (128 if tile else 160)
+    K = 16 * int(rng.integers(1, 9))
+    in_dt, out_dt, kind = [("i32", "i32", "int17"), ("f32", "f32", "uniform"), ("bf16", "f32", "int5")][case % 3]
+    store = str(rng.choice(["array", "array", "quad_cas", "cuckoo"]))
+    mask = str(rng.choice(["mod", "mod|xor", "xor|adler", "mod|xor|adler"])) if store == "array" else "mod|xor"
+    run_cycle(M, N, K, 32, 32, in_dt, out_dt, kind, mask, "simt", store=store, frac=float(rng.choice([0.1, 0.5])),
+              seed=5 + case)
