@@ -513,3 +513,15 @@ def test_simt_fuzz_shapes(case):
     mask = str(rng.choice(["mod", "mod|xor", "xor|adler", "mod|xor|adler"])) if store == "array" else "mod|xor"
     run_cycle(M, N, K, 32, 32, in_dt, out_dt, kind, mask, "simt", store=store, frac=float(rng.choice([0.1, 0.5])),
               seed=5 + case)
+
+
+@pytest.mark.parametrize("case", range(6))
+def test_tf32x3_fuzz_shapes(case):
+    """Seeded random 3xTF32 shapes (M, N multiples of 256, K multiples of 32 across the 512-K chunk boundaries):
+    A's hi operand read raw from the TMA stage must stay within 1e-5 of the fp64 oracle (it would not if the tensor
+    core rounded instead of truncating the low mantissa bits) and integer-valued inputs bit-exact."""
+    rng = np.random.default_rng(3000 + case)
+    M, N = 256 * int(rng.integers(1, 4)), 256 * int(rng.integers(1, 4))
+    K = 32 * int(rng.integers(1, 40))
+    kind = "uniform" if case % 2 == 0 else "int5"
+    run_cycle(M, N, K, 128, 128, "f32", "f32", kind, "mod|xor", "tcgen05", frac=0.25, seed=7 + case)
